@@ -1,0 +1,123 @@
+// ddt_internal.h -- host-side internals of libddt (types, layout cache, queue).
+#pragma once
+#include <atomic>
+#include <cstdint>
+#include <map>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/ddt.h"
+#include "device_desc.h"
+
+namespace ddt {
+
+// ---------------------------------------------------------------- errors
+void set_error(const std::string& msg);
+const char* last_error();
+ddt_status_t cuda_fail(const char* what, int cuda_err);
+
+// ---------------------------------------------------------------- types
+enum TypeKind { T_BASIC, T_CONTIG, T_VECTOR, T_HVECTOR, T_INDEXED, T_HINDEXED, T_SUBARRAY };
+
+// A closed-form strided description of the typemap's contiguous segments:
+// segment (i_0..i_{D-1}) (outermost first, typemap order = row-major over the
+// dims) is at  base + sum_d i_d * dims[d].stride  and has seg_len bytes.
+struct Dim {
+    int64_t n, stride;
+};
+struct Form {
+    int64_t base = 0;
+    int64_t seg_len = 0;
+    std::vector<Dim> dims;  // outermost first
+    int64_t num_segments() const;
+};
+// Drop unit dims, merge dims whose strides chain, fold contiguous inner dims
+// into the segment.  Returns false for an empty form (some n == 0 or len 0).
+bool normalize(Form& f);
+
+struct Seg {
+    int64_t off, len;
+};
+
+// Per-device copy of list-layout metadata (the device-resident layout cache).
+struct DeviceLayout {
+    void* offsets = nullptr;  // u32 or i64
+    void* lens = nullptr;     // i64 (general)
+    void* prefix = nullptr;   // i64 (general)
+};
+
+struct Layout {
+    int32_t kind = DDT_LAYOUT_EMPTY;
+    int64_t nseg = 0;          // segments per instance
+    int64_t seg_len = 0;       // strided / uniform
+    Form form;                 // strided (dims <= kMaxDims)
+    bool off32 = false;        // uniform: offsets fit in int32
+    std::vector<int64_t> offsets, lens, prefix;  // lists (host copy)
+    int align = 16;            // power of two <= 16 dividing every offset & length
+    bool overlaps = false;
+};
+
+struct ddt_type_impl;
+}  // namespace ddt
+
+struct ddt_type_s {
+    int kind;
+    int base = -1;
+    bool predefined = false;
+    int64_t elem = 0;
+    int64_t count = 0, blocklen = 0, stride = 0;   // contig / vector / hvector (stride in bytes for hvector)
+    std::vector<int64_t> blocklens, displs;       // indexed / hindexed
+    int ndims = 0, order = 0;
+    std::vector<int64_t> sizes, subsizes, starts;
+    ddt_type_s* old = nullptr;
+    std::atomic<int64_t> refs{1};
+
+    // closed-form properties (computed at construction)
+    bool nonempty = false;
+    int64_t size = 0, lb = 0, ub = 0, true_lb = 0, true_ub = 0;
+    bool has_form = false;
+    ddt::Form form;  // normalized strided form if derivable (any number of dims)
+
+    // committed layout
+    std::mutex mu;
+    bool committed = false;
+    ddt::Layout layout;
+    std::map<int, ddt::DeviceLayout> dev;  // device ordinal -> device cache
+};
+
+namespace ddt {
+void type_retain(ddt_type_s* t);
+void type_release(ddt_type_s* t);
+// Upload list metadata to `device` if needed (caller has set the device).
+ddt_status_t type_device_layout(ddt_type_s* t, int device, DeviceLayout** out);
+inline int64_t type_extent(const ddt_type_s* t) { return t->ub - t->lb; }
+
+// ------------------------------------------------------------ kernels
+// Builds the u32 reciprocal for DivU32.
+DivU32 make_div(uint32_t d);
+// Fill a descriptor for one request; returns DDT_OK or an error.
+ddt_status_t build_desc(ddt_type_s* t, const DeviceLayout* dl, int op, const void* noncontig,
+                        const void* packed, int64_t count, ReqDesc* out);
+// Items of a descriptor.
+inline uint32_t desc_items(const ReqDesc& d) {
+    return (uint32_t)((d.nvec + (uint64_t)kItemVecs - 1) / (uint64_t)kItemVecs);
+}
+// Launch the fused kernel over a device batch table.  grid_cap <= 0 => default.
+int launch_fused(const void* dev_table, uint32_t total_items, void* stream, int grid_cap);
+int device_sm_count(int device);
+int launch_exchange(const void* dev_table, uint32_t total_items, void* ctrl, int* err_flag_dev, uint64_t timeout_ns,
+                    void* stream, int grid_cap);
+size_t table_bytes(size_t nreq);
+uint32_t write_table(void* dst, const ReqDesc* descs, size_t nreq);
+
+// queue accessors (queue.cpp)
+int queue_device(ddt_queue_s* q);
+void* queue_stream(ddt_queue_s* q);
+int queue_sm_count(ddt_queue_s* q);
+ddt_status_t queue_sticky(ddt_queue_s* q);
+void queue_set_sticky(ddt_queue_s* q, ddt_status_t s);
+void queue_count_launches(ddt_queue_s* q, int64_t launches, int64_t bytes);
+ddt_status_t nccl_fail(const char* what, int r);
+
+}  // namespace ddt

@@ -1,0 +1,78 @@
+// device_desc.h -- the device-side request descriptor and batch table.
+//
+// One descriptor = one request of the paper's request list (§IV-A.1 P:189-197:
+// UID, operation, origin/target buffer, cached layout entry) flattened into the
+// closed-form / list parameters the fused kernel needs.  A batch table = the
+// "array of requests" handed to the single fused kernel plus the work
+// table built by an exclusive prefix sum over per-request item counts (SURVEY
+// §8(a) a4), which maps every CTA work item to a (request, vector range) pair.
+#pragma once
+#include <stdint.h>
+
+namespace ddt {
+
+constexpr int kMaxDims = 4;          // closed-form strided dims per layout (R7)
+constexpr int kThreads = 256;        // threads per CTA of the fused kernel
+constexpr int kUnroll = 4;           // vectors per thread per item (loads in flight)
+constexpr int kItemVecs = kThreads * kUnroll;  // vectors per work item
+
+enum DescOp : uint8_t { OP_PACK = 0, OP_UNPACK = 1 };
+enum DescKind : uint8_t { K_STRIDED = 0, K_UNIFORM32 = 1, K_UNIFORM64 = 2, K_GENERAL = 3 };
+
+// Unsigned 32-bit division by a runtime constant d via a 64-bit reciprocal:
+// q = umulhi64(n, ceil(2^64 / d)) is exact for n, d < 2^32 (error < 1/d);
+// d == 1 is flagged by magic == 0.
+struct DivU32 {
+    uint32_t d;
+    uint32_t pad;
+    uint64_t magic;
+};
+
+struct alignas(16) ReqDesc {
+    uint64_t noncontig;     // non-contiguous side (pack: source, unpack: destination)
+    uint64_t packed;        // contiguous side     (pack: destination, unpack: source)
+    uint32_t nvec;          // vectors in the request (count*size / w), < 2^32
+    uint8_t op;             // DescOp
+    uint8_t kind;           // DescKind
+    uint8_t lw;             // log2 of the vector width w in bytes (0..4)
+    uint8_t ndim;           // strided dims (innermost first), K_STRIDED only
+    DivU32 vps;             // vectors per segment (uniform kinds) / per instance (general)
+    int64_t base;           // byte offset of segment 0 of instance 0 (strided)
+    int64_t extent;         // byte stride between instances (count)
+    DivU32 nseg;            // segments per instance (uniform lists)
+    DivU32 radix[kMaxDims]; // strided: dim sizes, innermost first
+    int64_t stride[kMaxDims];
+    uint64_t list;          // device pointer: offsets (u32 / i64) for lists
+    uint64_t lens;          // general: int64 lengths
+    uint64_t prefix;        // general: int64 exclusive packed prefix (nseg + 1 entries)
+    uint32_t list_n;        // general: number of segments per instance
+    uint32_t uid_lo;        // low bits of the request UID (debug / tracing)
+};
+
+// Header of a batch table in device memory:
+//   BatchHeader | uint32 item_prefix[nreq + 1] (padded to 16 B) | ReqDesc[nreq]
+struct alignas(16) BatchHeader {
+    uint32_t nreq;
+    uint32_t total_items;
+    uint32_t desc_offset;   // byte offset of ReqDesc[0] from the header
+    uint32_t pad;
+};
+
+// Exchange-only side info of a descriptor (fused P2P halo kernel).
+struct alignas(16) XInfo {
+    uint64_t flag;          // pack: peer's flag slot; unpack: own flag slot (u64 epoch)
+    uint32_t counter;       // pack: index of the per-message completion counter
+    uint32_t nitems;        // pack: items of the message (counter target = epoch * nitems)
+    int64_t parity_stride;  // window half size: iteration e uses half (e & 1)
+    int64_t pad;
+};
+
+// Control block of the fused exchange kernel (device memory, zeroed at create).
+struct XCtrl {
+    unsigned int ticket;          // next work item (reset by the last CTA to exit)
+    unsigned int done;            // CTAs finished
+    unsigned long long epoch;     // completed exchanges
+    unsigned long long counters[1];  // [nsend] monotonic per-message item counters
+};
+
+}  // namespace ddt

@@ -1,0 +1,633 @@
+// halo.cpp -- persistent halo-exchange plans (ddt_halo_create / ddt_exchange).
+//
+// Paper: Alg 3 -- one MPI_Isend / MPI_Irecv per boundary buffer,
+// the runtime packs and unpacks implicitly; §IV-B -- the sender
+// enqueues packing and sends once a pack completes, the receiver
+// enqueues unpacking on arrival, and pack, unpack and DirectIPC may be
+// fused into one kernel.  Domain decomposition (Fig. 3) is the
+// only parallelism in the paper.
+//
+// B200 realisation:
+//   NCCL mode: fused pack launch (all outgoing messages, per-peer contiguous
+//     staging ordered by tag; self messages straight into the receive staging)
+//     -> ncclGroupStart / {ncclSend, ncclRecv} per remote peer / ncclGroupEnd
+//     over NVLink 5 -> fused unpack launch.  Work tables are built once here.
+//   P2P mode: ONE kernel: pack stores go straight into the peer's window
+//     (CUDA IPC mapping, NVSwitch), a per-message epoch flag is released when
+//     the message is complete, unpack work waits on its flag (see
+//     fused_kernel.cu).  Windows are double-buffered by iteration parity;
+//     this requires a symmetric pattern (every peer we send to sends to us),
+//     which is checked here.
+//   Both: a one-time metadata exchange over NCCL validates that every send
+//   matches the peer's receive of the same tag and size (DDT_ERR_SIZE_MISMATCH)
+//   and tells each sender where its messages land; iterations can be replayed
+//   from a CUDA graph captured on first use.
+#include <algorithm>
+#include <cstring>
+#include <map>
+#include <tuple>
+#include <vector>
+
+#include <cuda_runtime.h>
+
+#include "ddt_internal.h"
+#include "nccl_min.h"
+
+using namespace ddt;
+
+namespace {
+
+constexpr int64_t kAlign = 16;
+
+int64_t round_up(int64_t v, int64_t a) { return (v + a - 1) / a * a; }
+
+// Receive-side layout shared by the window (P2P) and the receive staging (NCCL).
+struct RecvLayout {
+    std::vector<int> order;          // recv indices sorted by (peer, tag)
+    std::vector<int64_t> data_off;   // per recv index: offset inside one parity half
+    std::vector<int> flag_idx;       // per recv index
+    int64_t flags_bytes = 0, parity_stride = 0, window_bytes = 0;
+};
+
+RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs) {
+    RecvLayout L;
+    L.order.resize((size_t)nrecv);
+    for (int i = 0; i < nrecv; i++) L.order[(size_t)i] = i;
+    std::sort(L.order.begin(), L.order.end(), [&](int a, int b) {
+        return std::make_pair(recvs[a].peer, recvs[a].tag) < std::make_pair(recvs[b].peer, recvs[b].tag);
+    });
+    L.data_off.assign((size_t)nrecv, 0);
+    L.flag_idx.assign((size_t)nrecv, 0);
+    int64_t off = 0;
+    for (size_t k = 0; k < L.order.size(); k++) {
+        int i = L.order[k];
+        int64_t bytes = recvs[i].count * recvs[i].type->size;
+        off = round_up(off, kAlign);
+        L.data_off[(size_t)i] = off;
+        L.flag_idx[(size_t)i] = (int)k;
+        off += bytes;
+    }
+    L.flags_bytes = round_up(std::max<int64_t>(8 * (int64_t)nrecv, 8), 256);
+    L.parity_stride = round_up(std::max<int64_t>(off, 16), 256);
+    L.window_bytes = L.flags_bytes + 2 * L.parity_stride;
+    return L;
+}
+
+struct DirEntry {
+    int64_t tag, bytes, data_off, flag_idx;
+};
+struct Directory {  // what a receiver tells one sender
+    int64_t parity_stride = 0, data_base = 0;
+    std::vector<DirEntry> e;  // sorted by tag
+};
+
+struct Xfer {
+    int peer;
+    int64_t send_off, send_bytes;  // in send staging
+    int64_t recv_off, recv_bytes;  // in receive staging
+};
+
+}  // namespace
+
+struct ddt_halo_s {
+    ddt_queue_s* q = nullptr;
+    int device = 0;
+    cudaStream_t stream = nullptr;
+    int rank = 0, nranks = 1, mode = DDT_XCHG_NCCL;
+    void* comm = nullptr;
+    std::vector<ddt_send_t> sends;
+    std::vector<ddt_recv_t> recvs;
+    // NCCL mode
+    void* send_stage = nullptr;
+    void* recv_stage = nullptr;
+    std::vector<Xfer> xfers;
+    void* pack_table = nullptr;
+    uint32_t pack_items = 0;
+    void* unpack_table = nullptr;
+    uint32_t unpack_items = 0;
+    // P2P mode
+    void* xtable = nullptr;
+    uint32_t xitems = 0;
+    void* ctrl = nullptr;
+    int* err_host = nullptr;
+    int* err_dev = nullptr;
+    uint64_t timeout_ns = 10ull * 1000 * 1000 * 1000;
+    int grid_cap = 0;
+    // graph replay
+    bool use_graph = false;
+    cudaGraphExec_t gexec = nullptr;
+    int32_t launches = 0;
+    int64_t bytes = 0;
+};
+
+namespace {
+
+struct DevGuard {
+    int prev = -1;
+    explicit DevGuard(int d) {
+        cudaGetDevice(&prev);
+        if (prev != d) cudaSetDevice(d);
+    }
+    ~DevGuard() {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+ddt_status_t upload(const std::vector<uint8_t>& host, void** dev) {
+    cudaError_t e = cudaMalloc(dev, std::max<size_t>(host.size(), 16));
+    if (e != cudaSuccess) return cuda_fail("cudaMalloc(halo)", e);
+    e = cudaMemcpy(*dev, host.data(), host.size(), cudaMemcpyHostToDevice);
+    if (e != cudaSuccess) return cuda_fail("cudaMemcpy(halo)", e);
+    return DDT_OK;
+}
+
+ddt_status_t make_table(const std::vector<ReqDesc>& d, void** dev, uint32_t* items) {
+    std::vector<uint8_t> host(table_bytes(d.size()));
+    *items = write_table(host.data(), d.data(), d.size());
+    return upload(host, dev);
+}
+
+// Exchange every receiver->sender directory over NCCL (nranks > 1), then agree
+// on a status with an all-reduce(min) so that all ranks fail or succeed together.
+ddt_status_t exchange_directories(ddt_halo_s* h, const std::vector<std::vector<int64_t>>& out,
+                                  std::vector<std::vector<int64_t>>& in) {
+    const NcclApi* n = nccl();
+    if (!n) {
+        set_error("NCCL not available for the halo metadata exchange");
+        return DDT_ERR_UNSUPPORTED;
+    }
+    int P = h->nranks;
+    in.assign((size_t)P, {});
+    std::vector<int64_t> cnt_out((size_t)P, 0), cnt_in((size_t)P, 0);
+    for (int p = 0; p < P; p++) cnt_out[(size_t)p] = (int64_t)out[(size_t)p].size();
+    int64_t* d_cnt = nullptr;
+    cudaError_t e = cudaMalloc(&d_cnt, 2 * sizeof(int64_t) * (size_t)P);
+    if (e != cudaSuccess) return cuda_fail("cudaMalloc(meta)", e);
+    cudaMemcpy(d_cnt, cnt_out.data(), sizeof(int64_t) * (size_t)P, cudaMemcpyHostToDevice);
+    int r = n->GroupStart();
+    for (int p = 0; p < P && r == 0; p++) {
+        if (p == h->rank) continue;
+        r = n->Send(d_cnt + p, 8, kNcclUint8, p, h->comm, h->stream);
+        if (r == 0) r = n->Recv(d_cnt + P + p, 8, kNcclUint8, p, h->comm, h->stream);
+    }
+    int r2 = n->GroupEnd();
+    if (r == 0) r = r2;
+    if (r != 0) {
+        cudaFree(d_cnt);
+        return nccl_fail("halo metadata (counts)", r);
+    }
+    cudaStreamSynchronize(h->stream);
+    cudaMemcpy(cnt_in.data(), d_cnt + P, sizeof(int64_t) * (size_t)P, cudaMemcpyDeviceToHost);
+    cudaFree(d_cnt);
+    int64_t tot_out = 0, tot_in = 0;
+    for (int p = 0; p < P; p++) {
+        if (p == h->rank) continue;
+        tot_out += cnt_out[(size_t)p];
+        tot_in += cnt_in[(size_t)p];
+    }
+    int64_t* d_buf = nullptr;
+    e = cudaMalloc(&d_buf, sizeof(int64_t) * (size_t)std::max<int64_t>(tot_out + tot_in, 1));
+    if (e != cudaSuccess) return cuda_fail("cudaMalloc(meta)", e);
+    std::vector<int64_t> flat_out;
+    for (int p = 0; p < P; p++)
+        if (p != h->rank) flat_out.insert(flat_out.end(), out[(size_t)p].begin(), out[(size_t)p].end());
+    if (tot_out) cudaMemcpy(d_buf, flat_out.data(), sizeof(int64_t) * (size_t)tot_out, cudaMemcpyHostToDevice);
+    r = n->GroupStart();
+    int64_t oo = 0, io = tot_out;
+    for (int p = 0; p < P && r == 0; p++) {
+        if (p == h->rank) continue;
+        if (cnt_out[(size_t)p]) r = n->Send(d_buf + oo, (size_t)cnt_out[(size_t)p] * 8, kNcclUint8, p, h->comm, h->stream);
+        if (r == 0 && cnt_in[(size_t)p])
+            r = n->Recv(d_buf + io, (size_t)cnt_in[(size_t)p] * 8, kNcclUint8, p, h->comm, h->stream);
+        oo += cnt_out[(size_t)p];
+        io += cnt_in[(size_t)p];
+    }
+    r2 = n->GroupEnd();
+    if (r == 0) r = r2;
+    if (r != 0) {
+        cudaFree(d_buf);
+        return nccl_fail("halo metadata (directories)", r);
+    }
+    cudaStreamSynchronize(h->stream);
+    std::vector<int64_t> flat_in((size_t)tot_in);
+    if (tot_in)
+        cudaMemcpy(flat_in.data(), d_buf + tot_out, sizeof(int64_t) * (size_t)tot_in, cudaMemcpyDeviceToHost);
+    cudaFree(d_buf);
+    io = 0;
+    for (int p = 0; p < P; p++) {
+        if (p == h->rank) continue;
+        in[(size_t)p].assign(flat_in.begin() + io, flat_in.begin() + io + cnt_in[(size_t)p]);
+        io += cnt_in[(size_t)p];
+    }
+    return DDT_OK;
+}
+
+ddt_status_t agree(ddt_halo_s* h, ddt_status_t mine) {
+    if (h->nranks == 1) return mine;
+    const NcclApi* n = nccl();
+    if (!n) return DDT_ERR_UNSUPPORTED;
+    int32_t* d = nullptr;
+    if (cudaMalloc(&d, 8) != cudaSuccess) return DDT_ERR_CUDA;
+    int32_t v = mine;
+    cudaMemcpy(d, &v, 4, cudaMemcpyHostToDevice);
+    int r = n->AllReduce(d, d + 1, 1, kNcclInt32, kNcclMin, h->comm, h->stream);
+    cudaStreamSynchronize(h->stream);
+    int32_t res = DDT_OK;
+    cudaMemcpy(&res, d + 1, 4, cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    if (r != 0) return nccl_fail("halo status all-reduce", r);
+    return res;
+}
+
+Directory parse_dir(const std::vector<int64_t>& v) {
+    Directory d;
+    if (v.size() < 3) return d;
+    int64_t n = v[0];
+    d.parity_stride = v[1];
+    d.data_base = v[2];
+    for (int64_t i = 0; i < n && (size_t)(3 + 4 * i + 3) < v.size(); i++)
+        d.e.push_back({v[(size_t)(3 + 4 * i)], v[(size_t)(4 + 4 * i)], v[(size_t)(5 + 4 * i)], v[(size_t)(6 + 4 * i)]});
+    return d;
+}
+
+void free_halo(ddt_halo_s* h) {
+    if (h->gexec) cudaGraphExecDestroy(h->gexec);
+    cudaFree(h->send_stage);
+    cudaFree(h->recv_stage);
+    cudaFree(h->pack_table);
+    cudaFree(h->unpack_table);
+    cudaFree(h->xtable);
+    cudaFree(h->ctrl);
+    if (h->err_host) cudaFreeHost(h->err_host);
+    for (auto& s : h->sends) type_release(s.type);
+    for (auto& r : h->recvs) type_release(r.type);
+    delete h;
+}
+
+ddt_status_t record_exchange(ddt_halo_s* h) {
+    if (h->mode == DDT_XCHG_P2P) {
+        int e = launch_exchange(h->xtable, h->xitems, h->ctrl, h->err_dev, h->timeout_ns, h->stream, h->grid_cap);
+        if (e) return cuda_fail("exchange kernel launch", e);
+        return DDT_OK;
+    }
+    if (h->pack_items) {
+        int e = launch_fused(h->pack_table, h->pack_items, h->stream, 0);
+        if (e) return cuda_fail("pack launch", e);
+    }
+    bool remote = false;
+    for (auto& x : h->xfers) remote |= x.peer != h->rank;
+    if (remote) {
+        const NcclApi* n = nccl();
+        if (!n) return DDT_ERR_UNSUPPORTED;
+        int r = n->GroupStart();
+        for (auto& x : h->xfers) {
+            if (x.peer == h->rank || r != 0) continue;
+            if (x.send_bytes)
+                r = n->Send((char*)h->send_stage + x.send_off, (size_t)x.send_bytes, kNcclUint8, x.peer, h->comm,
+                            h->stream);
+            if (r == 0 && x.recv_bytes)
+                r = n->Recv((char*)h->recv_stage + x.recv_off, (size_t)x.recv_bytes, kNcclUint8, x.peer, h->comm,
+                            h->stream);
+        }
+        int r2 = n->GroupEnd();
+        if (r == 0) r = r2;
+        if (r != 0) return nccl_fail("halo send/recv", r);
+    }
+    if (h->unpack_items) {
+        int e = launch_fused(h->unpack_table, h->unpack_items, h->stream, 0);
+        if (e) return cuda_fail("unpack launch", e);
+    }
+    return DDT_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+ddt_status_t ddt_halo_window_bytes(int32_t nrecv, const ddt_recv_t* recvs, int64_t* bytes) {
+    if (nrecv < 0 || (nrecv > 0 && !recvs) || !bytes) return DDT_ERR_ARG;
+    for (int i = 0; i < nrecv; i++)
+        if (!recvs[i].type || recvs[i].count < 0) return DDT_ERR_ARG;
+    *bytes = layout_recvs(nrecv, recvs).window_bytes;
+    return DDT_OK;
+}
+
+ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, const ddt_send_t* sends, int32_t nrecv,
+                             const ddt_recv_t* recvs, int32_t mode, ddt_halo_t* out) {
+    if (!q || !c || !out || nsend < 0 || nrecv < 0 || (nsend && !sends) || (nrecv && !recvs)) return DDT_ERR_ARG;
+    if (mode != DDT_XCHG_NCCL && mode != DDT_XCHG_P2P) return DDT_ERR_ARG;
+    if (c->nranks < 1 || c->rank < 0 || c->rank >= c->nranks) return DDT_ERR_ARG;
+    if (c->nranks > 1 && !c->nccl_comm) return DDT_ERR_ARG;
+    if (mode == DDT_XCHG_P2P && (!c->peer_windows || c->window_bytes <= 0)) return DDT_ERR_ARG;
+    if (queue_sticky(q) != DDT_OK) return queue_sticky(q);
+    // validate messages
+    std::map<std::pair<int, int>, int> seen_s, seen_r;
+    for (int i = 0; i < nsend; i++) {
+        auto& s = sends[i];
+        if (!s.type || s.count < 0 || s.peer < 0 || s.peer >= c->nranks) return DDT_ERR_ARG;
+        if (!s.type->committed) return DDT_ERR_STATE;
+        if (s.count * s.type->size > 0 && !s.buf) return DDT_ERR_ARG;
+        if (!seen_s.emplace(std::make_pair(s.peer, s.tag), i).second) return DDT_ERR_ARG;
+    }
+    for (int i = 0; i < nrecv; i++) {
+        auto& r = recvs[i];
+        if (!r.type || r.count < 0 || r.peer < 0 || r.peer >= c->nranks) return DDT_ERR_ARG;
+        if (!r.type->committed) return DDT_ERR_STATE;
+        if (r.count * r.type->size > 0 && !r.buf) return DDT_ERR_ARG;
+        if (r.count * r.type->size > 0 && r.type->layout.overlaps) return DDT_ERR_OVERLAP;
+        if (!seen_r.emplace(std::make_pair(r.peer, r.tag), i).second) return DDT_ERR_ARG;
+    }
+    if (mode == DDT_XCHG_P2P) {  // symmetric pattern required by the parity double buffering
+        for (auto& kv : seen_s)
+            if (kv.first.first != c->rank) {
+                bool back = false;
+                for (auto& rv : seen_r) back |= rv.first.first == kv.first.first;
+                if (!back) {
+                    set_error("P2P exchange needs a symmetric pattern (send to p => receive from p)");
+                    return DDT_ERR_ARG;
+                }
+            }
+    }
+    auto* h = new (std::nothrow) ddt_halo_s();
+    if (!h) return DDT_ERR_NOMEM;
+    h->q = q;
+    h->device = queue_device(q);
+    h->stream = (cudaStream_t)queue_stream(q);
+    h->rank = c->rank;
+    h->nranks = c->nranks;
+    h->mode = mode;
+    h->comm = c->nccl_comm;
+    h->sends.assign(sends, sends + nsend);
+    h->recvs.assign(recvs, recvs + nrecv);
+    for (auto& s : h->sends) type_retain(s.type);
+    for (auto& r : h->recvs) type_retain(r.type);
+    DevGuard g(h->device);
+
+    // ---- receive layout and directories (receiver -> each sender)
+    RecvLayout RL = layout_recvs(nrecv, recvs);
+    if (mode == DDT_XCHG_P2P && c->window_bytes < RL.window_bytes) {
+        free_halo(h);
+        set_error("window smaller than ddt_halo_window_bytes()");
+        return DDT_ERR_ARG;
+    }
+    const int P = c->nranks;
+    std::vector<std::vector<int64_t>> dir_out((size_t)P), dir_in;
+    for (int p = 0; p < P; p++) {
+        std::vector<int> mine;
+        for (int k : RL.order)
+            if (recvs[k].peer == p) mine.push_back(k);
+        auto& v = dir_out[(size_t)p];
+        v = {(int64_t)mine.size(), RL.parity_stride, RL.flags_bytes};
+        for (int k : mine) {
+            v.push_back(recvs[k].tag);
+            v.push_back(recvs[k].count * recvs[k].type->size);
+            v.push_back(RL.data_off[(size_t)k]);
+            v.push_back(RL.flag_idx[(size_t)k]);
+        }
+    }
+    ddt_status_t st = DDT_OK;
+    if (P > 1) {
+        st = exchange_directories(h, dir_out, dir_in);
+        if (st != DDT_OK) {
+            free_halo(h);
+            return st;
+        }
+    } else {
+        dir_in.assign(1, {});
+    }
+    dir_in[(size_t)c->rank] = dir_out[(size_t)c->rank];
+    std::vector<Directory> dirs((size_t)P);
+    for (int p = 0; p < P; p++) dirs[(size_t)p] = parse_dir(dir_in[(size_t)p]);
+
+    // ---- match sends against the peers' directories
+    std::vector<const DirEntry*> match((size_t)nsend, nullptr);
+    for (int i = 0; i < nsend && st == DDT_OK; i++) {
+        const auto& s = sends[i];
+        const Directory& d = dirs[(size_t)s.peer];
+        for (auto& e : d.e)
+            if (e.tag == s.tag) match[(size_t)i] = &e;
+        if (!match[(size_t)i]) {
+            set_error("send without a matching receive (peer " + std::to_string(s.peer) + ", tag " +
+                      std::to_string(s.tag) + ")");
+            st = DDT_ERR_SIZE_MISMATCH;
+        } else if (match[(size_t)i]->bytes != s.count * s.type->size) {
+            set_error("send/recv size mismatch (peer " + std::to_string(s.peer) + ", tag " + std::to_string(s.tag) +
+                      ")");
+            st = DDT_ERR_SIZE_MISMATCH;
+        }
+    }
+    for (int p = 0; p < P && st == DDT_OK; p++) {  // every receive must have a send
+        size_t nsend_p = 0;
+        for (int i = 0; i < nsend; i++) nsend_p += sends[i].peer == p;
+        if (nsend_p != dirs[(size_t)p].e.size()) {
+            set_error("receive without a matching send");
+            st = DDT_ERR_SIZE_MISMATCH;
+        }
+    }
+    st = agree(h, st);
+    if (st != DDT_OK) {
+        free_halo(h);
+        return st;
+    }
+
+    // ---- build the device work tables
+    std::vector<ReqDesc> pack, unpack;
+    auto desc_for = [&](ddt_type_s* t, int op, const void* nc, const void* pk, int64_t count, ReqDesc* d) {
+        DeviceLayout* dl = nullptr;
+        ddt_status_t s2 = type_device_layout(t, h->device, &dl);
+        if (s2 != DDT_OK) return s2;
+        return build_desc(t, dl, op, nc, pk, count, d);
+    };
+    for (auto& s : h->sends) h->bytes += s.count * s.type->size;
+    if (mode == DDT_XCHG_NCCL) {
+        cudaError_t e = cudaMalloc(&h->recv_stage, (size_t)RL.parity_stride);
+        // send staging: one region per remote peer reproducing the receiver's layout
+        std::map<int, std::pair<int64_t, int64_t>> span;  // peer -> (first_off, end_off) in the peer's layout
+        for (int i = 0; i < nsend; i++) {
+            if (sends[i].peer == c->rank) continue;
+            int64_t a = match[(size_t)i]->data_off, b = a + match[(size_t)i]->bytes;
+            auto it = span.find(sends[i].peer);
+            if (it == span.end()) span[sends[i].peer] = {a, b};
+            else it->second = {std::min(it->second.first, a), std::max(it->second.second, b)};
+        }
+        std::map<int, int64_t> region;
+        int64_t soff = 0;
+        for (auto& kv : span) {
+            region[kv.first] = soff;
+            soff = round_up(soff + (kv.second.second - kv.second.first), 256);
+        }
+        if (e == cudaSuccess) e = cudaMalloc(&h->send_stage, (size_t)std::max<int64_t>(soff, 256));
+        if (e != cudaSuccess) {
+            free_halo(h);
+            return cuda_fail("cudaMalloc(staging)", e);
+        }
+        // my receive spans per peer
+        std::map<int, std::pair<int64_t, int64_t>> rspan;
+        for (int i = 0; i < nrecv; i++) {
+            int64_t a = RL.data_off[(size_t)i], b = a + recvs[i].count * recvs[i].type->size;
+            auto it = rspan.find(recvs[i].peer);
+            if (it == rspan.end()) rspan[recvs[i].peer] = {a, b};
+            else it->second = {std::min(it->second.first, a), std::max(it->second.second, b)};
+        }
+        std::map<int, Xfer> xf;
+        for (auto& kv : span) {
+            Xfer& x = xf[kv.first];
+            x.peer = kv.first;
+            x.send_off = region[kv.first];
+            x.send_bytes = kv.second.second - kv.second.first;
+        }
+        for (auto& kv : rspan) {
+            if (kv.first == c->rank) continue;
+            Xfer& x = xf[kv.first];
+            x.peer = kv.first;
+            x.recv_off = kv.second.first;
+            x.recv_bytes = kv.second.second - kv.second.first;
+        }
+        for (auto& kv : xf) h->xfers.push_back(kv.second);
+        for (int i = 0; i < nsend && st == DDT_OK; i++) {
+            const auto& s = sends[i];
+            if (s.count * s.type->size == 0) continue;
+            char* dst;
+            if (s.peer == c->rank) dst = (char*)h->recv_stage + match[(size_t)i]->data_off;
+            else dst = (char*)h->send_stage + region[s.peer] + (match[(size_t)i]->data_off - span[s.peer].first);
+            ReqDesc d;
+            st = desc_for(s.type, OP_PACK, s.buf, dst, s.count, &d);
+            pack.push_back(d);
+        }
+        for (int i = 0; i < nrecv && st == DDT_OK; i++) {
+            const auto& r = recvs[i];
+            if (r.count * r.type->size == 0) continue;
+            ReqDesc d;
+            st = desc_for(r.type, OP_UNPACK, r.buf, (char*)h->recv_stage + RL.data_off[(size_t)i], r.count, &d);
+            unpack.push_back(d);
+        }
+        if (st == DDT_OK && !pack.empty()) st = make_table(pack, &h->pack_table, &h->pack_items);
+        if (st == DDT_OK && !unpack.empty()) st = make_table(unpack, &h->unpack_table, &h->unpack_items);
+        h->launches = (pack.empty() ? 0 : 1) + (unpack.empty() ? 0 : 1);
+    } else {
+        // P2P: one table, pack descriptors first, then unpack descriptors
+        std::vector<XInfo> xi;
+        char* mywin = (char*)c->peer_windows[c->rank];
+        for (int i = 0; i < nsend && st == DDT_OK; i++) {
+            const auto& s = sends[i];
+            if (s.count * s.type->size == 0) continue;
+            const Directory& d = dirs[(size_t)s.peer];
+            char* win = (char*)c->peer_windows[s.peer];
+            ReqDesc rd;
+            st = desc_for(s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, &rd);
+            XInfo x{};
+            x.flag = (uint64_t)(uintptr_t)(win + 8 * match[(size_t)i]->flag_idx);
+            x.counter = (uint32_t)pack.size();
+            x.nitems = desc_items(rd);
+            x.parity_stride = d.parity_stride;
+            pack.push_back(rd);
+            xi.push_back(x);
+        }
+        size_t npack = pack.size();
+        for (int i = 0; i < nrecv && st == DDT_OK; i++) {
+            const auto& r = recvs[i];
+            if (r.count * r.type->size == 0) continue;
+            ReqDesc rd;
+            st = desc_for(r.type, OP_UNPACK, r.buf, mywin + RL.flags_bytes + RL.data_off[(size_t)i], r.count, &rd);
+            XInfo x{};
+            x.flag = (uint64_t)(uintptr_t)(mywin + 8 * RL.flag_idx[(size_t)i]);
+            x.parity_stride = RL.parity_stride;
+            pack.push_back(rd);
+            xi.push_back(x);
+        }
+        if (st == DDT_OK && !pack.empty()) {
+            std::vector<uint8_t> host(table_bytes(pack.size()) + xi.size() * sizeof(XInfo));
+            h->xitems = write_table(host.data(), pack.data(), pack.size());
+            std::memcpy(host.data() + table_bytes(pack.size()), xi.data(), xi.size() * sizeof(XInfo));
+            st = upload(host, &h->xtable);
+        }
+        size_t ctrl_bytes = sizeof(XCtrl) + sizeof(unsigned long long) * std::max<size_t>(npack, 1);
+        if (st == DDT_OK) {
+            cudaError_t e = cudaMalloc(&h->ctrl, ctrl_bytes);
+            if (e == cudaSuccess) e = cudaMemset(h->ctrl, 0, ctrl_bytes);
+            if (e == cudaSuccess) e = cudaHostAlloc((void**)&h->err_host, sizeof(int), cudaHostAllocMapped);
+            if (e == cudaSuccess) {
+                *h->err_host = 0;
+                e = cudaHostGetDevicePointer((void**)&h->err_dev, h->err_host, 0);
+            }
+            if (e != cudaSuccess) st = cuda_fail("exchange control block", e);
+        }
+        h->launches = pack.empty() ? 0 : 1;
+    }
+    if (st == DDT_OK) {
+        cudaError_t e = cudaDeviceSynchronize();
+        if (e != cudaSuccess) st = cuda_fail("halo create", e);
+    }
+    if (st != DDT_OK) {
+        free_halo(h);
+        return st;
+    }
+    *out = h;
+    return DDT_OK;
+}
+
+ddt_status_t ddt_halo_set_graph(ddt_halo_t h, int32_t use_graph) {
+    if (!h) return DDT_ERR_ARG;
+    h->use_graph = use_graph != 0;
+    return DDT_OK;
+}
+
+ddt_status_t ddt_exchange(ddt_halo_t h) {
+    if (!h) return DDT_ERR_ARG;
+    ddt_status_t st = queue_sticky(h->q);
+    if (st != DDT_OK) return st;
+    if (h->err_host && *(volatile int*)h->err_host) {
+        set_error("P2P exchange: a peer flag wait exceeded the timeout");
+        queue_set_sticky(h->q, DDT_ERR_TIMEOUT);
+        return DDT_ERR_TIMEOUT;
+    }
+    DevGuard g(h->device);
+    if (h->use_graph && h->stream) {
+        if (!h->gexec) {
+            cudaError_t e = cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal);
+            if (e != cudaSuccess) return cuda_fail("graph capture begin", e);
+            ddt_status_t rs = record_exchange(h);
+            cudaGraph_t graph = nullptr;
+            e = cudaStreamEndCapture(h->stream, &graph);
+            if (rs != DDT_OK) {
+                if (graph) cudaGraphDestroy(graph);
+                return rs;
+            }
+            if (e != cudaSuccess) return cuda_fail("graph capture end", e);
+            e = cudaGraphInstantiate(&h->gexec, graph, 0);
+            cudaGraphDestroy(graph);
+            if (e != cudaSuccess) return cuda_fail("graph instantiate", e);
+        }
+        cudaError_t e = cudaGraphLaunch(h->gexec, h->stream);
+        if (e != cudaSuccess) return cuda_fail("graph launch", e);
+    } else {
+        st = record_exchange(h);
+        if (st != DDT_OK) {
+            queue_set_sticky(h->q, st);
+            return st;
+        }
+    }
+    queue_count_launches(h->q, h->launches, 2 * h->bytes);
+    return DDT_OK;
+}
+
+ddt_status_t ddt_halo_launches_per_exchange(ddt_halo_t h, int32_t* launches) {
+    if (!h || !launches) return DDT_ERR_ARG;
+    *launches = h->launches;
+    return DDT_OK;
+}
+
+ddt_status_t ddt_halo_destroy(ddt_halo_t h) {
+    if (!h) return DDT_ERR_ARG;
+    {
+        DevGuard g(h->device);
+        if (h->stream) cudaStreamSynchronize(h->stream);
+        else cudaDeviceSynchronize();
+        free_halo(h);
+    }
+    return DDT_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,143 @@
+"""Halo exchange plans (Alg 3, §IV-B) and the
+communicator plumbing under them.  Marshalling only (csrc/halo.cpp,
+csrc/comm.cpp); torch.distributed is used solely to broadcast the NCCL unique
+id and to all-gather CUDA-IPC window handles."""
+from __future__ import annotations
+
+import ctypes
+
+from ._abi import (lib, check, P, ddt_send_t, ddt_recv_t, ddt_comm_t, DDT_XCHG_NCCL, DDT_XCHG_P2P)
+from .queue import ptr_of
+
+
+class Comm:
+    """rank / nranks, an NCCL communicator (nranks > 1) and, for the P2P mode,
+    the device pointers of every rank's receive window."""
+
+    def __init__(self, rank: int = 0, nranks: int = 1, device: int = 0, nccl_comm=None, group=None):
+        self.rank, self.nranks, self.device = int(rank), int(nranks), int(device)
+        self.nccl_comm = nccl_comm
+        self.group = group
+        self.window = None          # own window (device pointer)
+        self.window_bytes = 0
+        self.peer_windows = None    # ctypes array of device pointers (own included)
+        self._opened = []
+
+    @staticmethod
+    def single(device: int = 0) -> "Comm":
+        return Comm(0, 1, device)
+
+    @staticmethod
+    def from_torch(device: int, group=None) -> "Comm":
+        """One process per GPU under torch.distributed: creates an NCCL
+        communicator of the same ranks (unique id broadcast by the group)."""
+        import torch.distributed as dist
+        rank, n = dist.get_rank(group), dist.get_world_size(group)
+        c = Comm(rank, n, device, group=group)
+        if n > 1:
+            uid = ctypes.create_string_buffer(128)
+            if rank == 0:
+                check(lib().ddt_nccl_unique_id(uid), "ddt_nccl_unique_id")
+            obj = [bytes(uid.raw) if rank == 0 else None]
+            dist.broadcast_object_list(obj, src=0, group=group)
+            uid = ctypes.create_string_buffer(obj[0], 128)
+            comm = P()
+            import torch
+            with torch.cuda.device(device):
+                check(lib().ddt_nccl_comm_create(n, uid, rank, ctypes.byref(comm)), "ddt_nccl_comm_create")
+            c.nccl_comm = comm
+        return c
+
+    def setup_windows(self, nbytes: int):
+        """Allocate this rank's receive window and map every peer's (CUDA IPC)."""
+        ptr = P()
+        handle = ctypes.create_string_buffer(64)
+        check(lib().ddt_window_alloc(self.device, int(nbytes), ctypes.byref(ptr), handle), "ddt_window_alloc")
+        self.window, self.window_bytes = ptr.value, int(nbytes)
+        ptrs = [0] * self.nranks
+        ptrs[self.rank] = ptr.value
+        if self.nranks > 1:
+            import torch.distributed as dist
+            allh = [None] * self.nranks
+            dist.all_gather_object(allh, (bytes(handle.raw), int(nbytes)), group=self.group)
+            for p, (h, nb) in enumerate(allh):
+                if p == self.rank:
+                    continue
+                q = P()
+                check(lib().ddt_window_open(self.device, ctypes.create_string_buffer(h, 64), ctypes.byref(q)),
+                      "ddt_window_open")
+                ptrs[p] = q.value
+                self._opened.append(q.value)
+        self.peer_windows = (P * self.nranks)(*ptrs)
+        return self.window
+
+    def as_struct(self) -> ddt_comm_t:
+        c = ddt_comm_t()
+        c.rank, c.nranks = self.rank, self.nranks
+        c.nccl_comm = self.nccl_comm.value if isinstance(self.nccl_comm, P) else self.nccl_comm
+        c.peer_windows = ctypes.cast(self.peer_windows, ctypes.POINTER(P)) if self.peer_windows else None
+        c.window_bytes = self.window_bytes
+        return c
+
+    def close(self):
+        for q in self._opened:
+            lib().ddt_window_close(ctypes.c_void_p(q))
+        self._opened = []
+        if self.window:
+            lib().ddt_window_free(ctypes.c_void_p(self.window))
+            self.window = None
+        if self.nccl_comm is not None:
+            lib().ddt_nccl_comm_destroy(self.nccl_comm)
+            self.nccl_comm = None
+
+
+def _msgs(items, cls):
+    arr = (cls * max(1, len(items)))()
+    for i, m in enumerate(items):
+        peer, tag, t, buf, count = m
+        arr[i].peer, arr[i].tag, arr[i].type = int(peer), int(tag), t.handle.value
+        arr[i].buf, arr[i].count = ptr_of(buf), int(count)
+    return arr
+
+
+class Halo:
+    """A persistent exchange plan.  sends / recvs: lists of
+    (peer, tag, Type, buffer, count); a send to (peer, tag) matches the peer's
+    receive from (this rank, tag)."""
+
+    def __init__(self, queue, comm: Comm, sends, recvs, mode: str = "nccl", graph: bool = True):
+        self.queue, self.comm = queue, comm
+        self._keep = [m[2] for m in sends] + [m[2] for m in recvs]
+        s_arr = _msgs(sends, ddt_send_t)
+        r_arr = _msgs(recvs, ddt_recv_t)
+        self.mode = DDT_XCHG_P2P if mode == "p2p" else DDT_XCHG_NCCL
+        if self.mode == DDT_XCHG_P2P and comm.window is None:
+            nb = ctypes.c_int64()
+            check(lib().ddt_halo_window_bytes(len(recvs), r_arr, ctypes.byref(nb)), "ddt_halo_window_bytes")
+            comm.setup_windows(nb.value)
+        cs = comm.as_struct()
+        out = P()
+        check(lib().ddt_halo_create(queue.handle, ctypes.byref(cs), len(sends), s_arr, len(recvs), r_arr,
+                                    self.mode, ctypes.byref(out)), "ddt_halo_create")
+        self._h = out
+        check(lib().ddt_halo_set_graph(self._h, 1 if graph else 0), "ddt_halo_set_graph")
+
+    def exchange(self):
+        check(lib().ddt_exchange(self._h), "ddt_exchange")
+
+    @property
+    def launches_per_exchange(self) -> int:
+        v = ctypes.c_int32()
+        check(lib().ddt_halo_launches_per_exchange(self._h, ctypes.byref(v)), "ddt_halo_launches_per_exchange")
+        return v.value
+
+    def destroy(self):
+        if self._h and self._h.value:
+            check(lib().ddt_halo_destroy(self._h), "ddt_halo_destroy")
+        self._h = P()
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass

@@ -1,0 +1,91 @@
+"""Request list + scheduler (§IV-A): enqueue -> uid, flush
+-> one fused launch, query by uid, wait.  Marshalling only (csrc/queue.cpp)."""
+from __future__ import annotations
+
+import ctypes
+
+from ._abi import lib, check, P, ddt_queue_stats_t, STATE_NAMES
+
+
+def ptr_of(buf) -> int:
+    """Device address of a buffer: an int, a torch tensor, or (buffer, byte_offset)."""
+    if isinstance(buf, tuple):
+        base, off = buf
+        return ptr_of(base) + int(off)
+    if isinstance(buf, int):
+        return buf
+    if hasattr(buf, "data_ptr"):
+        return int(buf.data_ptr())
+    raise TypeError(f"cannot take a device pointer of {type(buf)!r}")
+
+
+def current_stream_handle(device=None) -> int:
+    import torch
+    return int(torch.cuda.current_stream(device).cuda_stream)
+
+
+class Queue:
+    """A request list bound to (device, CUDA stream).  Default stream: torch's
+    current stream on `device` at construction time."""
+
+    def __init__(self, device: int | None = None, stream=None, capacity: int = 0):
+        import torch
+        if device is None:
+            device = torch.cuda.current_device()
+        if stream is None:
+            stream = torch.cuda.current_stream(device)
+        self.device = int(device)
+        self.stream = stream
+        handle = int(stream.cuda_stream) if hasattr(stream, "cuda_stream") else int(stream)
+        out = P()
+        check(lib().ddt_queue_create(self.device, ctypes.c_void_p(handle), int(capacity), ctypes.byref(out)),
+              "ddt_queue_create")
+        self._h = out
+
+    @property
+    def handle(self):
+        return self._h
+
+    def pack(self, t, src, count: int, dst_packed) -> int:
+        """Scheduler (1): enqueue a packing request; returns its uid."""
+        return check(lib().ddt_pack_enqueue(self._h, t.handle, ctypes.c_void_p(ptr_of(src)), int(count),
+                                            ctypes.c_void_p(ptr_of(dst_packed))), "ddt_pack_enqueue")
+
+    def unpack(self, t, src_packed, count: int, dst) -> int:
+        """Scheduler (1): enqueue an unpacking request; returns its uid."""
+        return check(lib().ddt_unpack_enqueue(self._h, t.handle, ctypes.c_void_p(ptr_of(src_packed)), int(count),
+                                              ctypes.c_void_p(ptr_of(dst))), "ddt_unpack_enqueue")
+
+    def try_pack(self, t, src, count, dst_packed) -> int:
+        """Like pack() but returns the negative status instead of raising."""
+        return lib().ddt_pack_enqueue(self._h, t.handle, ctypes.c_void_p(ptr_of(src)), int(count),
+                                      ctypes.c_void_p(ptr_of(dst_packed)))
+
+    def flush(self) -> int:
+        """Scheduler (2): one fused launch for every pending request."""
+        return check(lib().ddt_flush(self._h), "ddt_flush")
+
+    def query(self, uid: int) -> str:
+        """Scheduler (4): 'pending' | 'busy' | 'completed'."""
+        st = ctypes.c_int32()
+        check(lib().ddt_query(self._h, int(uid), ctypes.byref(st)), "ddt_query")
+        return STATE_NAMES[st.value]
+
+    def wait(self):
+        check(lib().ddt_wait(self._h), "ddt_wait")
+
+    def stats(self) -> dict:
+        s = ddt_queue_stats_t()
+        check(lib().ddt_queue_get_stats(self._h, ctypes.byref(s)), "ddt_queue_get_stats")
+        return {"requests": s.requests, "launches": s.launches, "flushes": s.flushes, "bytes": s.bytes}
+
+    def destroy(self):
+        if self._h and self._h.value:
+            check(lib().ddt_queue_destroy(self._h), "ddt_queue_destroy")
+        self._h = P()
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass

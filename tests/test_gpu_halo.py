@@ -1,0 +1,129 @@
+"""GPU halo-exchange parity on one B200 (every message a self message at P=1):
+after each ddt_exchange the ghost cells equal numpy's periodic padding of the
+interior (SURVEY §8(c) 'Halo exchange' pin, an independent library routine),
+the interior is untouched, and un-targeted ghosts keep the sentinel.  Both the
+NCCL-mode plan (fused pack -> fused unpack) and the fused single-kernel P2P
+plan (window + epoch flags, double-buffered by parity) are exercised over
+several iterations, with and without CUDA-graph replay."""
+import numpy as np
+import pytest
+
+from ddt_inputs import halo_messages, ghost_mask, FACE_DIRS, ALL_DIRS, random_bytes, seed
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ddt():
+    import torch
+    assert torch.cuda.is_available()
+    from paper_conf_cluster_chukzsp20_b200.build import build
+    build()
+    import paper_conf_cluster_chukzsp20_b200 as m
+    return m
+
+
+def _setup(ddt, local, dirs, nvars, mode, graph, cfg):
+    import torch
+    q = ddt.Queue()
+    shape = tuple(n + 2 for n in local)
+    arrs = []
+    for v in range(nvars):
+        a = torch.full(shape, 0, dtype=torch.int64, device="cuda")
+        a.view(torch.uint8).fill_(0xA5)
+        arrs.append(a)
+    msgs = halo_messages(0, 1, local, dirs=dirs, nvars=nvars)
+    types = {}
+
+    def T(spec):
+        key = repr(spec)
+        if key not in types:
+            types[key] = ddt.Type.from_spec(spec)
+        return types[key]
+
+    sends = [(m["peer"], m["tag"], T(m["send_spec"]), arrs[m["var"]], 1) for m in msgs]
+    recvs = [(m["recv_peer"], m["recv_tag"], T(m["recv_spec"]), arrs[m["var"]], 1) for m in msgs]
+    comm = ddt.Comm.single(torch.cuda.current_device())
+    h = ddt.Halo(q, comm, sends, recvs, mode=mode, graph=graph)
+    return q, arrs, h, comm
+
+
+def _fill_interior(arrs, local, it, cfg):
+    import torch
+    for v, a in enumerate(arrs):
+        n = int(np.prod(local))
+        vals = random_bytes(n * 8, seed(cfg, 10 * it + v)).view(np.int64).reshape(local)
+        a[1:-1, 1:-1, 1:-1] = torch.from_numpy(vals).cuda()
+
+
+def _check(arrs, local, dirs):
+    gm = ghost_mask(local, dirs)
+    for a in arrs:
+        h = a.cpu().numpy()
+        exp = np.pad(h[1:-1, 1:-1, 1:-1], 1, mode="wrap")
+        assert np.array_equal(h[gm], exp[gm]), "ghost cells differ from np.pad(wrap)"
+        rest = ~gm
+        rest[1:-1, 1:-1, 1:-1] = False
+        assert np.all(h.view(np.uint8).reshape(h.shape + (8,))[rest] == 0xA5)
+
+
+@pytest.mark.parametrize("mode", ["nccl", "p2p"])
+@pytest.mark.parametrize("graph", [False, True])
+@pytest.mark.parametrize("local,dirs,nvars,cfg", [
+    ((5, 6, 7), ALL_DIRS, 2, 4),
+    ((9, 4, 3), FACE_DIRS, 1, 2),
+])
+def test_halo_small(ddt, mode, graph, local, dirs, nvars, cfg):
+    import torch
+    q, arrs, h, comm = _setup(ddt, local, dirs, nvars, mode, graph, cfg)
+    for it in range(4):
+        _fill_interior(arrs, local, it, cfg)
+        torch.cuda.synchronize()
+        h.exchange()
+        torch.cuda.synchronize()
+        _check(arrs, local, dirs)
+    assert h.launches_per_exchange == (1 if mode == "p2p" else 2)
+    h.destroy()
+    comm.close()
+
+
+@pytest.mark.parametrize("mode", ["nccl", "p2p"])
+def test_config2_face_halo_full_size(ddt, mode):
+    """BASELINE.json configs[1] per-rank size (128^3 doubles, 6 face messages),
+    P = 1, as bench.py runs it (graph replay)."""
+    import torch
+    local = (128, 128, 128)
+    q, arrs, h, comm = _setup(ddt, local, FACE_DIRS, 1, mode, True, 2)
+    for it in range(3):
+        _fill_interior(arrs, local, it, 2)
+        torch.cuda.synchronize()
+        h.exchange()
+        torch.cuda.synchronize()
+        _check(arrs, local, FACE_DIRS)
+    h.destroy()
+    comm.close()
+
+
+def test_config4_comb_halo_full_size_p1(ddt):
+    """BASELINE.json configs[3] at its 1-GPU point: 512^3 doubles, 4 variables,
+    26 neighbours, 104 + 104 messages per iteration; variable 0 fully checked,
+    the others on their ghost faces."""
+    import torch
+    local = (512, 512, 512)
+    q, arrs, h, comm = _setup(ddt, local, ALL_DIRS, 4, "p2p", True, 4)
+    g = torch.Generator(device="cuda")
+    g.manual_seed(seed(4))
+    for a in arrs:
+        a[1:-1, 1:-1, 1:-1] = torch.randint(-2**62, 2**62, local, device="cuda", dtype=torch.int64, generator=g)
+    torch.cuda.synchronize()
+    h.exchange()
+    torch.cuda.synchronize()
+    _check(arrs[:1], local, ALL_DIRS)
+    for a in arrs[1:]:
+        # faces: ghost plane == opposite interior plane (periodic, P = 1)
+        assert torch.equal(a[0, 1:-1, 1:-1], a[-2, 1:-1, 1:-1])
+        assert torch.equal(a[1:-1, -1, 1:-1], a[1:-1, 1, 1:-1])
+        assert torch.equal(a[1:-1, 1:-1, 0], a[1:-1, 1:-1, -2])
+        assert torch.equal(a[0, 0, 0], a[-2, -2, -2])
+    h.destroy()
+    comm.close()

@@ -1,0 +1,233 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle, bit-exact
+(zero tolerance: pure byte movement), with 0xA5 sentinels
+outside every footprint.  Covers random nested types, misaligned pointers,
+count > 1, the BASELINE.json configs 1, 3, 5 at full size, fused mixed
+batches (one launch per flush), the request-list states and limits."""
+import numpy as np
+import pytest
+from hypothesis import given, settings, strategies as st, HealthCheck
+
+import oracle
+from ddt_inputs import (random_bytes, SENTINEL, config1_spec, config3_spec, config5_spec, seed)
+from gpu_util import Case, cuda_bytes, host, assert_bytes_equal
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ddt():
+    import torch
+    assert torch.cuda.is_available(), "GPU tests need a CUDA device"
+    from paper_conf_cluster_chukzsp20_b200.build import build
+    build()
+    import paper_conf_cluster_chukzsp20_b200 as m
+    return m
+
+
+@pytest.fixture(scope="module")
+def q(ddt):
+    return ddt.Queue()
+
+
+def _run_case(ddt, q, c: Case):
+    import torch
+    launches0 = q.stats()["launches"]
+    uid_p, _, dp = c.gpu_pack(q)
+    uid_u, _, du = c.gpu_unpack(q)
+    n = q.flush()
+    assert n == 2
+    q.wait()
+    assert q.query(uid_p) == "completed" and q.query(uid_u) == "completed"
+    torch.cuda.synchronize()
+    assert_bytes_equal(host(dp), c.expect_pack(), f"pack {c.spec} count={c.count}")
+    if not c.o.num_entries or not _overlaps(c):
+        assert_bytes_equal(host(du), c.expect_unpack(), f"unpack {c.spec} count={c.count}")
+    assert q.stats()["launches"] - launches0 == (1 if c.psize else 0)
+
+
+def _overlaps(c):
+    d, ln = c.o.typemap(c.count)
+    b = np.concatenate([np.arange(a, a + n) for a, n in zip(d, ln)]) if len(d) else np.zeros(0)
+    return len(np.unique(b)) != len(b)
+
+
+# --------------------------------------------------------------- random types
+from test_abi_cpu import spec_strategy  # noqa: E402
+
+
+@settings(max_examples=250, deadline=None, suppress_health_check=list(HealthCheck))
+@given(spec=spec_strategy(), count=st.integers(1, 3), mis=st.integers(0, 15), pkm=st.sampled_from([0, 0, 4, 8, 1]),
+       s=st.integers(0, 1000))
+def test_random_types_bit_exact(ddt, q, spec, count, mis, pkm, s):
+    c = Case(ddt, spec, count, misalign=mis, seed=s, pk_misalign=pkm)
+    if c.psize and _overlaps(c):
+        # unpack into overlapping entries is rejected (R5); pack still parity-checked
+        import torch
+        uid, _, dp = c.gpu_pack(q)
+        q.flush()
+        q.wait()
+        assert_bytes_equal(host(dp), c.expect_pack(), f"pack {spec}")
+        from paper_conf_cluster_chukzsp20_b200 import DDTError
+        with pytest.raises(DDTError):
+            c.gpu_unpack(q)
+        return
+    _run_case(ddt, q, c)
+
+
+# --------------------------------------------------------------- config 1
+@pytest.mark.parametrize("count", [1, 2, 5])
+@pytest.mark.parametrize("mis", [0, 8, 3])
+def test_config1_vector(ddt, q, count, mis):
+    _run_case(ddt, q, Case(ddt, config1_spec(), count, misalign=mis, seed=seed(1)))
+
+
+def test_config1_golden_values(ddt, q):
+    """Labelled source: the packed doubles are the golden byte offsets."""
+    import torch
+    t = ddt.Type.from_spec(config1_spec())
+    lab = torch.arange(1000, dtype=torch.int64, device="cuda") * 8
+    out = torch.zeros(64, dtype=torch.int64, device="cuda")
+    q.pack(t, lab, 1, out)
+    q.wait()
+    exp = np.concatenate([np.arange(512 * i, 512 * i + 32, 8) for i in range(16)])
+    assert host(out).tolist() == exp.tolist()
+
+
+# --------------------------------------------------------------- config 3
+@pytest.mark.parametrize("shuffled", [False, True])
+def test_config3_sparse_hindexed_full(ddt, q, shuffled):
+    """10^5 blocks of 3 floats over 2^20 points (12 MiB source), batch of 4
+    requests with distinct sources, all in one launch."""
+    import torch
+    spec, nb = config3_spec(shuffled=shuffled)
+    t = ddt.Type.from_spec(spec)
+    o = oracle.Type(spec)
+    assert t.layout_kind == "uniform_list"
+    B = 4
+    srcs = [random_bytes(nb, seed(3, v)) for v in range(B)]
+    d_src = [cuda_bytes(s) for s in srcs]
+    d_pk = [torch.full((t.size,), SENTINEL, dtype=torch.uint8, device="cuda") for _ in range(B)]
+    d_un = [torch.full((nb,), SENTINEL, dtype=torch.uint8, device="cuda") for _ in range(B)]
+    l0 = q.stats()["launches"]
+    for v in range(B):
+        q.pack(t, d_src[v], 1, d_pk[v])
+    q.flush()
+    for v in range(B):
+        q.unpack(t, d_pk[v], 1, d_un[v])
+    q.flush()
+    q.wait()
+    assert q.stats()["launches"] - l0 == 2
+    for v in range(B):
+        exp = oracle.pack(o, srcs[v])
+        assert_bytes_equal(host(d_pk[v]), exp, "config3 pack")
+        eu = np.full(nb, SENTINEL, np.uint8)
+        oracle.unpack(o, exp, eu)
+        assert_bytes_equal(host(d_un[v]), eu, "config3 unpack")
+
+
+# --------------------------------------------------------------- config 5
+@pytest.mark.parametrize("S,B", [(64, 1), (64, 64), (1024, 16), (16384, 4), (262144, 16), (4 << 20, 4),
+                                 (64 << 20, 1)])
+def test_config5_dense_vector_batches(ddt, q, S, B):
+    """Message-size sweep cells: B requests of S bytes, fused pack then fused
+    unpack; every request checked against the oracle."""
+    import torch
+    spec, fp = config5_spec(S)
+    t = ddt.Type.from_spec(spec)
+    o = oracle.Type(spec)
+    srcs = [random_bytes(fp, seed(5, i)) for i in range(B)]
+    d_src = [cuda_bytes(s) for s in srcs]
+    d_pk = [torch.full((S,), SENTINEL, dtype=torch.uint8, device="cuda") for _ in range(B)]
+    d_un = [torch.full((fp,), SENTINEL, dtype=torch.uint8, device="cuda") for _ in range(B)]
+    for i in range(B):
+        q.pack(t, d_src[i], 1, d_pk[i])
+    assert q.flush() == B
+    for i in range(B):
+        q.unpack(t, d_pk[i], 1, d_un[i])
+    assert q.flush() == B
+    q.wait()
+    for i in range(B):
+        exp = oracle.pack(o, srcs[i])
+        assert_bytes_equal(host(d_pk[i]), exp, f"config5 pack S={S}")
+        eu = np.full(fp, SENTINEL, np.uint8)
+        oracle.unpack(o, exp, eu)
+        assert_bytes_equal(host(d_un[i]), eu, f"config5 unpack S={S}")
+
+
+# --------------------------------------------------------------- batches / scheduler
+def test_mixed_batch_one_launch_equals_sequential_oracle(ddt, q):
+    """A fused batch of 96 mixed pack/unpack requests of different types is ONE
+    launch and equals the oracle executing the requests one by one (R6)."""
+    import torch
+    rng = np.random.default_rng(7)
+    specs = [config1_spec(), ("subarray", [9, 10, 11], [3, 4, 5], [1, 2, 3], "C", ("basic", "double")),
+             ("subarray", [9, 10, 11], [9, 1, 11], [0, 4, 0], "F", ("basic", "float")),
+             ("hindexed", [3, 1, 2], [100, 4, 37], ("basic", "byte")),
+             ("indexed", [1, 2, 3], [0, 10, 20], ("basic", "int32")),
+             ("vector", 5, 3, -4, ("basic", "int64"))]
+    cases = [Case(ddt, specs[i % len(specs)], count=int(rng.integers(1, 4)), misalign=int(rng.integers(0, 16)),
+                  seed=i) for i in range(96)]
+    bufs = []
+    l0 = q.stats()["launches"]
+    for i, c in enumerate(cases):
+        bufs.append(c.gpu_pack(q) if i % 2 == 0 else c.gpu_unpack(q))
+    assert q.flush() == 96
+    q.wait()
+    assert q.stats()["launches"] - l0 == 1
+    for i, (c, (_, _, d)) in enumerate(zip(cases, bufs)):
+        exp = c.expect_pack() if i % 2 == 0 else c.expect_unpack()
+        assert_bytes_equal(host(d), exp, f"batch item {i}")
+
+
+def test_queue_full_gives_negative_uid_then_recovers(ddt):
+    import torch
+    q4 = ddt.Queue(capacity=4)
+    t = ddt.Type.from_spec(config1_spec())
+    s = torch.zeros(8192, dtype=torch.uint8, device="cuda")
+    d = torch.zeros(512 * 8, dtype=torch.uint8, device="cuda")
+    uids = [q4.pack(t, s, 1, (d, 512 * i)) for i in range(4)]
+    assert uids == [0, 1, 2, 3]
+    assert q4.try_pack(t, s, 1, d) == -3  # DDT_ERR_QUEUE_FULL: the paper's negative UID
+    assert q4.query(3) == "pending"
+    q4.flush()
+    q4.wait()
+    assert all(q4.query(u) == "completed" for u in uids)
+    assert q4.pack(t, s, 1, d) == 4
+    q4.wait()
+    q4.destroy()
+
+
+def test_zero_size_and_empty_requests(ddt, q):
+    import torch
+    t = ddt.Type.from_spec(("vector", 0, 3, 2, ("basic", "double")))
+    s = torch.zeros(16, dtype=torch.uint8, device="cuda")
+    uid = q.pack(t, s, 5, s)
+    assert q.query(uid) == "completed"
+    t1 = ddt.Type.from_spec(config1_spec())
+    uid2 = q.pack(t1, s, 0, s)
+    assert q.query(uid2) == "completed"
+    l0 = q.stats()["launches"]
+    q.flush()
+    q.wait()
+    assert q.stats()["launches"] == l0  # nothing to move -> no launch
+
+
+def test_oversized_request_rejected(ddt, q):
+    from paper_conf_cluster_chukzsp20_b200 import DDTError
+    t = ddt.Type.from_spec(("contiguous", 1 << 33, ("basic", "byte")))
+    with pytest.raises(DDTError) as e:
+        q.pack(t, 1, 1, 3)  # odd pointers -> 1-byte vectors -> 2^33 vectors > 2^32
+    assert e.value.code == -10
+
+
+def test_nan_and_negative_zero_survive(ddt, q):
+    import torch
+    vals = np.array([np.nan, -0.0, np.inf, -np.inf, 5e-324, 1.0] * 40, dtype=np.float64)
+    vals.view(np.uint64)[0] = 0x7FF0000000000123  # signalling-NaN payload
+    t = ddt.Type.from_spec(("vector", 60, 2, 4, ("basic", "double")))
+    s = cuda_bytes(vals)
+    d = torch.zeros(t.size, dtype=torch.uint8, device="cuda")
+    q.pack(t, s, 1, d)
+    q.wait()
+    exp = oracle.pack(oracle.Type(("vector", 60, 2, 4, ("basic", "double"))), vals.view(np.uint8))
+    assert_bytes_equal(host(d), exp, "nan payloads")
