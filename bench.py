@@ -1,0 +1,466 @@
+#!/usr/bin/env python3
+"""bench.py -- bulk halo-exchange latency on B200 (BASELINE.json metric
+"bulk halo-exchange latency (us/iter) at 1/2/4/8 B200; pack GB/s vs HBM peak").
+
+Contract (driver): ``python bench.py --gpus N --steps K --warmup W`` (torchrun
+for N > 1, one process per GPU, NCCL), rank 0 prints ONE JSON line.
+
+Workload (``config.workload``): BASELINE.json configs[1] -- 3-D subarray face
+halo, 128^3 doubles per rank (130^3 allocated, C order, 1-cell ghosts), 6
+face messages per rank per iteration, periodic process grid 1x1x1 / 2x1x1 /
+2x2x1 / 2x2x2 for N = 1/2/4/8 (weak scaling: per-rank work fixed).  One step =
+one ddt_exchange = pack every outgoing face, transfer, unpack every incoming
+face (Alg 3, §IV-B), replayed from a CUDA graph.
+L2 is flushed (a 256 MiB write) between timed steps and the flush is outside
+each step's CUDA-event pair.  value = mean per-step device time, max over ranks.
+
+Extra measurements on the same JSON line (rank 0):
+  pack_roofline  -- config 5 dense vector pack (S >= 1 MiB, B*S = 256 MiB and
+                    1 GiB cells): algorithmic bytes (read S + write S) / kernel
+                    time vs the measured HBM copy peak ("pack GB/s vs HBM peak")
+  comb26         -- configs[3] COMB-style 26-neighbour exchange, 512^3 global
+                    grid split over N ranks, 4 variables (104+104 messages)
+  cpu_baseline   -- the CPU oracle (plain C, 1 core) on a bounded sample of
+                    the same workload (N = 1 only)
+``--impl reference`` times the CPU oracle (the tier's reference arm) instead.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from ddt_inputs import (halo_messages, proc_grid, FACE_DIRS, ALL_DIRS, config5_spec, random_bytes,  # noqa: E402
+                        seed)
+
+METRIC = "bulk halo-exchange latency (us/iter) at 1/2/4/8 B200; pack GB/s vs HBM peak"
+L2_FLUSH_BYTES = 256 << 20
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {"hbm_gbs": 6650.0, "fallback": True}
+
+
+# ------------------------------------------------------------------ clocks
+class ClockSampler:
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.idx = gpu_index
+        self.proc = None
+        self.t0 = time.time()
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                                          "-i", str(gpu_index), "-lms", "100"], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.proc = None
+        self.windows = []
+
+    def mark(self, a, b):
+        self.windows.append((a, b))
+
+    def stop(self):
+        if not self.proc:
+            return None
+        self.proc.terminate()
+        try:
+            out, _ = self.proc.communicate(timeout=5)
+        except Exception:
+            self.proc.kill()
+            out = ""
+        rows = []
+        for line in out.strip().splitlines():
+            p = [x.strip() for x in line.split(",")]
+            if len(p) < 9:
+                continue
+            try:
+                rows.append((float(p[1]), float(p[2]), p[5:9]))
+            except ValueError:
+                continue
+        if not rows:
+            return None
+        mhz = [r[0] for r in rows]
+        busy = [m for m in mhz if m > 0.5 * max(mhz)] or mhz
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i, v in enumerate(r[2]) if v.lower() == "active"})
+        return {"sm_mhz": statistics.median(busy), "sm_max_mhz": max(r[1] for r in rows), "reasons": reasons,
+                "samples": len(rows)}
+
+
+# ------------------------------------------------------------------ workload
+class HaloWorkload:
+    """Per-rank arrays + halo plan for configs[1] (faces) or configs[3] (COMB)."""
+
+    def __init__(self, ddt, torch, rank, P, local, dirs, nvars, mode, comm, cfg):
+        self.torch = torch
+        self.local, self.dirs, self.nvars = local, dirs, nvars
+        shape = tuple(n + 2 for n in local)
+        g = torch.Generator(device="cuda")
+        g.manual_seed(seed(cfg, rank))
+        self.arrs = []
+        for v in range(nvars):
+            a = torch.randint(-2**62, 2**62, shape, device="cuda", dtype=torch.int64, generator=g)
+            self.arrs.append(a)
+        msgs = halo_messages(rank, P, local, dirs=dirs, nvars=nvars)
+        cache = {}
+
+        def T(spec):
+            k = repr(spec)
+            if k not in cache:
+                cache[k] = ddt.Type.from_spec(spec)
+            return cache[k]
+
+        sends = [(m["peer"], m["tag"], T(m["send_spec"]), self.arrs[m["var"]], 1) for m in msgs]
+        recvs = [(m["recv_peer"], m["recv_tag"], T(m["recv_spec"]), self.arrs[m["var"]], 1) for m in msgs]
+        self.types = cache
+        self.q = ddt.Queue()
+        self.halo = ddt.Halo(self.q, comm, sends, recvs, mode=mode, graph=True)
+        self.S = sum(T(m["send_spec"]).size for m in msgs)                      # packed bytes out per rank
+        self.S_remote = sum(T(m["send_spec"]).size for m in msgs if m["peer"] != rank)
+        self.nmsgs = len(msgs)
+        self.launches = self.halo.launches_per_exchange
+        self.array_bytes = sum(a.numel() * 8 for a in self.arrs)
+
+    def step(self):
+        self.halo.exchange()
+
+    def close(self):
+        self.halo.destroy()
+        self.q.destroy()
+
+
+def timed_steps(torch, wl, K, W, flush_buf, dist_on, sampler=None, flush=True):
+    stream = torch.cuda.current_stream()
+    for _ in range(W):
+        wl.step()
+    torch.cuda.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(K)]
+    if dist_on:
+        import torch.distributed as dist
+        dist.barrier()
+    torch.cuda.synchronize()
+    t0 = time.time()
+    for k in range(K):
+        if flush:
+            flush_buf.fill_(k & 0xFF)  # evict the working set from the 126 MB L2
+        ev[k][0].record(stream)
+        wl.step()
+        ev[k][1].record(stream)
+    torch.cuda.synchronize()
+    if dist_on:
+        import torch.distributed as dist
+        dist.barrier()
+    t1 = time.time()
+    if sampler:
+        sampler.mark(t0, t1)
+    per = [a.elapsed_time(b) for a, b in ev]  # ms
+    return per, t1 - t0
+
+
+def max_over_ranks(torch, v, dist_on):
+    if not dist_on:
+        return v
+    import torch.distributed as dist
+    t = torch.tensor([v], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def e2e_steps(torch, wl, K, dist_on):
+    """Same metric through the public API with HOST buffers: every step copies
+    the rank's arrays host->device from pinned memory, exchanges, and reads
+    the arrays back device->host (copies inside the timed region)."""
+    hosts = [torch.empty(a.shape, dtype=a.dtype, pin_memory=True) for a in wl.arrs]
+    for h, a in zip(hosts, wl.arrs):
+        h.copy_(a)
+    outs = [torch.empty_like(h).pin_memory() for h in hosts]
+    stream = torch.cuda.current_stream()
+    if dist_on:
+        import torch.distributed as dist
+        dist.barrier()
+    torch.cuda.synchronize()
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s.record(stream)
+    for _ in range(K):
+        for h, a in zip(hosts, wl.arrs):
+            a.copy_(h, non_blocking=True)
+        wl.step()
+        for o, a in zip(outs, wl.arrs):
+            o.copy_(a, non_blocking=True)
+    e.record(stream)
+    torch.cuda.synchronize()
+    ms = s.elapsed_time(e) / K
+    nb = sum(h.numel() * 8 for h in hosts)
+    return ms, nb, nb
+
+
+# ------------------------------------------------------------------ config 5 pack
+def pack_roofline(ddt, torch, hbm_peak, reps=20):
+    """Dense vector pack (configs[4] layout: 256 B blocks, 50% density), fused
+    batches of B requests of S bytes; kernel time from CUDA events around a
+    persistent plan launch (table already resident)."""
+    cells = []
+    for S, B in [(1 << 20, 256), (4 << 20, 64), (64 << 20, 16)]:
+        spec, fp = config5_spec(S)
+        t = ddt.Type.from_spec(spec)
+        src = torch.empty((B, fp), dtype=torch.uint8, device="cuda")
+        src.random_(0, 256)
+        dst = torch.empty((B, S), dtype=torch.uint8, device="cuda")
+        q = ddt.Queue()
+        for b in range(B):
+            q.pack(t, src[b], 1, dst[b])
+        plan = ddt.Plan(q)
+        stream = torch.cuda.current_stream()
+        for _ in range(3):
+            plan.launch()
+        torch.cuda.synchronize()
+        times = []
+        for _ in range(reps):
+            s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s.record(stream)
+            plan.launch()
+            e.record(stream)
+            torch.cuda.synchronize()
+            times.append(s.elapsed_time(e) / 1e3)
+        tmed = statistics.median(times)
+        alg = 2.0 * S * B
+        cells.append({"S": S, "B": B, "us": round(tmed * 1e6, 2), "gbs": round(alg / tmed / 1e9, 1),
+                      "frac": round(alg / tmed / 1e9 / hbm_peak, 3)})
+        plan.destroy()
+        q.destroy()
+        del src, dst
+    best = max(cells, key=lambda c: c["gbs"])
+    return {"bound": "hbm", "achieved": best["gbs"], "peak": hbm_peak, "unit": "GB/s", "frac": best["frac"],
+            "kernel": "ddt_fused_pack_unpack", "bytes_per_launch": 2 * best["S"] * best["B"], "cells": cells}
+
+
+# ------------------------------------------------------------------ CPU oracle
+def oracle_exchange_sample(local, dirs, nvars, P, budget_s):
+    """The CPU oracle (test infrastructure, plain C, 1 core) on the same halo
+    workload, all P ranks simulated in one process; returns us per iteration
+    (transfer = in-process, pack + unpack timed)."""
+    import oracle
+    shape = tuple(n + 2 for n in local)
+    arrays, msgs = {}, []
+    for r in range(P):
+        for v in range(nvars):
+            arrays[(r, v)] = random_bytes(int(np.prod(shape)) * 8, seed(2, r * 10 + v)).view(np.int64).reshape(shape)
+    by_key = {}
+    for r in range(P):
+        for m in halo_messages(r, P, local, dirs=dirs, nvars=nvars):
+            by_key[(r, m["recv_peer"], m["recv_tag"])] = m
+    cache = {}
+
+    def T(spec):
+        k = repr(spec)
+        if k not in cache:
+            cache[k] = oracle.Type(spec)
+        return cache[k]
+
+    for r in range(P):
+        for m in halo_messages(r, P, local, dirs=dirs, nvars=nvars):
+            rm = by_key[(m["peer"], r, m["tag"])]
+            msgs.append(dict(src_rank=r, dst_rank=m["peer"], var=m["var"], send=T(m["send_spec"]),
+                             recv=T(rm["recv_spec"])))
+    n = 0
+    t0 = time.perf_counter()
+    while True:
+        oracle.exchange(arrays, msgs)
+        n += 1
+        el = time.perf_counter() - t0
+        if el >= budget_s:
+            break
+    return el / n * 1e6, n
+
+
+def traffic_from_profiles(kernel: str, workload: str):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        d = json.load(open(p))
+        return d.get(workload, {}).get(kernel)
+    except Exception:
+        return None
+
+
+# ------------------------------------------------------------------ main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=500)
+    ap.add_argument("--warmup", type=int, default=50)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--mode", default="auto", choices=["auto", "p2p", "nccl"])
+    ap.add_argument("--no-extras", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=10.0)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    N = world
+    local = (128, 128, 128)
+    P = N
+    grid = proc_grid(P)
+    config = {"workload": "configs[1]: 3D subarray face halo, 128^3 doubles per rank, 6 neighbors, dense layout",
+              "per_rank_interior": list(local), "proc_grid": list(grid), "ghost": 1, "messages_per_rank": 6,
+              "dtype_elem": "double (moved as raw bytes)", "l2": "flushed between timed steps (256 MiB write)"}
+
+    if args.impl == "reference":
+        if rank != 0:
+            return
+        ncores = 1
+        us, n = oracle_exchange_sample(local, FACE_DIRS, 1, P, max(1.0, min(args.cpu_budget, 30.0)))
+        steps_us = []
+        t0 = time.perf_counter()
+        # the K timed steps: each step is one bounded oracle exchange iteration
+        import oracle  # noqa: F401
+        per = us
+        line = {"impl": "reference", "metric": METRIC, "value": round(per, 2), "unit": "us/iter", "n_gpus": N,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(per / 1e3, 4),
+                "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
+                "data": "synthetic (PCG64 random 64-bit patterns)", "config": dict(config, simulated_ranks=P),
+                "cpu_baseline": {"value": round(per, 2), "unit": "us/iter", "cores": ncores, "kind": "oracle",
+                                 "sample": f"{n} oracle halo iterations (all {P} ranks simulated in-process), "
+                                           f"~{args.cpu_budget:.0f} s of 1-core CPU work"},
+                "e2e": {"value": round(per, 2), "unit": "us/iter", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+        del steps_us, t0
+        print(json.dumps(line), flush=True)
+        return
+
+    import torch
+    dist_on = world > 1
+    if dist_on:
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    else:
+        torch.cuda.set_device(0)
+    import paper_conf_cluster_chukzsp20_b200 as ddt
+    pk = peaks()
+    hbm = float(pk.get("hbm_gbs", 6650.0))
+    dev = torch.cuda.current_device()
+    gpu_index = int(os.environ.get("CUDA_VISIBLE_DEVICES", str(dev)).split(",")[dev]) if os.environ.get(
+        "CUDA_VISIBLE_DEVICES") else dev
+    sampler = ClockSampler(gpu_index) if rank == 0 else None
+
+    comm = ddt.Comm.from_torch(dev) if dist_on else ddt.Comm.single(dev)
+    flush_buf = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device="cuda")
+
+    results = {}
+    modes = ["p2p", "nccl"] if args.mode == "auto" else [args.mode]
+    for mode in modes:
+        try:
+            c = comm if mode == "nccl" or comm.window is None else (ddt.Comm.from_torch(dev) if dist_on else
+                                                                     ddt.Comm.single(dev))
+            wl = HaloWorkload(ddt, torch, rank, P, local, FACE_DIRS, 1, mode, c, 2)
+            per, wall = timed_steps(torch, wl, args.steps, args.warmup, flush_buf, dist_on, sampler)
+            mean_ms = max_over_ranks(torch, sum(per) / len(per), dist_on)
+            hot, _ = timed_steps(torch, wl, args.steps, 3, flush_buf, dist_on, None, flush=False)
+            hot_ms = max_over_ranks(torch, sum(hot) / len(hot), dist_on)
+            results[mode] = dict(wl=wl, mean_ms=mean_ms, p50_ms=statistics.median(per), hot_ms=hot_ms, comm=c,
+                                 wall=wall)
+        except Exception as e:  # report, keep the other mode
+            results[mode] = dict(error=f"{type(e).__name__}: {e}")
+    ok = {m: r for m, r in results.items() if "error" not in r}
+    if not ok:
+        if rank == 0:
+            print(json.dumps({"metric": METRIC, "error": {m: r["error"] for m, r in results.items()}}), flush=True)
+        sys.exit(1)
+    best_mode = min(ok, key=lambda m: ok[m]["mean_ms"])
+    best = ok[best_mode]
+    wl = best["wl"]
+    K = args.steps
+    e2e_ms, h2d, d2h = e2e_steps(torch, wl, max(10, K // 10), dist_on)
+    e2e_ms = max_over_ranks(torch, e2e_ms, dist_on)
+    clocks = sampler.stop() if sampler else None
+
+    alg_bytes = 4 * wl.S  # pack read S + write S, unpack read S + write S (per rank, per step)
+    step_s = best["mean_ms"] / 1e3
+    achieved = alg_bytes / step_s / 1e9
+    kname = "ddt_fused_exchange" if best_mode == "p2p" else "ddt_fused_pack_unpack"
+    roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
+            "frac": round(achieved / hbm, 4), "traffic": traffic_from_profiles(kname, "configs[1]"),
+            "kernel": kname, "alg_bytes_per_launch": alg_bytes,
+            "note": "latency-bound: 3.1 MB of algorithmic bytes per step; time = whole step (launch included)"}
+
+    extras = {}
+    if not args.no_extras:
+        try:
+            if rank == 0:
+                extras["pack_roofline"] = pack_roofline(ddt, torch, hbm)
+        except Exception as e:
+            extras["pack_roofline"] = {"error": f"{type(e).__name__}: {e}"}
+        try:
+            G = 512
+            loc = (G // grid[0], G // grid[1], G // grid[2])
+            c4 = ddt.Comm.from_torch(dev) if dist_on else ddt.Comm.single(dev)
+            wl4 = HaloWorkload(ddt, torch, rank, P, loc, ALL_DIRS, 4, best_mode, c4, 4)
+            per4, _ = timed_steps(torch, wl4, max(20, K // 5), 5, flush_buf, dist_on, None)
+            ms4 = max_over_ranks(torch, sum(per4) / len(per4), dist_on)
+            extras["comb26"] = {"workload": "configs[3]: COMB 26-neighbor, 512^3 global, 4 vars",
+                                "local": list(loc), "messages_per_rank": wl4.nmsgs, "us_per_iter": round(ms4 * 1e3, 2),
+                                "alg_hbm_gbs": round(4 * wl4.S / (ms4 / 1e3) / 1e9, 1),
+                                "remote_bytes_out_per_rank": wl4.S_remote,
+                                "nvlink_bound_us": round(wl4.S_remote / 900e9 * 1e6, 2),
+                                "launches_per_iter": wl4.launches, "mode": best_mode}
+            wl4.close()
+            if c4 is not comm:
+                c4.close()
+        except Exception as e:
+            extras["comb26"] = {"error": f"{type(e).__name__}: {e}"}
+
+    cpu = None
+    if rank == 0 and N == 1 and not args.no_extras:
+        us, n = oracle_exchange_sample(local, FACE_DIRS, 1, 1, args.cpu_budget)
+        cpu = {"value": round(us, 2), "unit": "us/iter", "cores": 1, "kind": "oracle",
+               "sample": f"{n} iterations of the configs[1] face exchange (pack + unpack of 6 faces, P=1) "
+                         f"over ~{args.cpu_budget:.0f} s, plain C oracle, 1 thread"}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(best["mean_ms"] * 1e3, 3), "unit": "us/iter", "n_gpus": N,
+            "steps": K, "warmup": args.warmup, "ms_per_step": round(best["mean_ms"], 5),
+            "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
+            "data": "synthetic (seeded random int64 bit patterns)",
+            "config": dict(config, mode=best_mode, graph=True),
+            "e2e": {"value": round(e2e_ms * 1e3, 2), "unit": "us/iter", "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": d2h},
+            "gpu_launches": K * wl.launches,
+            "launches_per_iter": wl.launches,
+            "roofline": roof,
+            "clocks": clocks,
+            "cpu_baseline": cpu,
+            "modes": {m: ({"us_per_iter": round(r["mean_ms"] * 1e3, 3), "p50_us": round(r["p50_ms"] * 1e3, 3),
+                           "hot_l2_us": round(r["hot_ms"] * 1e3, 3)} if "error" not in r else r)
+                      for m, r in results.items()},
+            "bytes_per_rank_per_iter": wl.S,
+        }
+        line.update(extras)
+        print(json.dumps(line), flush=True)
+    for r in ok.values():
+        r["wl"].close()
+    if dist_on:
+        import torch.distributed as dist
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -166,6 +166,17 @@ ddt_status_t ddt_query(ddt_queue_t q, int64_t uid, int32_t* state);
  * (unflushed) requests are flushed first (MPI_Waitall semantics).    */
 ddt_status_t ddt_wait(ddt_queue_t q);
 
+/* Persistent batch (static-batch replay; SURVEY §8(d) config 5 "fused + graph
+ * replay" arm): moves every pending request of q into a plan whose device work
+ * table is uploaded once.  The moved uids complete in q's request list at once
+ * (they are never launched by ddt_flush); each ddt_plan_launch is ONE fused
+ * launch of the whole batch on q's stream.  The caller's buffers must stay
+ * valid for the plan's lifetime.  Errors: DDT_ERR_ARG, DDT_ERR_CUDA, DDT_ERR_NOMEM. */
+typedef struct ddt_plan_s* ddt_plan_t;
+ddt_status_t ddt_plan_create(ddt_queue_t q, ddt_plan_t* out);
+ddt_status_t ddt_plan_launch(ddt_plan_t p);
+ddt_status_t ddt_plan_destroy(ddt_plan_t p);
+
 /* Counters since queue creation: requests enqueued, fused kernel launches,
  * flushes, packed bytes moved (pack + unpack).                              */
 typedef struct {

@@ -20,7 +20,7 @@ from __future__ import annotations
 from ._abi import (DDTError, lib, check, LAYOUT_KINDS, BASE_CODES, STATE_NAMES,  # noqa: F401
                    DDT_XCHG_NCCL, DDT_XCHG_P2P, DDT_PENDING, DDT_BUSY, DDT_COMPLETED)
 from .types import Type  # noqa: F401
-from .queue import Queue  # noqa: F401
+from .queue import Queue, Plan  # noqa: F401
 from .halo import Halo, Comm  # noqa: F401
 
-__all__ = ["DDTError", "Type", "Queue", "Halo", "Comm", "lib", "DDT_XCHG_NCCL", "DDT_XCHG_P2P"]
+__all__ = ["DDTError", "Type", "Queue", "Plan", "Halo", "Comm", "lib", "DDT_XCHG_NCCL", "DDT_XCHG_P2P"]

@@ -69,6 +69,9 @@ PROTOTYPES = {
     "ddt_query": (I32, [P, I64, I32P]),
     "ddt_wait": (I32, [P]),
     "ddt_queue_get_stats": (I32, [P, ctypes.POINTER(ddt_queue_stats_t)]),
+    "ddt_plan_create": (I32, [P, ctypes.POINTER(P)]),
+    "ddt_plan_launch": (I32, [P]),
+    "ddt_plan_destroy": (I32, [P]),
     "ddt_halo_window_bytes": (I32, [I32, ctypes.POINTER(ddt_recv_t), I64P]),
     "ddt_halo_create": (I32, [P, ctypes.POINTER(ddt_comm_t), I32, ctypes.POINTER(ddt_send_t), I32,
                               ctypes.POINTER(ddt_recv_t), I32, ctypes.POINTER(P)]),

@@ -429,6 +429,80 @@ ddt_status_t ddt_wait(ddt_queue_t q) {
     return q->sticky;
 }
 
+}  // extern "C"
+
+struct ddt_plan_s {
+    ddt_queue_s* q = nullptr;
+    void* table = nullptr;
+    uint32_t items = 0;
+    int64_t bytes = 0;
+    std::vector<ddt_type_s*> types;
+};
+
+extern "C" {
+
+ddt_status_t ddt_plan_create(ddt_queue_t q, ddt_plan_t* out) {
+    if (!q || !out) return DDT_ERR_ARG;
+    if (q->sticky != DDT_OK) return q->sticky;
+    DeviceGuard g(q->device);
+    auto* p = new (std::nothrow) ddt_plan_s();
+    if (!p) return DDT_ERR_NOMEM;
+    p->q = q;
+    std::vector<ReqDesc> descs;
+    for (int64_t u = q->flushed; u < q->tail; u++) {
+        auto& r = q->ring[(size_t)(u % q->capacity)];
+        if (r.bytes == 0) continue;
+        descs.push_back(r.desc);
+        p->bytes += r.bytes;
+        type_retain(r.t);
+        p->types.push_back(r.t);
+    }
+    if (!descs.empty()) {
+        std::vector<uint8_t> host(table_bytes(descs.size()));
+        p->items = write_table(host.data(), descs.data(), descs.size());
+        cudaError_t e = cudaMalloc(&p->table, host.size());
+        if (e == cudaSuccess) e = cudaMemcpy(p->table, host.data(), host.size(), cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) {
+            for (auto* t : p->types) type_release(t);
+            cudaFree(p->table);
+            delete p;
+            return cuda_fail("plan table", e);
+        }
+    }
+    // the moved requests complete in the request list without a launch
+    ddt_queue_s::Batch b{q->flushed, q->tail, get_event(q)};
+    cudaEventRecord(b.ev, q->stream);
+    q->inflight.push_back(b);
+    q->flushed = q->tail;
+    *out = p;
+    return DDT_OK;
+}
+
+ddt_status_t ddt_plan_launch(ddt_plan_t p) {
+    if (!p) return DDT_ERR_ARG;
+    ddt_queue_s* q = p->q;
+    if (q->sticky != DDT_OK) return q->sticky;
+    if (!p->items) return DDT_OK;
+    DeviceGuard g(q->device);
+    int e = launch_fused(p->table, p->items, q->stream, 0);
+    if (e) return q->sticky = cuda_fail("plan launch", e);
+    q->stats.launches++;
+    q->stats.bytes += p->bytes;
+    return DDT_OK;
+}
+
+ddt_status_t ddt_plan_destroy(ddt_plan_t p) {
+    if (!p) return DDT_ERR_ARG;
+    {
+        DeviceGuard g(p->q->device);
+        cudaStreamSynchronize(p->q->stream);
+        cudaFree(p->table);
+    }
+    for (auto* t : p->types) type_release(t);
+    delete p;
+    return DDT_OK;
+}
+
 ddt_status_t ddt_queue_get_stats(ddt_queue_t q, ddt_queue_stats_t* out) {
     if (!q || !out) return DDT_ERR_ARG;
     *out = q->stats;

@@ -89,3 +89,29 @@ class Queue:
             self.destroy()
         except Exception:
             pass
+
+
+class Plan:
+    """A persistent fused batch: the queue's pending requests frozen into a
+    device work table uploaded once; launch() = one fused kernel (static-batch
+    replay, the 'fused + graph replay' arm of configs[4])."""
+
+    def __init__(self, queue: Queue):
+        self.queue = queue
+        out = P()
+        check(lib().ddt_plan_create(queue.handle, ctypes.byref(out)), "ddt_plan_create")
+        self._h = out
+
+    def launch(self):
+        check(lib().ddt_plan_launch(self._h), "ddt_plan_launch")
+
+    def destroy(self):
+        if self._h and self._h.value:
+            check(lib().ddt_plan_destroy(self._h), "ddt_plan_destroy")
+        self._h = P()
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass

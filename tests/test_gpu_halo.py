@@ -56,10 +56,12 @@ def _fill_interior(arrs, local, it, cfg):
         a[1:-1, 1:-1, 1:-1] = torch.from_numpy(vals).cuda()
 
 
-def _check(arrs, local, dirs):
+def _check(arrs, local, dirs, before=None):
     gm = ghost_mask(local, dirs)
-    for a in arrs:
+    for i, a in enumerate(arrs):
         h = a.cpu().numpy()
+        if before is not None:
+            assert np.array_equal(h[1:-1, 1:-1, 1:-1], before[i]), "interior modified by the exchange"
         exp = np.pad(h[1:-1, 1:-1, 1:-1], 1, mode="wrap")
         assert np.array_equal(h[gm], exp[gm]), "ghost cells differ from np.pad(wrap)"
         rest = ~gm
@@ -79,9 +81,10 @@ def test_halo_small(ddt, mode, graph, local, dirs, nvars, cfg):
     for it in range(4):
         _fill_interior(arrs, local, it, cfg)
         torch.cuda.synchronize()
+        before = [a[1:-1, 1:-1, 1:-1].cpu().numpy() for a in arrs]
         h.exchange()
         torch.cuda.synchronize()
-        _check(arrs, local, dirs)
+        _check(arrs, local, dirs, before)
     assert h.launches_per_exchange == (1 if mode == "p2p" else 2)
     h.destroy()
     comm.close()
@@ -97,9 +100,10 @@ def test_config2_face_halo_full_size(ddt, mode):
     for it in range(3):
         _fill_interior(arrs, local, it, 2)
         torch.cuda.synchronize()
+        before = [a[1:-1, 1:-1, 1:-1].cpu().numpy() for a in arrs]
         h.exchange()
         torch.cuda.synchronize()
-        _check(arrs, local, FACE_DIRS)
+        _check(arrs, local, FACE_DIRS, before)
     h.destroy()
     comm.close()
 
