@@ -154,6 +154,16 @@ ddt_status_t ddt_queue_destroy(ddt_queue_t q);
 int64_t ddt_pack_enqueue(ddt_queue_t q, ddt_type_t t, const void* src, int64_t count, void* dst_packed);
 int64_t ddt_unpack_enqueue(ddt_queue_t q, ddt_type_t t, const void* src_packed, int64_t count, void* dst);
 
+/* DirectIPC request ("a direct non-contiguous data transfer", fused with
+ * packing / unpacking in one kernel): gather `src_count` instances of
+ * `src_type` at `src` and scatter them as `dst_count` instances of `dst_type`
+ * at `dst`, with no packed intermediate.  The packed sizes must match
+ * (DDT_ERR_SIZE_MISMATCH) and dst_type must not overlap (DDT_ERR_OVERLAP).
+ * Both pointers are device pointers of the queue's device (or peer-mapped).
+ * Returns a uid >= 0 or a negative error, like the other enqueues.          */
+int64_t ddt_direct_enqueue(ddt_queue_t q, ddt_type_t src_type, const void* src, int64_t src_count,
+                           ddt_type_t dst_type, void* dst, int64_t dst_count);
+
 /* Scheduler (2): launch every pending request (Head..Tail) as ONE fused
  * kernel on the queue's stream (P:217, P:221, P:255 trigger (1)).  Returns
  * the number of requests launched (0 => nothing pending, no launch) or < 0. */

@@ -1,0 +1,100 @@
+// batch.cpp -- the work table in its two launch forms.
+//
+// The paper hands the fused kernel "an array of requests" (§IV-A.2) and
+// partitions thread blocks over requests by size (§IV-A.3).  Here the
+// partition is an exclusive prefix sum of per-request item counts
+// (kItemVecs vectors per item); the kernel maps item -> request by binary
+// search.  Batches of up to kParamLarge requests travel inside the kernel's
+// parameters, so ddt_flush is exactly one stream operation; larger batches are
+// serialised into a device table (one cudaMemcpyAsync per flush, or once for
+// persistent plans and halo plans).
+#include <algorithm>
+#include <cstring>
+
+#include "ddt_internal.h"
+
+namespace ddt {
+
+static uint32_t fill_prefix(uint32_t* prefix, const std::vector<ReqDesc>& d) {
+    uint64_t acc = 0;
+    for (size_t i = 0; i < d.size(); i++) {
+        prefix[i] = (uint32_t)acc;
+        acc += desc_items(d[i]);
+    }
+    prefix[d.size()] = (uint32_t)acc;
+    return (uint32_t)acc;
+}
+
+static size_t pad16(size_t v) { return (v + 15) & ~(size_t)15; }
+
+size_t device_table_bytes(const HostBatch& b) {
+    size_t n = b.descs.size();
+    size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
+    off += n * sizeof(ReqDesc) + b.aux.size() * sizeof(ReqDesc);
+    if (!b.xinfo.empty()) off += n * sizeof(XInfo);
+    return off;
+}
+
+uint32_t write_device_table(void* dst, const HostBatch& b) {
+    size_t n = b.descs.size();
+    auto* h = reinterpret_cast<BatchHeader*>(dst);
+    std::memset(h, 0, sizeof(*h));
+    auto* prefix = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(dst) + sizeof(BatchHeader));
+    uint32_t items = fill_prefix(prefix, b.descs);
+    size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
+    h->nreq = (uint32_t)n;
+    h->total_items = items;
+    h->desc_offset = (uint32_t)off;
+    std::memcpy(reinterpret_cast<char*>(dst) + off, b.descs.data(), n * sizeof(ReqDesc));
+    off += n * sizeof(ReqDesc);
+    h->aux_offset = (uint32_t)off;
+    h->naux = (uint32_t)b.aux.size();
+    if (!b.aux.empty()) std::memcpy(reinterpret_cast<char*>(dst) + off, b.aux.data(), b.aux.size() * sizeof(ReqDesc));
+    off += b.aux.size() * sizeof(ReqDesc);
+    if (!b.xinfo.empty()) {
+        h->xinfo_offset = (uint32_t)off;
+        std::memcpy(reinterpret_cast<char*>(dst) + off, b.xinfo.data(), n * sizeof(XInfo));
+    }
+    return items;
+}
+
+template <int CAP>
+static void to_param(const HostBatch& b, Launchable& out) {
+    out.blob.assign(sizeof(ParamBatch<CAP>), 0);
+    auto* p = reinterpret_cast<ParamBatch<CAP>*>(out.blob.data());
+    p->h.nreq = (uint32_t)b.descs.size();
+    p->h.total_items = fill_prefix(p->prefix, b.descs);
+    std::copy(b.descs.begin(), b.descs.end(), p->descs);
+    std::copy(b.aux.begin(), b.aux.end(), p->aux);
+    std::copy(b.xinfo.begin(), b.xinfo.end(), p->xinfo);
+    out.total_items = p->h.total_items;
+}
+
+void make_launchable(const HostBatch& b, bool allow_param, Launchable& out) {
+    size_t n = std::max(b.descs.size(), b.aux.size());
+    out.blob.clear();
+    if (allow_param && n <= (size_t)kParamSmall) {
+        out.form = 1;
+        to_param<kParamSmall>(b, out);
+    } else if (allow_param && n <= (size_t)kParamLarge) {
+        out.form = 2;
+        to_param<kParamLarge>(b, out);
+    } else {
+        out.form = 3;
+        std::vector<uint32_t> prefix(b.descs.size() + 1);
+        out.total_items = fill_prefix(prefix.data(), b.descs);
+    }
+}
+
+int launch_fused(const Launchable& l, void* stream, int grid_cap) {
+    const void* src = l.form == 3 ? l.dev : (const void*)l.blob.data();
+    return launch_fused_form(l.form, src, l.total_items, stream, grid_cap);
+}
+
+int launch_exchange(const Launchable& l, void* ctrl, int* err_flag_dev, uint64_t timeout_ns, void* stream,
+                    int grid_cap) {
+    const void* src = l.form == 3 ? l.dev : (const void*)l.blob.data();
+    return launch_exchange_form(l.form, src, l.total_items, ctrl, err_flag_dev, timeout_ns, stream, grid_cap);
+}
+
+}  // namespace ddt

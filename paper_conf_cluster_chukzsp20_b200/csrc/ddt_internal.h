@@ -96,20 +96,44 @@ inline int64_t type_extent(const ddt_type_s* t) { return t->ub - t->lb; }
 // ------------------------------------------------------------ kernels
 // Builds the u32 reciprocal for DivU32.
 DivU32 make_div(uint32_t d);
-// Fill a descriptor for one request; returns DDT_OK or an error.
+// Fill a descriptor for one request; max_lw caps the vector width (DIRECT
+// pairs share one width).  Returns DDT_OK or an error.
 ddt_status_t build_desc(ddt_type_s* t, const DeviceLayout* dl, int op, const void* noncontig,
-                        const void* packed, int64_t count, ReqDesc* out);
+                        const void* packed, int64_t count, ReqDesc* out, int max_lw = 4);
+// Build a DIRECT pair (source layout -> destination layout, equal packed sizes).
+ddt_status_t build_direct(ddt_type_s* ts, const DeviceLayout* dls, const void* src, int64_t scount, ddt_type_s* td,
+                          const DeviceLayout* dld, void* dst, int64_t dcount, ReqDesc* d, ReqDesc* a);
 // Items of a descriptor.
 inline uint32_t desc_items(const ReqDesc& d) {
     return (uint32_t)((d.nvec + (uint64_t)kItemVecs - 1) / (uint64_t)kItemVecs);
 }
-// Launch the fused kernel over a device batch table.  grid_cap <= 0 => default.
-int launch_fused(const void* dev_table, uint32_t total_items, void* stream, int grid_cap);
+
+// A batch on the host: descriptors (items come from these), DIRECT
+// destination layouts, and exchange side info (empty, or one per descriptor).
+struct HostBatch {
+    std::vector<ReqDesc> descs, aux;
+    std::vector<XInfo> xinfo;
+    void clear() { descs.clear(); aux.clear(); xinfo.clear(); }
+};
+// A batch ready to launch: carried in the kernel parameters (form 1 / 2) or
+// as a device table (form 3, `dev` owned by the caller).
+struct Launchable {
+    int form = 0;
+    std::vector<uint8_t> blob;  // ParamBatch<CAP> bytes (form 1 / 2)
+    void* dev = nullptr;        // device table (form 3)
+    uint32_t total_items = 0;
+};
+size_t device_table_bytes(const HostBatch& b);
+uint32_t write_device_table(void* dst, const HostBatch& b);
+// Param form if it fits (and allowed), else form 3 with `dev` left to the caller.
+void make_launchable(const HostBatch& b, bool allow_param, Launchable& out);
+int launch_fused(const Launchable& l, void* stream, int grid_cap);
+int launch_exchange(const Launchable& l, void* ctrl, int* err_flag_dev, uint64_t timeout_ns, void* stream,
+                    int grid_cap);
+int launch_fused_form(int form, const void* param_or_table, uint32_t total_items, void* stream, int grid_cap);
+int launch_exchange_form(int form, const void* param_or_table, uint32_t total_items, void* ctrl, int* err_flag_dev,
+                         uint64_t timeout_ns, void* stream, int grid_cap);
 int device_sm_count(int device);
-int launch_exchange(const void* dev_table, uint32_t total_items, void* ctrl, int* err_flag_dev, uint64_t timeout_ns,
-                    void* stream, int grid_cap);
-size_t table_bytes(size_t nreq);
-uint32_t write_table(void* dst, const ReqDesc* descs, size_t nreq);
 
 // queue accessors (queue.cpp)
 int queue_device(ddt_queue_s* q);

@@ -1,4 +1,4 @@
-// device_desc.h -- the device-side request descriptor and batch table.
+// device_desc.h -- the device-side request descriptor and batch tables.
 //
 // One descriptor = one request of the paper's request list (§IV-A.1 P:189-197:
 // UID, operation, origin/target buffer, cached layout entry) flattened into the
@@ -6,6 +6,13 @@
 // "array of requests" handed to the single fused kernel plus the work
 // table built by an exclusive prefix sum over per-request item counts (SURVEY
 // §8(a) a4), which maps every CTA work item to a (request, vector range) pair.
+//
+// A batch reaches the kernel in one of two forms:
+//   * ParamBatch<CAP>: small batches travel INSIDE the kernel's parameters
+//     (__grid_constant__, <= 32 KB on sm_70+ / CUDA >= 12.1): the flush is one
+//     stream operation and no dependent global load precedes the data loads;
+//   * a device table (BatchHeader | prefix | descs | aux | xinfo) uploaded with
+//     one cudaMemcpyAsync (flush) or once (persistent plans, halo plans).
 #pragma once
 #include <stdint.h>
 
@@ -16,7 +23,10 @@ constexpr int kThreads = 256;        // threads per CTA of the fused kernel
 constexpr int kUnroll = 4;           // vectors per thread per item (loads in flight)
 constexpr int kItemVecs = kThreads * kUnroll;  // vectors per work item
 
-enum DescOp : uint8_t { OP_PACK = 0, OP_UNPACK = 1 };
+// PACK: gather non-contiguous -> packed; UNPACK: packed -> scatter;
+// DIRECT: non-contiguous -> non-contiguous with a second layout (the paper's
+// DirectIPC op), used for self messages of a halo exchange.
+enum DescOp : uint8_t { OP_PACK = 0, OP_UNPACK = 1, OP_DIRECT = 2 };
 enum DescKind : uint8_t { K_STRIDED = 0, K_UNIFORM32 = 1, K_UNIFORM64 = 2, K_GENERAL = 3 };
 
 // Unsigned 32-bit division by a runtime constant d via a 64-bit reciprocal:
@@ -29,7 +39,7 @@ struct DivU32 {
 };
 
 struct alignas(16) ReqDesc {
-    uint64_t noncontig;     // non-contiguous side (pack: source, unpack: destination)
+    uint64_t noncontig;     // non-contiguous side (pack: source, unpack / direct-aux: destination)
     uint64_t packed;        // contiguous side     (pack: destination, unpack: source)
     uint32_t nvec;          // vectors in the request (count*size / w), < 2^32
     uint8_t op;             // DescOp
@@ -47,30 +57,48 @@ struct alignas(16) ReqDesc {
     uint64_t prefix;        // general: int64 exclusive packed prefix (nseg + 1 entries)
     uint32_t list_n;        // general: number of segments per instance
     uint32_t uid_lo;        // low bits of the request UID (debug / tracing)
-};
-
-// Header of a batch table in device memory:
-//   BatchHeader | uint32 item_prefix[nreq + 1] (padded to 16 B) | ReqDesc[nreq]
-struct alignas(16) BatchHeader {
-    uint32_t nreq;
-    uint32_t total_items;
-    uint32_t desc_offset;   // byte offset of ReqDesc[0] from the header
-    uint32_t pad;
+    uint32_t aux;           // DIRECT: index of the destination-layout descriptor in aux[]
+    uint32_t pad2;
 };
 
 // Exchange-only side info of a descriptor (fused P2P halo kernel).
 struct alignas(16) XInfo {
-    uint64_t flag;          // pack: peer's flag slot; unpack: own flag slot (u64 epoch)
+    uint64_t flag;          // pack: peer's flag slot; unpack: own flag slot (u64 epoch); 0 = none
     uint32_t counter;       // pack: index of the per-message completion counter
     uint32_t nitems;        // pack: items of the message (counter target = epoch * nitems)
     int64_t parity_stride;  // window half size: iteration e uses half (e & 1)
     int64_t pad;
 };
 
+// Header of a device batch table:
+//   BatchHeader | uint32 prefix[nreq + 1] (16 B padded) | ReqDesc[nreq] | ReqDesc aux[naux] | XInfo[nreq]?
+struct alignas(16) BatchHeader {
+    uint32_t nreq;
+    uint32_t total_items;
+    uint32_t desc_offset;   // byte offsets from the header
+    uint32_t aux_offset;
+    uint32_t xinfo_offset;  // 0 = no exchange info
+    uint32_t naux;
+    uint32_t pad[2];
+};
+
+// A small batch carried in the kernel parameters.
+template <int CAP>
+struct alignas(16) ParamBatch {
+    BatchHeader h;                 // offsets unused
+    uint32_t prefix[CAP + 4];
+    ReqDesc descs[CAP];
+    ReqDesc aux[CAP];
+    XInfo xinfo[CAP];
+};
+constexpr int kParamSmall = 8;
+constexpr int kParamLarge = 32;
+static_assert(sizeof(ParamBatch<kParamLarge>) <= 32000, "kernel parameter limit");
+
 // Control block of the fused exchange kernel (device memory, zeroed at create).
 struct XCtrl {
-    unsigned int ticket;          // next work item (reset by the last CTA to exit)
-    unsigned int done;            // CTAs finished
+    unsigned int done;            // CTAs finished (reset by the last CTA to exit)
+    unsigned int pad;
     unsigned long long epoch;     // completed exchanges
     unsigned long long counters[1];  // [nsend] monotonic per-message item counters
 };

@@ -1,18 +1,19 @@
-// fused_kernel.cu -- the single fused pack/unpack kernel (sm_100a).
+// fused_kernel.cu -- the single fused pack/unpack/direct kernel and the fused
+// P2P halo-exchange kernel (sm_100a).
 //
 // Paper §IV-A.3 (Fig. 6): one kernel executes an array of requests;
 // thread blocks are partitioned over requests by size and each runs the device
-// function of its request's operation (packing / unpacking), synchronising and
-// completing independently.  The paper used Cooperative Groups on V100 to give
-// small requests fewer threads.
+// function of its request's operation (packing / unpacking / DirectIPC),
+// synchronising and completing independently.  The paper used Cooperative
+// Groups on V100 to give small requests fewer threads.
 //
 // B200 design: pure HBM-bound byte movement, no tensor
 // cores.  The host builds a work table (exclusive prefix sum of per-request
-// item counts); every CTA walks items blockIdx.x,
-// blockIdx.x + gridDim.x, ... (grid = resident CTAs on 148 SMs), finds its
-// request with a binary search of the prefix, caches the descriptor in shared
-// memory, and moves kItemVecs vectors of the request's packed stream.  Lane i
-// of the CTA takes vectors v0 + i + u*kThreads, so the packed side is perfectly
+// item counts); CTA b walks items b, b + gridDim.x, ... in
+// increasing order (grid <= resident CTAs on the 148 SMs), finds its request
+// with a binary search of the prefix, caches the descriptor in shared memory
+// and moves kItemVecs vectors of the request's packed stream.  Thread i of the
+// CTA takes vectors v0 + i + u*kThreads, so the packed side is perfectly
 // coalesced and the strided side is coalesced within each segment.  The vector
 // width w (1..16 B) is the largest power of two dividing every segment offset,
 // segment length, both user pointers and (count > 1) the extent, so every
@@ -20,8 +21,9 @@
 // store (memory-level parallelism).  Vector -> byte offset uses only integer
 // arithmetic: 32-bit reciprocal division for the segment index and each
 // strided dim (closed form, no metadata), one table lookup for uniform lists,
-// one binary search for general lists.  Bytes are moved as integers (uint4,
-// uint2, ...): NaN payloads and -0.0 survive bit-exactly.
+// one binary search for general lists.  Bytes move as integers (uint4, uint2,
+// ...): NaN payloads and -0.0 survive bit-exactly.  Small batches arrive in the
+// kernel parameters (ParamBatch), large ones as a device table.
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -33,10 +35,13 @@ __device__ __forceinline__ uint32_t divu(uint32_t n, const DivU32& d) {
     return d.magic ? (uint32_t)__umul64hi((uint64_t)n, d.magic) : n;
 }
 
-// Vector width is a runtime, CTA-uniform property of the request (lw = log2 w).
-// One code path serves every width: the load / store below is a uniform
-// switch around a single instruction, so register allocation does not grow
-// with the number of (kind, width) combinations.
+// The vector width is a runtime, CTA-uniform property of the request
+// (lw = log2 w).  One code path serves every width: the load / store below is
+// a uniform switch around a single instruction, so register allocation does
+// not grow with the number of (kind, width) combinations.
+// NC: read-only data for the kernel's lifetime -> non-coherent path, no L1
+// allocation.  !NC: data another agent writes during the kernel (P2P window)
+// -> ld.global.cg (L2, coherent).
 template <bool NC>
 __device__ __forceinline__ uint4 ld_vec(const uint8_t* p, int lw) {
     uint4 r = make_uint4(0, 0, 0, 0);
@@ -125,27 +130,16 @@ __device__ __forceinline__ int64_t vec_offset(const ReqDesc& d, uint32_t v) {
     }
 }
 
-// COH: the packed side of an unpack is written by another GPU during this
-// kernel (P2P exchange) -> read it through L2 (ld.global.cg), never nc/L1.
-template <bool COH = false>
-__device__ __forceinline__ void run_desc(const ReqDesc& d, uint32_t v0) {
+// One work item: kItemVecs vectors starting at v0.  COH: the packed side of an
+// unpack is written by another GPU during this kernel.
+template <bool COH>
+__device__ __forceinline__ void run_desc(const ReqDesc& d, const ReqDesc& a, uint32_t v0) {
     const uint32_t nvec = d.nvec;
     const int lw = d.lw;
     uint8_t* nc = reinterpret_cast<uint8_t*>(d.noncontig);
     uint8_t* pk = reinterpret_cast<uint8_t*>(d.packed);
     uint4 buf[kUnroll];
-    if (d.op == OP_PACK) {
-#pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
-            uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-            if (v < nvec) buf[u] = ld_vec<true>(nc + vec_offset(d, v), lw);
-        }
-#pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
-            uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-            if (v < nvec) st_vec(pk + ((uint64_t)v << lw), lw, buf[u]);
-        }
-    } else {
+    if (d.op == OP_UNPACK) {
 #pragma unroll
         for (int u = 0; u < kUnroll; u++) {
             uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
@@ -156,6 +150,26 @@ __device__ __forceinline__ void run_desc(const ReqDesc& d, uint32_t v0) {
             uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
             if (v < nvec) st_vec(nc + vec_offset(d, v), lw, buf[u]);
         }
+        return;
+    }
+#pragma unroll
+    for (int u = 0; u < kUnroll; u++) {
+        uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+        if (v < nvec) buf[u] = ld_vec<true>(nc + vec_offset(d, v), lw);
+    }
+    if (d.op == OP_PACK) {
+#pragma unroll
+        for (int u = 0; u < kUnroll; u++) {
+            uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+            if (v < nvec) st_vec(pk + ((uint64_t)v << lw), lw, buf[u]);
+        }
+    } else {  // OP_DIRECT: scatter through the destination layout
+        uint8_t* dn = reinterpret_cast<uint8_t*>(a.noncontig);
+#pragma unroll
+        for (int u = 0; u < kUnroll; u++) {
+            uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+            if (v < nvec) st_vec(dn + vec_offset(a, v), lw, buf[u]);
+        }
     }
 }
 
@@ -164,47 +178,51 @@ __device__ __forceinline__ uint32_t find_request(const uint32_t* prefix, uint32_
     uint32_t lo = 0, hi = nreq;
     while (hi - lo > 1) {
         uint32_t mid = (lo + hi) >> 1;
-        if (__ldg(prefix + mid) <= item) lo = mid;
+        if (prefix[mid] <= item) lo = mid;
         else hi = mid;
     }
     return lo;
 }
 
-__global__ void __launch_bounds__(kThreads) ddt_fused_pack_unpack(const uint8_t* __restrict__ table) {
-    __shared__ ReqDesc sd;
-    const BatchHeader* h = reinterpret_cast<const BatchHeader*>(table);
-    const uint32_t nreq = h->nreq;
-    const uint32_t total = h->total_items;
-    const uint32_t* prefix = reinterpret_cast<const uint32_t*>(table + sizeof(BatchHeader));
-    const ReqDesc* descs = reinterpret_cast<const ReqDesc*>(table + h->desc_offset);
-    uint32_t cur = 0xffffffffu;
-    uint32_t cur_first = 0;
-    for (uint32_t item = blockIdx.x; item < total; item += gridDim.x) {
-        uint32_t r = find_request(prefix, nreq, item);
-        if (r != cur) {
-            __syncthreads();
-            constexpr int kWords = (int)(sizeof(ReqDesc) / 16);
-            if (threadIdx.x < kWords)
-                reinterpret_cast<uint4*>(&sd)[threadIdx.x] = __ldg(reinterpret_cast<const uint4*>(descs + r) + threadIdx.x);
-            cur_first = __ldg(prefix + r);
-            cur = r;
-            __syncthreads();
-        }
-        run_desc(sd, (item - cur_first) * (uint32_t)kItemVecs);
-    }
+struct TableView {
+    uint32_t nreq, total;
+    const uint32_t* prefix;
+    const ReqDesc* descs;
+    const ReqDesc* aux;
+    const XInfo* xinfo;
+};
+
+__device__ __forceinline__ TableView view_of(const uint8_t* t) {
+    const BatchHeader* h = reinterpret_cast<const BatchHeader*>(t);
+    TableView v;
+    v.nreq = h->nreq;
+    v.total = h->total_items;
+    v.prefix = reinterpret_cast<const uint32_t*>(t + sizeof(BatchHeader));
+    v.descs = reinterpret_cast<const ReqDesc*>(t + h->desc_offset);
+    v.aux = reinterpret_cast<const ReqDesc*>(t + h->aux_offset);
+    v.xinfo = h->xinfo_offset ? reinterpret_cast<const XInfo*>(t + h->xinfo_offset) : nullptr;
+    return v;
+}
+
+template <int CAP>
+__device__ __forceinline__ TableView view_of(const ParamBatch<CAP>& p) {
+    TableView v;
+    v.nreq = p.h.nreq;
+    v.total = p.h.total_items;
+    v.prefix = p.prefix;
+    v.descs = p.descs;
+    v.aux = p.aux;
+    v.xinfo = p.xinfo;
+    return v;
+}
+
+__device__ __forceinline__ void copy_words(void* dst, const void* src, int words, int tid0) {
+    int t = (int)threadIdx.x - tid0;
+    if (t >= 0 && t < words) reinterpret_cast<uint4*>(dst)[t] = reinterpret_cast<const uint4*>(src)[t];
 }
 
 // ------------------------------------------------------------------------
-// Fused P2P halo exchange: ONE kernel per iteration.
-// Pack items store straight into the peer's receive window over NVLink /
-// NVSwitch; the CTA completing the last item of a message releases the
-// message's epoch flag in the peer's window (the paper's "GPU thread signals
-// completion", across GPUs).  Unpack items wait (acquire, system
-// scope) on their message's flag and scatter as soon as it arrives -- the
-// receiver callback of §IV-B.2 done on the GPU, pack / transfer /
-// unpack fused into one launch.  Items are claimed through a global
-// ticket and every pack item precedes every unpack item, so pack work never
-// waits behind a spinning unpack CTA (deadlock freedom without co-residency).
+// P2P exchange signalling.
 __device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
     uint64_t v;
     asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
@@ -219,93 +237,129 @@ __device__ __forceinline__ uint64_t globaltimer() {
     return t;
 }
 
-__global__ void __launch_bounds__(kThreads)
-    ddt_fused_exchange(const uint8_t* __restrict__ table, XCtrl* ctrl, int* err_flag, uint64_t timeout_ns) {
+// The body shared by both kernels.  XCHG: pack items with a flag release the
+// message's epoch flag in the peer's window when the message is complete (the
+// paper's "GPU thread signals completion", across GPUs); unpack
+// items with a flag wait for it (the receiver callback of P:247, on the GPU).
+// Items are ordered [pack / direct ..., unpack ...] and every CTA walks its
+// items in increasing order, so a CTA only ever waits after finishing all of
+// its own pack items; with grid <= resident CTAs nothing waits on work that
+// cannot run (deadlock freedom without a global ticket).
+template <bool XCHG>
+__device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int* err_flag, uint64_t timeout_ns) {
     __shared__ ReqDesc sd;
+    __shared__ ReqDesc sa;
     __shared__ XInfo sx;
-    __shared__ uint32_t s_item;
     __shared__ uint64_t s_epoch;
     __shared__ int s_ok;
-    const BatchHeader* h = reinterpret_cast<const BatchHeader*>(table);
-    const uint32_t nreq = h->nreq;
-    const uint32_t total = h->total_items;
-    const uint32_t* prefix = reinterpret_cast<const uint32_t*>(table + sizeof(BatchHeader));
-    const ReqDesc* descs = reinterpret_cast<const ReqDesc*>(table + h->desc_offset);
-    const XInfo* xinfo = reinterpret_cast<const XInfo*>(descs + nreq);
-    if (threadIdx.x == 0) s_epoch = *reinterpret_cast<volatile unsigned long long*>(&ctrl->epoch) + 1ull;
-    __syncthreads();
-    const uint64_t epoch = s_epoch;
-    const uint64_t parity = epoch & 1ull;
-    uint32_t cur = 0xffffffffu, cur_first = 0;
-    for (;;) {
-        if (threadIdx.x == 0) s_item = atomicAdd(&ctrl->ticket, 1u);
+    uint64_t epoch = 0;
+    if constexpr (XCHG) {
+        if (threadIdx.x == 0) s_epoch = *reinterpret_cast<volatile unsigned long long*>(&ctrl->epoch) + 1ull;
         __syncthreads();
-        const uint32_t item = s_item;
-        if (item >= total) break;
-        uint32_t r = find_request(prefix, nreq, item);
+        epoch = s_epoch;
+    }
+    constexpr int kWords = (int)(sizeof(ReqDesc) / 16);
+    constexpr int kXWords = (int)(sizeof(XInfo) / 16);
+    uint32_t cur = 0xffffffffu, cur_first = 0;
+    for (uint32_t item = blockIdx.x; item < tv.total; item += gridDim.x) {
+        const uint32_t r = find_request(tv.prefix, tv.nreq, item);
         if (r != cur) {
-            constexpr int kWords = (int)(sizeof(ReqDesc) / 16);
-            constexpr int kXWords = (int)(sizeof(XInfo) / 16);
-            if (threadIdx.x < kWords)
-                reinterpret_cast<uint4*>(&sd)[threadIdx.x] = reinterpret_cast<const uint4*>(descs + r)[threadIdx.x];
-            else if (threadIdx.x < kWords + kXWords)
-                reinterpret_cast<uint4*>(&sx)[threadIdx.x - kWords] =
-                    reinterpret_cast<const uint4*>(xinfo + r)[threadIdx.x - kWords];
-            cur_first = prefix[r];
+            __syncthreads();  // every warp is done with the previous descriptor
+            copy_words(&sd, tv.descs + r, kWords, 0);
+            if constexpr (XCHG) copy_words(&sx, tv.xinfo + r, kXWords, 32);
+            __syncthreads();
+            if (sd.op == OP_DIRECT) {
+                copy_words(&sa, tv.aux + sd.aux, kWords, 0);
+                __syncthreads();
+            }
+            if constexpr (XCHG) {
+                if (sx.parity_stride) {
+                    if (threadIdx.x == 0) sd.packed += (epoch & 1ull) * (uint64_t)sx.parity_stride;
+                    __syncthreads();
+                }
+            }
+            cur_first = tv.prefix[r];
             cur = r;
-            __syncthreads();
-            if (threadIdx.x == 0) sd.packed += parity * (uint64_t)sx.parity_stride;  // double-buffered window
-            __syncthreads();
         }
-        const bool is_pack = sd.op == OP_PACK;
-        if (!is_pack) {
-            if (threadIdx.x == 0) {
-                const uint64_t* flag = reinterpret_cast<const uint64_t*>(sx.flag);
-                int ok = 1;
-                if (ld_acquire_sys(flag) < epoch) {
-                    const uint64_t t0 = globaltimer();
-                    while (ld_acquire_sys(flag) < epoch) {
-                        if (globaltimer() - t0 > timeout_ns) {
-                            ok = 0;
-                            *reinterpret_cast<volatile int*>(err_flag) = 1;
-                            __threadfence_system();
-                            break;
+        const uint32_t v0 = (item - cur_first) * (uint32_t)kItemVecs;
+        if constexpr (XCHG) {
+            if (sd.op == OP_UNPACK && sx.flag) {
+                if (threadIdx.x == 0) {
+                    const uint64_t* flag = reinterpret_cast<const uint64_t*>(sx.flag);
+                    int ok = 1;
+                    if (ld_acquire_sys(flag) < epoch) {
+                        const uint64_t t0 = globaltimer();
+                        while (ld_acquire_sys(flag) < epoch) {
+                            if (globaltimer() - t0 > timeout_ns) {
+                                ok = 0;
+                                *reinterpret_cast<volatile int*>(err_flag) = 1;
+                                __threadfence_system();
+                                break;
+                            }
+                            __nanosleep(32);
                         }
-                        __nanosleep(64);
+                    }
+                    s_ok = ok;
+                }
+                __syncthreads();
+                if (s_ok) run_desc<true>(sd, sa, v0);
+                continue;
+            }
+        }
+        run_desc<false>(sd, sa, v0);
+        if constexpr (XCHG) {
+            if (sd.op == OP_PACK && sx.flag) {
+                __syncthreads();  // the CTA's peer stores precede thread 0's release
+                if (threadIdx.x == 0) {
+                    if (sx.nitems == 1) {
+                        st_release_sys(reinterpret_cast<uint64_t*>(sx.flag), epoch);
+                    } else {
+                        __threadfence_system();
+                        unsigned long long old = atomicAdd_system(&ctrl->counters[sx.counter], 1ull);
+                        if (old + 1ull == epoch * (unsigned long long)sx.nitems) {
+                            __threadfence_system();
+                            st_release_sys(reinterpret_cast<uint64_t*>(sx.flag), epoch);
+                        }
                     }
                 }
-                s_ok = ok;
-            }
-            __syncthreads();
-            if (s_ok) run_desc<true>(sd, (item - cur_first) * (uint32_t)kItemVecs);
-        } else {
-            run_desc<false>(sd, (item - cur_first) * (uint32_t)kItemVecs);
-            __syncthreads();
-            if (threadIdx.x == 0) {
-                __threadfence_system();  // this CTA's peer stores before the count (release)
-                unsigned long long old = atomicAdd(&ctrl->counters[sx.counter], 1ull);
-                if (old + 1ull == epoch * (unsigned long long)sx.nitems) {
-                    __threadfence_system();  // acquire the other CTAs' stores, then publish
-                    st_release_sys(reinterpret_cast<uint64_t*>(sx.flag), epoch);
-                }
             }
         }
-        __syncthreads();
     }
-    if (threadIdx.x == 0) {
-        __threadfence();
-        unsigned int n = atomicAdd(&ctrl->done, 1u);
-        if (n == gridDim.x - 1) {
-            ctrl->ticket = 0;
-            ctrl->done = 0;
-            *reinterpret_cast<volatile unsigned long long*>(&ctrl->epoch) = epoch;
+    if constexpr (XCHG) {
+        __syncthreads();
+        if (threadIdx.x == 0) {
             __threadfence();
+            unsigned int n = atomicAdd(&ctrl->done, 1u);
+            if (n == gridDim.x - 1) {
+                ctrl->done = 0;
+                *reinterpret_cast<volatile unsigned long long*>(&ctrl->epoch) = epoch;
+                __threadfence();
+            }
         }
     }
 }
 
-static int g_blocks_per_sm = 0;
-static int g_xblocks_per_sm = 0;
+__global__ void __launch_bounds__(kThreads) ddt_fused_dev(const uint8_t* __restrict__ table) {
+    fused_body<false>(view_of(table), nullptr, nullptr, 0);
+}
+
+template <int CAP>
+__global__ void __launch_bounds__(kThreads) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
+    fused_body<false>(view_of(pb), nullptr, nullptr, 0);
+}
+
+__global__ void __launch_bounds__(kThreads)
+    ddt_exchange_dev(const uint8_t* __restrict__ table, XCtrl* ctrl, int* err_flag, uint64_t timeout_ns) {
+    fused_body<true>(view_of(table), ctrl, err_flag, timeout_ns);
+}
+
+template <int CAP>
+__global__ void __launch_bounds__(kThreads)
+    ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, XCtrl* ctrl, int* err_flag, uint64_t timeout_ns) {
+    fused_body<true>(view_of(pb), ctrl, err_flag, timeout_ns);
+}
+
+// ------------------------------------------------------------------ host side
 static int g_sm_count[64];
 
 int device_sm_count(int device) {
@@ -316,40 +370,61 @@ int device_sm_count(int device) {
     return n;
 }
 
-int launch_exchange(const void* dev_table, uint32_t total_items, void* ctrl, int* err_flag_dev, uint64_t timeout_ns,
-                    void* stream, int grid_cap) {
-    if (total_items == 0) return 0;
-    if (g_xblocks_per_sm == 0) {
+template <class K>
+static int resident_ctas(K kernel, int* cache) {
+    if (*cache == 0) {
         int b = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, ddt_fused_exchange, kThreads, 0) != cudaSuccess || b <= 0)
-            b = 4;
-        g_xblocks_per_sm = b;
+        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, kThreads, 0) != cudaSuccess || b <= 0) b = 1;
+        *cache = b;
     }
     int dev = 0;
     cudaGetDevice(&dev);
-    uint32_t cap = (uint32_t)(device_sm_count(dev) * g_xblocks_per_sm);
+    return *cache * device_sm_count(dev);
+}
+
+static uint32_t grid_for(uint32_t total, int resident, int grid_cap) {
+    uint32_t cap = (uint32_t)resident;
     if (grid_cap > 0 && (uint32_t)grid_cap < cap) cap = (uint32_t)grid_cap;
-    uint32_t grid = total_items < cap ? total_items : cap;
-    ddt_fused_exchange<<<grid, kThreads, 0, (cudaStream_t)stream>>>(reinterpret_cast<const uint8_t*>(dev_table),
-                                                                     reinterpret_cast<XCtrl*>(ctrl), err_flag_dev,
-                                                                     timeout_ns);
+    return total < cap ? total : cap;
+}
+
+// form: 1 = ParamBatch<kParamSmall>, 2 = ParamBatch<kParamLarge>, 3 = device table
+int launch_fused_form(int form, const void* param_or_table, uint32_t total_items, void* stream, int grid_cap) {
+    if (total_items == 0) return 0;
+    static int occ_dev = 0, occ_s = 0, occ_l = 0;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (form == 1) {
+        uint32_t g = grid_for(total_items, resident_ctas(ddt_fused_param<kParamSmall>, &occ_s), grid_cap);
+        ddt_fused_param<kParamSmall><<<g, kThreads, 0, s>>>(*reinterpret_cast<const ParamBatch<kParamSmall>*>(param_or_table));
+    } else if (form == 2) {
+        uint32_t g = grid_for(total_items, resident_ctas(ddt_fused_param<kParamLarge>, &occ_l), grid_cap);
+        ddt_fused_param<kParamLarge><<<g, kThreads, 0, s>>>(*reinterpret_cast<const ParamBatch<kParamLarge>*>(param_or_table));
+    } else {
+        uint32_t g = grid_for(total_items, resident_ctas(ddt_fused_dev, &occ_dev), grid_cap);
+        ddt_fused_dev<<<g, kThreads, 0, s>>>(reinterpret_cast<const uint8_t*>(param_or_table));
+    }
     return (int)cudaGetLastError();
 }
 
-int launch_fused(const void* dev_table, uint32_t total_items, void* stream, int grid_cap) {
+int launch_exchange_form(int form, const void* param_or_table, uint32_t total_items, void* ctrl, int* err_flag_dev,
+                         uint64_t timeout_ns, void* stream, int grid_cap) {
     if (total_items == 0) return 0;
-    if (g_blocks_per_sm == 0) {
-        int b = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, ddt_fused_pack_unpack, kThreads, 0) != cudaSuccess || b <= 0)
-            b = 4;
-        g_blocks_per_sm = b;
+    static int occ_dev = 0, occ_s = 0, occ_l = 0;
+    cudaStream_t s = (cudaStream_t)stream;
+    XCtrl* c = reinterpret_cast<XCtrl*>(ctrl);
+    if (form == 1) {
+        uint32_t g = grid_for(total_items, resident_ctas(ddt_exchange_param<kParamSmall>, &occ_s), grid_cap);
+        ddt_exchange_param<kParamSmall><<<g, kThreads, 0, s>>>(
+            *reinterpret_cast<const ParamBatch<kParamSmall>*>(param_or_table), c, err_flag_dev, timeout_ns);
+    } else if (form == 2) {
+        uint32_t g = grid_for(total_items, resident_ctas(ddt_exchange_param<kParamLarge>, &occ_l), grid_cap);
+        ddt_exchange_param<kParamLarge><<<g, kThreads, 0, s>>>(
+            *reinterpret_cast<const ParamBatch<kParamLarge>*>(param_or_table), c, err_flag_dev, timeout_ns);
+    } else {
+        uint32_t g = grid_for(total_items, resident_ctas(ddt_exchange_dev, &occ_dev), grid_cap);
+        ddt_exchange_dev<<<g, kThreads, 0, s>>>(reinterpret_cast<const uint8_t*>(param_or_table), c, err_flag_dev,
+                                                timeout_ns);
     }
-    int dev = 0;
-    cudaGetDevice(&dev);
-    uint32_t cap = (uint32_t)(device_sm_count(dev) * g_blocks_per_sm);
-    if (grid_cap > 0 && (uint32_t)grid_cap < cap) cap = (uint32_t)grid_cap;
-    uint32_t grid = total_items < cap ? total_items : cap;
-    ddt_fused_pack_unpack<<<grid, kThreads, 0, (cudaStream_t)stream>>>(reinterpret_cast<const uint8_t*>(dev_table));
     return (int)cudaGetLastError();
 }
 

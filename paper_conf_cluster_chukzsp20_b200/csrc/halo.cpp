@@ -101,13 +101,9 @@ struct ddt_halo_s {
     void* send_stage = nullptr;
     void* recv_stage = nullptr;
     std::vector<Xfer> xfers;
-    void* pack_table = nullptr;
-    uint32_t pack_items = 0;
-    void* unpack_table = nullptr;
-    uint32_t unpack_items = 0;
+    Launchable pack_l, unpack_l;  // NCCL mode: pack (+ direct self copies), unpack
     // P2P mode
-    void* xtable = nullptr;
-    uint32_t xitems = 0;
+    Launchable x_l;               // P2P mode: the single fused exchange kernel
     void* ctrl = nullptr;
     int* err_host = nullptr;
     int* err_dev = nullptr;
@@ -143,10 +139,14 @@ ddt_status_t upload(const std::vector<uint8_t>& host, void** dev) {
     return DDT_OK;
 }
 
-ddt_status_t make_table(const std::vector<ReqDesc>& d, void** dev, uint32_t* items) {
-    std::vector<uint8_t> host(table_bytes(d.size()));
-    *items = write_table(host.data(), d.data(), d.size());
-    return upload(host, dev);
+// Small batches ride in the kernel parameters (captured into the graph node);
+// larger ones are uploaded once as a device table.
+ddt_status_t make_table(const HostBatch& b, Launchable& l) {
+    make_launchable(b, true, l);
+    if (l.form != 3) return DDT_OK;
+    std::vector<uint8_t> host(device_table_bytes(b));
+    write_device_table(host.data(), b);
+    return upload(host, &l.dev);
 }
 
 // Exchange every receiver->sender directory over NCCL (nranks > 1), then agree
@@ -256,9 +256,9 @@ void free_halo(ddt_halo_s* h) {
     if (h->gexec) cudaGraphExecDestroy(h->gexec);
     cudaFree(h->send_stage);
     cudaFree(h->recv_stage);
-    cudaFree(h->pack_table);
-    cudaFree(h->unpack_table);
-    cudaFree(h->xtable);
+    cudaFree(h->pack_l.dev);
+    cudaFree(h->unpack_l.dev);
+    cudaFree(h->x_l.dev);
     cudaFree(h->ctrl);
     if (h->err_host) cudaFreeHost(h->err_host);
     for (auto& s : h->sends) type_release(s.type);
@@ -268,12 +268,12 @@ void free_halo(ddt_halo_s* h) {
 
 ddt_status_t record_exchange(ddt_halo_s* h) {
     if (h->mode == DDT_XCHG_P2P) {
-        int e = launch_exchange(h->xtable, h->xitems, h->ctrl, h->err_dev, h->timeout_ns, h->stream, h->grid_cap);
+        int e = launch_exchange(h->x_l, h->ctrl, h->err_dev, h->timeout_ns, h->stream, h->grid_cap);
         if (e) return cuda_fail("exchange kernel launch", e);
         return DDT_OK;
     }
-    if (h->pack_items) {
-        int e = launch_fused(h->pack_table, h->pack_items, h->stream, 0);
+    if (h->pack_l.total_items) {
+        int e = launch_fused(h->pack_l, h->stream, 0);
         if (e) return cuda_fail("pack launch", e);
     }
     bool remote = false;
@@ -295,8 +295,8 @@ ddt_status_t record_exchange(ddt_halo_s* h) {
         if (r == 0) r = r2;
         if (r != 0) return nccl_fail("halo send/recv", r);
     }
-    if (h->unpack_items) {
-        int e = launch_fused(h->unpack_table, h->unpack_items, h->stream, 0);
+    if (h->unpack_l.total_items) {
+        int e = launch_fused(h->unpack_l, h->stream, 0);
         if (e) return cuda_fail("unpack launch", e);
     }
     return DDT_OK;
@@ -433,12 +433,32 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     }
 
     // ---- build the device work tables
-    std::vector<ReqDesc> pack, unpack;
-    auto desc_for = [&](ddt_type_s* t, int op, const void* nc, const void* pk, int64_t count, ReqDesc* d) {
+    auto desc_for = [&](ddt_type_s* t, int op, const void* nc, const void* pk, int64_t count, ReqDesc* d) -> ddt_status_t {
         DeviceLayout* dl = nullptr;
         ddt_status_t s2 = type_device_layout(t, h->device, &dl);
         if (s2 != DDT_OK) return s2;
         return build_desc(t, dl, op, nc, pk, count, d);
+    };
+    // Self messages never touch a staging buffer or window: one DirectIPC
+    // descriptor gathers the send layout and scatters straight into the
+    // matching receive layout -- 2S instead of 4S HBM bytes.
+    auto self_recv = [&](int tag) {
+        for (int i = 0; i < nrecv; i++)
+            if (recvs[i].peer == c->rank && recvs[i].tag == tag) return i;
+        return -1;
+    };
+    auto add_direct = [&](HostBatch& b, const ddt_send_t& s, const ddt_recv_t& r, bool with_x) -> ddt_status_t {
+        DeviceLayout *dls = nullptr, *dld = nullptr;
+        ddt_status_t s2 = type_device_layout(s.type, h->device, &dls);
+        if (s2 == DDT_OK) s2 = type_device_layout(r.type, h->device, &dld);
+        ReqDesc d, a;
+        if (s2 == DDT_OK) s2 = build_direct(s.type, dls, s.buf, s.count, r.type, dld, r.buf, r.count, &d, &a);
+        if (s2 != DDT_OK) return s2;
+        d.aux = (uint32_t)b.aux.size();
+        b.aux.push_back(a);
+        b.descs.push_back(d);
+        if (with_x) b.xinfo.push_back(XInfo{});
+        return DDT_OK;
     };
     for (auto& s : h->sends) h->bytes += s.count * s.type->size;
     if (mode == DDT_XCHG_NCCL) {
@@ -463,9 +483,10 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             free_halo(h);
             return cuda_fail("cudaMalloc(staging)", e);
         }
-        // my receive spans per peer
+        // my receive spans per remote peer
         std::map<int, std::pair<int64_t, int64_t>> rspan;
         for (int i = 0; i < nrecv; i++) {
+            if (recvs[i].peer == c->rank) continue;
             int64_t a = RL.data_off[(size_t)i], b = a + recvs[i].count * recvs[i].type->size;
             auto it = rspan.find(recvs[i].peer);
             if (it == rspan.end()) rspan[recvs[i].peer] = {a, b};
@@ -479,70 +500,73 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             x.send_bytes = kv.second.second - kv.second.first;
         }
         for (auto& kv : rspan) {
-            if (kv.first == c->rank) continue;
             Xfer& x = xf[kv.first];
             x.peer = kv.first;
             x.recv_off = kv.second.first;
             x.recv_bytes = kv.second.second - kv.second.first;
         }
         for (auto& kv : xf) h->xfers.push_back(kv.second);
+        HostBatch packb, unpackb;
         for (int i = 0; i < nsend && st == DDT_OK; i++) {
             const auto& s = sends[i];
             if (s.count * s.type->size == 0) continue;
-            char* dst;
-            if (s.peer == c->rank) dst = (char*)h->recv_stage + match[(size_t)i]->data_off;
-            else dst = (char*)h->send_stage + region[s.peer] + (match[(size_t)i]->data_off - span[s.peer].first);
+            if (s.peer == c->rank) {
+                st = add_direct(packb, s, recvs[self_recv(s.tag)], false);
+                continue;
+            }
+            char* dst = (char*)h->send_stage + region[s.peer] + (match[(size_t)i]->data_off - span[s.peer].first);
             ReqDesc d;
             st = desc_for(s.type, OP_PACK, s.buf, dst, s.count, &d);
-            pack.push_back(d);
+            packb.descs.push_back(d);
         }
         for (int i = 0; i < nrecv && st == DDT_OK; i++) {
             const auto& r = recvs[i];
-            if (r.count * r.type->size == 0) continue;
+            if (r.count * r.type->size == 0 || r.peer == c->rank) continue;
             ReqDesc d;
             st = desc_for(r.type, OP_UNPACK, r.buf, (char*)h->recv_stage + RL.data_off[(size_t)i], r.count, &d);
-            unpack.push_back(d);
+            unpackb.descs.push_back(d);
         }
-        if (st == DDT_OK && !pack.empty()) st = make_table(pack, &h->pack_table, &h->pack_items);
-        if (st == DDT_OK && !unpack.empty()) st = make_table(unpack, &h->unpack_table, &h->unpack_items);
-        h->launches = (pack.empty() ? 0 : 1) + (unpack.empty() ? 0 : 1);
+        if (st == DDT_OK && !packb.descs.empty()) st = make_table(packb, h->pack_l);
+        if (st == DDT_OK && !unpackb.descs.empty()) st = make_table(unpackb, h->unpack_l);
+        h->launches = (packb.descs.empty() ? 0 : 1) + (unpackb.descs.empty() ? 0 : 1);
     } else {
-        // P2P: one table, pack descriptors first, then unpack descriptors
-        std::vector<XInfo> xi;
+        // P2P: one kernel; items ordered remote packs, self directs, then the
+        // unpacks that wait on flags (deadlock-freedom order, fused_kernel.cu)
+        HostBatch xb;
         char* mywin = (char*)c->peer_windows[c->rank];
+        uint32_t npack = 0;
         for (int i = 0; i < nsend && st == DDT_OK; i++) {
             const auto& s = sends[i];
-            if (s.count * s.type->size == 0) continue;
+            if (s.count * s.type->size == 0 || s.peer == c->rank) continue;
             const Directory& d = dirs[(size_t)s.peer];
             char* win = (char*)c->peer_windows[s.peer];
             ReqDesc rd;
             st = desc_for(s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, &rd);
             XInfo x{};
             x.flag = (uint64_t)(uintptr_t)(win + 8 * match[(size_t)i]->flag_idx);
-            x.counter = (uint32_t)pack.size();
+            x.counter = npack++;
             x.nitems = desc_items(rd);
             x.parity_stride = d.parity_stride;
-            pack.push_back(rd);
-            xi.push_back(x);
+            xb.descs.push_back(rd);
+            xb.xinfo.push_back(x);
         }
-        size_t npack = pack.size();
+        for (int i = 0; i < nsend && st == DDT_OK; i++) {
+            const auto& s = sends[i];
+            if (s.count * s.type->size == 0 || s.peer != c->rank) continue;
+            st = add_direct(xb, s, recvs[self_recv(s.tag)], true);
+        }
         for (int i = 0; i < nrecv && st == DDT_OK; i++) {
             const auto& r = recvs[i];
-            if (r.count * r.type->size == 0) continue;
+            if (r.count * r.type->size == 0 || r.peer == c->rank) continue;
             ReqDesc rd;
             st = desc_for(r.type, OP_UNPACK, r.buf, mywin + RL.flags_bytes + RL.data_off[(size_t)i], r.count, &rd);
             XInfo x{};
             x.flag = (uint64_t)(uintptr_t)(mywin + 8 * RL.flag_idx[(size_t)i]);
             x.parity_stride = RL.parity_stride;
-            pack.push_back(rd);
-            xi.push_back(x);
+            xb.descs.push_back(rd);
+            xb.xinfo.push_back(x);
         }
-        if (st == DDT_OK && !pack.empty()) {
-            std::vector<uint8_t> host(table_bytes(pack.size()) + xi.size() * sizeof(XInfo));
-            h->xitems = write_table(host.data(), pack.data(), pack.size());
-            std::memcpy(host.data() + table_bytes(pack.size()), xi.data(), xi.size() * sizeof(XInfo));
-            st = upload(host, &h->xtable);
-        }
+        if (st == DDT_OK && !xb.descs.empty()) st = make_table(xb, h->x_l);
         size_t ctrl_bytes = sizeof(XCtrl) + sizeof(unsigned long long) * std::max<size_t>(npack, 1);
         if (st == DDT_OK) {
             cudaError_t e = cudaMalloc(&h->ctrl, ctrl_bytes);
@@ -554,7 +578,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             }
             if (e != cudaSuccess) st = cuda_fail("exchange control block", e);
         }
-        h->launches = pack.empty() ? 0 : 1;
+        h->launches = xb.descs.empty() ? 0 : 1;
     }
     if (st == DDT_OK) {
         cudaError_t e = cudaDeviceSynchronize();

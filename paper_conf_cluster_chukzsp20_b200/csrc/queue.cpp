@@ -12,11 +12,13 @@
 //     status query by UID comparing request and response status.
 //   * a single host thread acts as scheduler.
 // B200 realisation: the ring holds host request records;
-// ddt_flush turns [flushed, Tail) into device descriptors plus an item prefix
-// sum (the work table), copies the table with one cudaMemcpyAsync and issues a
-// single launch; completion of a batch is a CUDA event recorded after the
-// launch (response status, reading R13/R15); ring entries are recycled once
-// their batch's event has fired.
+// every request's device descriptor is built at enqueue (O(1)); ddt_flush
+// turns [flushed, Tail) into a work table (item prefix sum) and issues ONE
+// launch -- batches of <= 32 requests ride in the kernel parameters (one stream
+// operation in total), larger ones are copied with one cudaMemcpyAsync first;
+// completion of a batch is a CUDA event recorded after the launch (response
+// status, readings R13/R15); ring entries are recycled once their batch's event
+// has fired.
 #include <algorithm>
 #include <cstring>
 #include <deque>
@@ -26,92 +28,6 @@
 
 #include "ddt_internal.h"
 
-namespace ddt {
-
-DivU32 make_div(uint32_t d) {
-    DivU32 r;
-    r.d = d;
-    r.pad = 0;
-    r.magic = d <= 1 ? 0ull : (~0ull) / d + 1ull;
-    return r;
-}
-
-static int lowbit16(uint64_t v) {
-    if (v == 0) return 16;
-    uint64_t a = v & (~v + 1);
-    return a > 16 ? 16 : (int)a;
-}
-
-static uint64_t uabs64(int64_t v) { return v < 0 ? (uint64_t)(-(v + 1)) + 1 : (uint64_t)v; }
-
-ddt_status_t build_desc(ddt_type_s* t, const DeviceLayout* dl, int op, const void* noncontig, const void* packed,
-                        int64_t count, ReqDesc* d) {
-    const Layout& L = t->layout;
-    std::memset(d, 0, sizeof(*d));
-    int64_t bytes = count * t->size;
-    int64_t ext = type_extent(t);
-    int w = L.align;
-    w = std::min(w, lowbit16((uint64_t)(uintptr_t)noncontig));
-    w = std::min(w, lowbit16((uint64_t)(uintptr_t)packed));
-    if (count > 1) w = std::min(w, lowbit16(uabs64(ext)));
-    int lw = 0;
-    while ((1 << lw) < w) lw++;
-    uint64_t nvec = (uint64_t)bytes >> lw;
-    if (nvec >= (1ull << 32)) {
-        set_error("request too large for one descriptor (>= 2^32 vectors)");
-        return DDT_ERR_UNSUPPORTED;
-    }
-    d->noncontig = (uint64_t)(uintptr_t)noncontig;
-    d->packed = (uint64_t)(uintptr_t)packed;
-    d->nvec = (uint32_t)nvec;
-    d->op = (uint8_t)op;
-    d->lw = (uint8_t)lw;
-    d->extent = ext;
-    if (L.kind == DDT_LAYOUT_STRIDED) {
-        Form f = L.form;
-        f.dims.insert(f.dims.begin(), Dim{count, ext});
-        normalize(f);
-        d->kind = K_STRIDED;
-        d->base = f.base;
-        d->vps = make_div((uint32_t)(f.seg_len >> lw));
-        if (f.dims.empty()) {
-            d->ndim = 0;
-            d->extent = 0;
-        } else {
-            int D = (int)f.dims.size();
-            if (D - 1 > kMaxDims) {
-                set_error("strided layout with too many dims after count folding");
-                return DDT_ERR_UNSUPPORTED;
-            }
-            d->ndim = (uint8_t)(D - 1);
-            // innermost first; the outermost dim is the final quotient
-            for (int k = 0; k < D - 1; k++) {
-                const Dim& x = f.dims[(size_t)(D - 1 - k)];
-                d->radix[k] = make_div((uint32_t)x.n);
-                d->stride[k] = x.stride;
-            }
-            d->extent = f.dims[0].stride;
-        }
-    } else if (L.kind == DDT_LAYOUT_UNIFORM_LIST) {
-        d->kind = L.off32 ? K_UNIFORM32 : K_UNIFORM64;
-        d->vps = make_div((uint32_t)(L.seg_len >> lw));
-        d->nseg = make_div((uint32_t)L.nseg);
-        d->list = (uint64_t)(uintptr_t)dl->offsets;
-    } else if (L.kind == DDT_LAYOUT_GENERAL_LIST) {
-        d->kind = K_GENERAL;
-        d->vps = make_div((uint32_t)(t->size >> lw));  // vectors per instance
-        d->list = (uint64_t)(uintptr_t)dl->offsets;
-        d->lens = (uint64_t)(uintptr_t)dl->lens;
-        d->prefix = (uint64_t)(uintptr_t)dl->prefix;
-        d->list_n = (uint32_t)L.nseg;
-    } else {
-        return DDT_ERR_STATE;
-    }
-    return DDT_OK;
-}
-
-}  // namespace ddt
-
 using namespace ddt;
 
 struct ddt_queue_s {
@@ -119,11 +35,10 @@ struct ddt_queue_s {
         int64_t uid;
         int op;
         ddt_type_s* t;
-        const void* src;
-        void* dst;
-        int64_t count;
+        ddt_type_s* t2;  // DIRECT destination type (else nullptr)
         int64_t bytes;
-        ReqDesc desc;  // built at enqueue (O(1)); flush only serializes
+        ReqDesc desc;    // built at enqueue (O(1)); flush only serializes
+        ReqDesc aux;     // DIRECT destination layout
     };
     struct Batch {
         int64_t first, end;  // uid range
@@ -149,7 +64,8 @@ struct ddt_queue_s {
     ddt_status_t sticky = DDT_OK;
     ddt_queue_stats_t stats{};
     int sm_count = 148;
-    std::vector<ReqDesc> scratch;
+    HostBatch scratch;
+    Launchable launch;
 };
 
 namespace {
@@ -178,21 +94,51 @@ cudaEvent_t get_event(ddt_queue_s* q) {
     return e;
 }
 
+void release_req(ddt_queue_s::Req& r) {
+    type_release(r.t);
+    type_release(r.t2);
+    r.t = r.t2 = nullptr;
+}
+
 void reclaim(ddt_queue_s* q, bool block) {
     while (!q->inflight.empty()) {
         auto& b = q->inflight.front();
         cudaError_t e = block ? cudaEventSynchronize(b.ev) : cudaEventQuery(b.ev);
         if (e == cudaErrorNotReady) return;
         if (e != cudaSuccess && q->sticky == DDT_OK) q->sticky = cuda_fail("batch completion", e);
-        for (int64_t u = b.first; u < b.end; u++) {
-            auto& r = q->ring[(size_t)(u % q->capacity)];
-            type_release(r.t);
-            r.t = nullptr;
-        }
+        for (int64_t u = b.first; u < b.end; u++) release_req(q->ring[(size_t)(u % q->capacity)]);
         q->head = b.end;
         q->event_pool.push_back(b.ev);
         q->inflight.pop_front();
     }
+}
+
+// Scheduler (1): claim the Tail slot (or fail with the paper's negative UID).
+int64_t claim(ddt_queue_s* q) {
+    if (q->tail - q->head >= q->capacity) {
+        DeviceGuard g(q->device);
+        reclaim(q, false);
+        if (q->tail - q->head >= q->capacity) return DDT_ERR_QUEUE_FULL;  // negative UID (P:215)
+    }
+    return q->tail;
+}
+
+int64_t commit_req(ddt_queue_s* q, int op, ddt_type_s* t, ddt_type_s* t2, int64_t bytes, const ReqDesc& d,
+                   const ReqDesc* a) {
+    int64_t uid = q->tail++;
+    auto& r = q->ring[(size_t)(uid % q->capacity)];
+    r.uid = uid;
+    r.op = op;
+    r.t = t;
+    r.t2 = t2;
+    type_retain(t);
+    type_retain(t2);
+    r.bytes = bytes;
+    r.desc = d;
+    r.desc.uid_lo = (uint32_t)uid;
+    if (a) r.aux = *a;
+    q->stats.requests++;
+    return uid;
 }
 
 int64_t enqueue(ddt_queue_s* q, int op, ddt_type_s* t, const void* src, int64_t count, void* dst) {
@@ -202,12 +148,10 @@ int64_t enqueue(ddt_queue_s* q, int op, ddt_type_s* t, const void* src, int64_t 
     int64_t bytes = count * t->size;
     if (bytes > 0 && (!src || !dst)) return DDT_ERR_ARG;
     if (op == OP_UNPACK && bytes > 0 && t->layout.overlaps) return DDT_ERR_OVERLAP;
-    if (q->tail - q->head >= q->capacity) {
-        DeviceGuard g(q->device);
-        reclaim(q, false);
-        if (q->tail - q->head >= q->capacity) return DDT_ERR_QUEUE_FULL;  // negative UID (P:215)
-    }
+    int64_t c = claim(q);
+    if (c < 0) return c;
     ReqDesc desc;
+    std::memset(&desc, 0, sizeof(desc));
     if (bytes > 0) {
         DeviceGuard g(q->device);
         DeviceLayout* dl = nullptr;
@@ -218,20 +162,7 @@ int64_t enqueue(ddt_queue_s* q, int op, ddt_type_s* t, const void* src, int64_t 
         s = build_desc(t, dl, op, nc, pk, count, &desc);
         if (s != DDT_OK) return s;
     }
-    int64_t uid = q->tail++;
-    auto& r = q->ring[(size_t)(uid % q->capacity)];
-    r.desc = desc;
-    r.desc.uid_lo = (uint32_t)uid;
-    r.uid = uid;
-    r.op = op;
-    r.t = t;
-    type_retain(t);
-    r.src = src;
-    r.dst = dst;
-    r.count = count;
-    r.bytes = bytes;
-    q->stats.requests++;
-    return uid;
+    return commit_req(q, op, t, nullptr, bytes, desc, nullptr);
 }
 
 ddt_status_t ensure_host_slot(ddt_queue_s* q, size_t bytes, ddt_queue_s::HostSlot** out) {
@@ -257,32 +188,26 @@ ddt_status_t ensure_host_slot(ddt_queue_s* q, size_t bytes, ddt_queue_s::HostSlo
     return DDT_OK;
 }
 
-}  // namespace
-
-namespace ddt {
-// Serialize a batch table: header | item prefix | descriptors.
-size_t table_bytes(size_t nreq) {
-    size_t pre = ((nreq + 1) * 4 + 15) & ~(size_t)15;
-    return sizeof(BatchHeader) + pre + nreq * sizeof(ReqDesc);
-}
-uint32_t write_table(void* dst, const ReqDesc* descs, size_t nreq) {
-    auto* h = (BatchHeader*)dst;
-    size_t pre = ((nreq + 1) * 4 + 15) & ~(size_t)15;
-    auto* prefix = (uint32_t*)((char*)dst + sizeof(BatchHeader));
-    uint64_t acc = 0;
-    for (size_t i = 0; i < nreq; i++) {
-        prefix[i] = (uint32_t)acc;
-        acc += desc_items(descs[i]);
+// Gather the pending requests' descriptors into q->scratch.
+int64_t gather_pending(ddt_queue_s* q) {
+    HostBatch& b = q->scratch;
+    b.clear();
+    int64_t moved = 0;
+    for (int64_t u = q->flushed; u < q->tail; u++) {
+        auto& r = q->ring[(size_t)(u % q->capacity)];
+        if (r.bytes == 0) continue;
+        ReqDesc d = r.desc;
+        if (r.op == OP_DIRECT) {
+            d.aux = (uint32_t)b.aux.size();
+            b.aux.push_back(r.aux);
+        }
+        b.descs.push_back(d);
+        moved += r.bytes;
     }
-    prefix[nreq] = (uint32_t)acc;
-    h->nreq = (uint32_t)nreq;
-    h->total_items = (uint32_t)acc;
-    h->desc_offset = (uint32_t)(sizeof(BatchHeader) + pre);
-    h->pad = 0;
-    std::memcpy((char*)dst + h->desc_offset, descs, nreq * sizeof(ReqDesc));
-    return (uint32_t)acc;
+    return moved;
 }
-}  // namespace ddt
+
+}  // namespace
 
 extern "C" {
 
@@ -320,7 +245,7 @@ ddt_status_t ddt_queue_destroy(ddt_queue_t q) {
     {
         DeviceGuard g(q->device);
         reclaim(q, true);
-        for (int64_t u = q->flushed; u < q->tail; u++) type_release(q->ring[(size_t)(u % q->capacity)].t);
+        for (int64_t u = q->flushed; u < q->tail; u++) release_req(q->ring[(size_t)(u % q->capacity)]);
         for (auto e : q->event_pool) cudaEventDestroy(e);
         for (auto& s : q->slots) {
             if (s.p) cudaFreeHost(s.p);
@@ -340,43 +265,65 @@ int64_t ddt_unpack_enqueue(ddt_queue_t q, ddt_type_t t, const void* src_packed, 
     return enqueue(q, OP_UNPACK, t, src_packed, count, dst);
 }
 
+int64_t ddt_direct_enqueue(ddt_queue_t q, ddt_type_t src_type, const void* src, int64_t src_count,
+                           ddt_type_t dst_type, void* dst, int64_t dst_count) {
+    if (!q || !src_type || !dst_type || src_count < 0 || dst_count < 0) return DDT_ERR_ARG;
+    if (q->sticky != DDT_OK) return q->sticky;
+    if (!src_type->committed || !dst_type->committed) return DDT_ERR_STATE;
+    int64_t bytes = src_count * src_type->size;
+    if (bytes != dst_count * dst_type->size) return DDT_ERR_SIZE_MISMATCH;
+    if (bytes > 0 && (!src || !dst)) return DDT_ERR_ARG;
+    if (bytes > 0 && dst_type->layout.overlaps) return DDT_ERR_OVERLAP;
+    int64_t c = claim(q);
+    if (c < 0) return c;
+    ReqDesc d, a;
+    std::memset(&d, 0, sizeof(d));
+    std::memset(&a, 0, sizeof(a));
+    if (bytes > 0) {
+        DeviceGuard g(q->device);
+        DeviceLayout *dls = nullptr, *dld = nullptr;
+        ddt_status_t s = type_device_layout(src_type, q->device, &dls);
+        if (s == DDT_OK) s = type_device_layout(dst_type, q->device, &dld);
+        if (s == DDT_OK) s = build_direct(src_type, dls, src, src_count, dst_type, dld, dst, dst_count, &d, &a);
+        if (s != DDT_OK) return s;
+    }
+    return commit_req(q, OP_DIRECT, src_type, dst_type, bytes, d, &a);
+}
+
 int32_t ddt_flush(ddt_queue_t q) {
     if (!q) return DDT_ERR_ARG;
     if (q->sticky != DDT_OK) return q->sticky;
     if (q->flushed == q->tail) return 0;
     DeviceGuard g(q->device);
-    auto& descs = q->scratch;
-    descs.clear();
-    int64_t moved = 0;
-    for (int64_t u = q->flushed; u < q->tail; u++) {
-        auto& r = q->ring[(size_t)(u % q->capacity)];
-        if (r.bytes == 0) continue;
-        descs.push_back(r.desc);
-        moved += r.bytes;
-    }
+    int64_t moved = gather_pending(q);
     int32_t nflushed = (int32_t)(q->tail - q->flushed);
-    if (!descs.empty()) {
-        size_t tb = table_bytes(descs.size());
-        ddt_queue_s::HostSlot* slot = nullptr;
-        ddt_status_t s = ensure_host_slot(q, tb, &slot);
-        if (s != DDT_OK) return q->sticky = s;
-        uint32_t items = write_table(slot->p, descs.data(), descs.size());
-        if (q->dev_cap < tb) {
-            if (q->dev_table) cudaFree(q->dev_table);  // synchronizes: old table no longer in use
-            size_t cap = std::max<size_t>(tb, 64 << 10);
-            cudaError_t e = cudaMalloc(&q->dev_table, cap);
-            if (e != cudaSuccess) {
-                q->dev_table = nullptr;
-                q->dev_cap = 0;
-                return q->sticky = cuda_fail("cudaMalloc(table)", e);
+    if (!q->scratch.descs.empty()) {
+        Launchable& L = q->launch;
+        make_launchable(q->scratch, true, L);
+        if (L.form == 3) {
+            size_t tb = device_table_bytes(q->scratch);
+            ddt_queue_s::HostSlot* slot = nullptr;
+            ddt_status_t s = ensure_host_slot(q, tb, &slot);
+            if (s != DDT_OK) return q->sticky = s;
+            write_device_table(slot->p, q->scratch);
+            if (q->dev_cap < tb) {
+                if (q->dev_table) cudaFree(q->dev_table);  // synchronizes: old table no longer in use
+                size_t cap = std::max<size_t>(tb, 64 << 10);
+                cudaError_t e = cudaMalloc(&q->dev_table, cap);
+                if (e != cudaSuccess) {
+                    q->dev_table = nullptr;
+                    q->dev_cap = 0;
+                    return q->sticky = cuda_fail("cudaMalloc(table)", e);
+                }
+                q->dev_cap = cap;
             }
-            q->dev_cap = cap;
+            cudaError_t e = cudaMemcpyAsync(q->dev_table, slot->p, tb, cudaMemcpyHostToDevice, q->stream);
+            if (e != cudaSuccess) return q->sticky = cuda_fail("table upload", e);
+            cudaEventRecord(slot->ev, q->stream);
+            slot->used = true;
+            L.dev = q->dev_table;
         }
-        cudaError_t e = cudaMemcpyAsync(q->dev_table, slot->p, tb, cudaMemcpyHostToDevice, q->stream);
-        if (e != cudaSuccess) return q->sticky = cuda_fail("table upload", e);
-        cudaEventRecord(slot->ev, q->stream);
-        slot->used = true;
-        int le = launch_fused(q->dev_table, items, q->stream, 0);
+        int le = launch_fused(L, q->stream, 0);
         if (le != 0) return q->sticky = cuda_fail("fused kernel launch", le);
         q->stats.launches++;
         q->stats.bytes += moved;
@@ -433,8 +380,7 @@ ddt_status_t ddt_wait(ddt_queue_t q) {
 
 struct ddt_plan_s {
     ddt_queue_s* q = nullptr;
-    void* table = nullptr;
-    uint32_t items = 0;
+    Launchable launch;
     int64_t bytes = 0;
     std::vector<ddt_type_s*> types;
 };
@@ -448,25 +394,29 @@ ddt_status_t ddt_plan_create(ddt_queue_t q, ddt_plan_t* out) {
     auto* p = new (std::nothrow) ddt_plan_s();
     if (!p) return DDT_ERR_NOMEM;
     p->q = q;
-    std::vector<ReqDesc> descs;
+    p->bytes = gather_pending(q);
     for (int64_t u = q->flushed; u < q->tail; u++) {
         auto& r = q->ring[(size_t)(u % q->capacity)];
         if (r.bytes == 0) continue;
-        descs.push_back(r.desc);
-        p->bytes += r.bytes;
-        type_retain(r.t);
-        p->types.push_back(r.t);
+        for (ddt_type_s* t : {r.t, r.t2})
+            if (t) {
+                type_retain(t);
+                p->types.push_back(t);
+            }
     }
-    if (!descs.empty()) {
-        std::vector<uint8_t> host(table_bytes(descs.size()));
-        p->items = write_table(host.data(), descs.data(), descs.size());
-        cudaError_t e = cudaMalloc(&p->table, host.size());
-        if (e == cudaSuccess) e = cudaMemcpy(p->table, host.data(), host.size(), cudaMemcpyHostToDevice);
-        if (e != cudaSuccess) {
-            for (auto* t : p->types) type_release(t);
-            cudaFree(p->table);
-            delete p;
-            return cuda_fail("plan table", e);
+    if (!q->scratch.descs.empty()) {
+        make_launchable(q->scratch, true, p->launch);
+        if (p->launch.form == 3) {
+            std::vector<uint8_t> host(device_table_bytes(q->scratch));
+            write_device_table(host.data(), q->scratch);
+            cudaError_t e = cudaMalloc(&p->launch.dev, host.size());
+            if (e == cudaSuccess) e = cudaMemcpy(p->launch.dev, host.data(), host.size(), cudaMemcpyHostToDevice);
+            if (e != cudaSuccess) {
+                for (auto* t : p->types) type_release(t);
+                cudaFree(p->launch.dev);
+                delete p;
+                return cuda_fail("plan table", e);
+            }
         }
     }
     // the moved requests complete in the request list without a launch
@@ -482,9 +432,9 @@ ddt_status_t ddt_plan_launch(ddt_plan_t p) {
     if (!p) return DDT_ERR_ARG;
     ddt_queue_s* q = p->q;
     if (q->sticky != DDT_OK) return q->sticky;
-    if (!p->items) return DDT_OK;
+    if (!p->launch.total_items) return DDT_OK;
     DeviceGuard g(q->device);
-    int e = launch_fused(p->table, p->items, q->stream, 0);
+    int e = launch_fused(p->launch, q->stream, 0);
     if (e) return q->sticky = cuda_fail("plan launch", e);
     q->stats.launches++;
     q->stats.bytes += p->bytes;
@@ -496,7 +446,7 @@ ddt_status_t ddt_plan_destroy(ddt_plan_t p) {
     {
         DeviceGuard g(p->q->device);
         cudaStreamSynchronize(p->q->stream);
-        cudaFree(p->table);
+        if (p->launch.dev) cudaFree(p->launch.dev);
     }
     for (auto* t : p->types) type_release(t);
     delete p;

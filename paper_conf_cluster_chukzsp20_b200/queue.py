@@ -56,6 +56,13 @@ class Queue:
         return check(lib().ddt_unpack_enqueue(self._h, t.handle, ctypes.c_void_p(ptr_of(src_packed)), int(count),
                                               ctypes.c_void_p(ptr_of(dst))), "ddt_unpack_enqueue")
 
+    def direct(self, src_type, src, src_count: int, dst_type, dst, dst_count: int) -> int:
+        """Enqueue a DirectIPC request: gather through src_type, scatter through
+        dst_type, no packed intermediate."""
+        return check(lib().ddt_direct_enqueue(self._h, src_type.handle, ctypes.c_void_p(ptr_of(src)), int(src_count),
+                                              dst_type.handle, ctypes.c_void_p(ptr_of(dst)), int(dst_count)),
+                     "ddt_direct_enqueue")
+
     def try_pack(self, t, src, count, dst_packed) -> int:
         """Like pack() but returns the negative status instead of raising."""
         return lib().ddt_pack_enqueue(self._h, t.handle, ctypes.c_void_p(ptr_of(src)), int(count),

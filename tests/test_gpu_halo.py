@@ -85,7 +85,7 @@ def test_halo_small(ddt, mode, graph, local, dirs, nvars, cfg):
         h.exchange()
         torch.cuda.synchronize()
         _check(arrs, local, dirs, before)
-    assert h.launches_per_exchange == (1 if mode == "p2p" else 2)
+    assert h.launches_per_exchange == 1  # P = 1: every message is a self message -> one DirectIPC launch
     h.destroy()
     comm.close()
 

@@ -231,3 +231,79 @@ def test_nan_and_negative_zero_survive(ddt, q):
     q.wait()
     exp = oracle.pack(oracle.Type(("vector", 60, 2, 4, ("basic", "double"))), vals.view(np.uint8))
     assert_bytes_equal(host(d), exp, "nan payloads")
+
+
+# --------------------------------------------------------------- launch forms, DirectIPC, plans
+@pytest.mark.parametrize("n", [1, 5, 8, 9, 20, 32, 33, 70])
+def test_batch_forms_param_and_device_table(ddt, q, n):
+    """Batches of <= 8 / <= 32 requests ride in the kernel parameters, larger
+    ones in a device table: all three forms are bit-exact and one launch."""
+    rng = np.random.default_rng(n)
+    specs = [config1_spec(), ("subarray", [7, 8, 9], [2, 8, 3], [4, 0, 5], "C", ("basic", "float")),
+             ("hindexed", [2, 5, 1], [3, 40, 17], ("basic", "byte"))]
+    cases = [Case(ddt, specs[i % 3], count=int(rng.integers(1, 3)), misalign=int(rng.integers(0, 8)), seed=50 + i)
+             for i in range(n)]
+    outs = [c.gpu_pack(q) for c in cases]
+    l0 = q.stats()["launches"]
+    assert q.flush() == n
+    q.wait()
+    assert q.stats()["launches"] - l0 == 1
+    for c, (_, _, d) in zip(cases, outs):
+        assert_bytes_equal(host(d), c.expect_pack(), f"form n={n}")
+
+
+@pytest.mark.parametrize("mis_s,mis_d", [(0, 0), (8, 0), (4, 12), (1, 3)])
+def test_direct_enqueue_equals_unpack_of_pack(ddt, q, mis_s, mis_d):
+    """DirectIPC: one gather->scatter pass == oracle unpack(pack(x))."""
+    import torch
+    pairs = [(("subarray", [10, 11, 12], [8, 9, 1], [1, 1, 10], "C", ("basic", "double")),
+              ("subarray", [10, 11, 12], [8, 9, 1], [1, 1, 0], "C", ("basic", "double"))),
+             (("vector", 72, 1, 3, ("basic", "double")), ("subarray", [12, 12], [8, 9], [2, 1], "F", ("basic", "double"))),
+             (config3_spec(nblocks=500, npoints=4096)[0], ("vector", 500, 3, 5, ("basic", "float")))]
+    for ss, ds in pairs:
+        os_, od = oracle.Type(ss), oracle.Type(ds)
+        assert os_.size == od.size
+        ts, td = ddt.Type.from_spec(ss), ddt.Type.from_spec(ds)
+        _, shi = os_.footprint()
+        _, dhi = od.footprint()
+        src = random_bytes(shi + 64, 9)
+        s = cuda_bytes(src)
+        d = torch.full((dhi + 64,), SENTINEL, dtype=torch.uint8, device="cuda")
+        q.direct(ts, (s, mis_s), 1, td, (d, mis_d), 1)
+        q.wait()
+        exp = np.full(dhi + 64, SENTINEL, np.uint8)
+        oracle.unpack(od, oracle.pack(os_, src, 1, mis_s), exp, 1, mis_d)
+        assert_bytes_equal(host(d), exp, f"direct {ss[0]}->{ds[0]}")
+
+
+def test_direct_size_mismatch_rejected(ddt, q):
+    from paper_conf_cluster_chukzsp20_b200 import DDTError
+    a = ddt.Type.from_spec(("vector", 4, 1, 2, ("basic", "double")))
+    b = ddt.Type.from_spec(("vector", 3, 1, 2, ("basic", "double")))
+    with pytest.raises(DDTError) as e:
+        q.direct(a, 256, 1, b, 512, 1)
+    assert e.value.code == -8
+
+
+@pytest.mark.parametrize("n", [3, 40])
+def test_plan_replay(ddt, q, n):
+    """A persistent plan relaunches the same fused batch; results follow the
+    current source contents each launch."""
+    import torch
+    spec, fp = config5_spec(4096)
+    o = oracle.Type(spec)
+    t = ddt.Type.from_spec(spec)
+    src = torch.zeros((n, fp), dtype=torch.uint8, device="cuda")
+    dst = torch.zeros((n, 4096), dtype=torch.uint8, device="cuda")
+    for i in range(n):
+        q.pack(t, src[i], 1, dst[i])
+    plan = ddt.Plan(q)
+    for it in range(3):
+        hs = random_bytes(n * fp, 300 + it).reshape(n, fp)
+        src.copy_(torch.from_numpy(hs))
+        plan.launch()
+        torch.cuda.synchronize()
+        got = host(dst)
+        for i in range(n):
+            assert_bytes_equal(got[i], oracle.pack(o, hs[i]), f"plan it={it} req={i}")
+    plan.destroy()
