@@ -9,17 +9,18 @@
 // serialised into a device table (one cudaMemcpyAsync per flush, or once for
 // persistent plans and halo plans).
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 #include "ddt_internal.h"
 
 namespace ddt {
 
-static uint32_t fill_prefix(uint32_t* prefix, const std::vector<ReqDesc>& d) {
+static uint32_t fill_prefix(uint32_t* prefix, const std::vector<ReqDesc>& d, int ub) {
     uint64_t acc = 0;
     for (size_t i = 0; i < d.size(); i++) {
         prefix[i] = (uint32_t)acc;
-        acc += desc_items(d[i]);
+        acc += desc_items(d[i], ub);
     }
     prefix[d.size()] = (uint32_t)acc;
     return (uint32_t)acc;
@@ -35,13 +36,25 @@ size_t device_table_bytes(const HostBatch& b) {
     return off;
 }
 
-uint32_t write_device_table(void* dst, const HostBatch& b) {
+int choose_ub(const HostBatch& b, int sm_count) {
+    const char* env = getenv("DDT_UB");
+    if (env && (atoi(env) == 1 || atoi(env) == 2 || atoi(env) == 4)) return atoi(env);
+    for (int ub : {4, 2}) {
+        uint64_t items = 0;
+        for (const auto& d : b.descs) items += desc_items(d, ub);
+        if (items >= 2ull * (uint64_t)sm_count) return ub;
+    }
+    return 1;
+}
+
+uint32_t write_device_table(void* dst, const HostBatch& b, int ub) {
     size_t n = b.descs.size();
     auto* h = reinterpret_cast<BatchHeader*>(dst);
     std::memset(h, 0, sizeof(*h));
     auto* prefix = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(dst) + sizeof(BatchHeader));
-    uint32_t items = fill_prefix(prefix, b.descs);
+    uint32_t items = fill_prefix(prefix, b.descs, ub);
     size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
+    h->ub = (uint32_t)ub;
     h->nreq = (uint32_t)n;
     h->total_items = items;
     h->desc_offset = (uint32_t)off;
@@ -63,16 +76,32 @@ static void to_param(const HostBatch& b, Launchable& out) {
     out.blob.assign(sizeof(ParamBatch<CAP>), 0);
     auto* p = reinterpret_cast<ParamBatch<CAP>*>(out.blob.data());
     p->h.nreq = (uint32_t)b.descs.size();
-    p->h.total_items = fill_prefix(p->prefix, b.descs);
+    p->h.ub = (uint32_t)out.ub;
+    p->h.total_items = fill_prefix(p->prefix, b.descs, out.ub);
     std::copy(b.descs.begin(), b.descs.end(), p->descs);
     std::copy(b.aux.begin(), b.aux.end(), p->aux);
     std::copy(b.xinfo.begin(), b.xinfo.end(), p->xinfo);
     out.total_items = p->h.total_items;
 }
 
-void make_launchable(const HostBatch& b, bool allow_param, Launchable& out) {
+// The compact kernel variant applies when every source and destination
+// descriptor is closed-form (strided or contiguous) with one vector width.
+static int batch_variant(const HostBatch& b) {
+    if (b.descs.empty()) return 0;
+    int lw = b.descs[0].lw;
+    for (const auto* v : {&b.descs, &b.aux})
+        for (const ReqDesc& d : *v)
+            if ((d.kind != K_STRIDED && d.kind != K_CONTIG) || d.lw != lw) return 0;
+    return 1 + lw;
+}
+
+void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count) {
     size_t n = std::max(b.descs.size(), b.aux.size());
+    out.variant = batch_variant(b);
+    out.ub = choose_ub(b, sm_count);
     out.blob.clear();
+    const char* force = getenv("DDT_FORCE_TABLE");  // experiments: always use the device-table form
+    if (force && force[0] == '1') allow_param = false;
     if (allow_param && n <= (size_t)kParamSmall) {
         out.form = 1;
         to_param<kParamSmall>(b, out);
@@ -82,19 +111,19 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out) {
     } else {
         out.form = 3;
         std::vector<uint32_t> prefix(b.descs.size() + 1);
-        out.total_items = fill_prefix(prefix.data(), b.descs);
+        out.total_items = fill_prefix(prefix.data(), b.descs, out.ub);
     }
 }
 
 int launch_fused(const Launchable& l, void* stream, int grid_cap) {
     const void* src = l.form == 3 ? l.dev : (const void*)l.blob.data();
-    return launch_fused_form(l.form, src, l.total_items, stream, grid_cap);
+    return launch_fused_form(l.form, l.variant, src, l.total_items, stream, grid_cap);
 }
 
 int launch_exchange(const Launchable& l, void* ctrl, int* err_flag_dev, uint64_t timeout_ns, void* stream,
                     int grid_cap) {
     const void* src = l.form == 3 ? l.dev : (const void*)l.blob.data();
-    return launch_exchange_form(l.form, src, l.total_items, ctrl, err_flag_dev, timeout_ns, stream, grid_cap);
+    return launch_exchange_form(l.form, l.variant, src, l.total_items, ctrl, err_flag_dev, timeout_ns, stream, grid_cap);
 }
 
 }  // namespace ddt

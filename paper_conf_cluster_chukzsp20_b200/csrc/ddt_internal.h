@@ -94,26 +94,30 @@ ddt_status_t type_device_layout(ddt_type_s* t, int device, DeviceLayout** out);
 inline int64_t type_extent(const ddt_type_s* t) { return t->ub - t->lb; }
 
 // ------------------------------------------------------------ kernels
-// Builds the u32 reciprocal for DivU32.
+// One request -> (source, destination) descriptor pair (desc.cpp).
 DivU32 make_div(uint32_t d);
-// Fill a descriptor for one request; max_lw caps the vector width (DIRECT
-// pairs share one width).  Returns DDT_OK or an error.
-ddt_status_t build_desc(ddt_type_s* t, const DeviceLayout* dl, int op, const void* noncontig,
-                        const void* packed, int64_t count, ReqDesc* out, int max_lw = 4);
-// Build a DIRECT pair (source layout -> destination layout, equal packed sizes).
+ddt_status_t build_request(int op, ddt_type_s* t, const DeviceLayout* dl, const void* src, const void* dst,
+                           int64_t count, ReqDesc* s, ReqDesc* d);
 ddt_status_t build_direct(ddt_type_s* ts, const DeviceLayout* dls, const void* src, int64_t scount, ddt_type_s* td,
-                          const DeviceLayout* dld, void* dst, int64_t dcount, ReqDesc* d, ReqDesc* a);
-// Items of a descriptor.
-inline uint32_t desc_items(const ReqDesc& d) {
-    return (uint32_t)((d.nvec + (uint64_t)kItemVecs - 1) / (uint64_t)kItemVecs);
+                          const DeviceLayout* dld, void* dst, int64_t dcount, ReqDesc* s, ReqDesc* d);
+// Items of a descriptor at ub vectors per thread per item.
+inline uint32_t desc_items(const ReqDesc& d, int ub = kUnroll) {
+    uint64_t per = (uint64_t)kThreads * (uint64_t)ub;
+    return (uint32_t)((d.nvec + per - 1) / per);
 }
 
-// A batch on the host: descriptors (items come from these), DIRECT
-// destination layouts, and exchange side info (empty, or one per descriptor).
+// A batch on the host: source descriptors (items come from these), their
+// destination descriptors (descs[i].aux indexes aux), and exchange side info
+// (empty, or one per source descriptor).
 struct HostBatch {
     std::vector<ReqDesc> descs, aux;
     std::vector<XInfo> xinfo;
     void clear() { descs.clear(); aux.clear(); xinfo.clear(); }
+    void add(ReqDesc s, const ReqDesc& d) {
+        s.aux = (uint32_t)aux.size();
+        aux.push_back(d);
+        descs.push_back(s);
+    }
 };
 // A batch ready to launch: carried in the kernel parameters (form 1 / 2) or
 // as a device table (form 3, `dev` owned by the caller).
@@ -122,16 +126,21 @@ struct Launchable {
     std::vector<uint8_t> blob;  // ParamBatch<CAP> bytes (form 1 / 2)
     void* dev = nullptr;        // device table (form 3)
     uint32_t total_items = 0;
+    int variant = 0;            // 0 generic; 1 + lw: strided-only, one vector width
+    int ub = kUnroll;           // vectors per thread per item
 };
 size_t device_table_bytes(const HostBatch& b);
-uint32_t write_device_table(void* dst, const HostBatch& b);
+uint32_t write_device_table(void* dst, const HostBatch& b, int ub);
+// Items per thread for a batch: the largest of {4, 2, 1} that still gives
+// >= 2 items per SM, so latency-bound batches use every SM.
+int choose_ub(const HostBatch& b, int sm_count);
 // Param form if it fits (and allowed), else form 3 with `dev` left to the caller.
-void make_launchable(const HostBatch& b, bool allow_param, Launchable& out);
+void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count = 148);
 int launch_fused(const Launchable& l, void* stream, int grid_cap);
 int launch_exchange(const Launchable& l, void* ctrl, int* err_flag_dev, uint64_t timeout_ns, void* stream,
                     int grid_cap);
-int launch_fused_form(int form, const void* param_or_table, uint32_t total_items, void* stream, int grid_cap);
-int launch_exchange_form(int form, const void* param_or_table, uint32_t total_items, void* ctrl, int* err_flag_dev,
+int launch_fused_form(int form, int variant, const void* param_or_table, uint32_t total_items, void* stream, int grid_cap);
+int launch_exchange_form(int form, int variant, const void* param_or_table, uint32_t total_items, void* ctrl, int* err_flag_dev,
                          uint64_t timeout_ns, void* stream, int grid_cap);
 int device_sm_count(int device);
 

@@ -1,9 +1,18 @@
-// desc.cpp -- one request -> one device descriptor (the per-request part of
-// the paper's request object, §IV-A.1: operation, origin / target
-// buffer, cached data layout entry), built once at enqueue in O(1) from the
-// committed layout cache.  All address arithmetic is signed 64-bit; the
-// vector width is the largest power of two (<= 16 B) dividing every offset,
-// length and pointer involved, so every device access is naturally aligned.
+// desc.cpp -- one request -> a (source, destination) pair of device layout
+// descriptors (the per-request part of the paper's request object, §IV-A.1
+// operation, origin / target buffer, cached data layout entry),
+// built once at enqueue in O(1) from the committed layout cache.
+//
+// Every operation is "load vector v through the source layout, store it
+// through the destination layout":
+//   pack   = (type layout over the origin buffer) -> (contiguous packed buffer)
+//   unpack = (contiguous packed buffer)           -> (type layout over the target)
+//   direct = (source type layout)                 -> (destination type layout)
+//            -- the paper's DirectIPC op, no packed intermediate.
+// All address arithmetic is signed 64-bit; the vector width w is the largest
+// power of two (<= 16 B) dividing every segment offset and length, both
+// pointers and (count > 1) the extent, so every device access is naturally
+// aligned and the two sides of a pair always share one width.
 #include <algorithm>
 #include <cstring>
 
@@ -27,28 +36,32 @@ static int lowbit16(uint64_t v) {
 
 static uint64_t uabs64(int64_t v) { return v < 0 ? (uint64_t)(-(v + 1)) + 1 : (uint64_t)v; }
 
-ddt_status_t build_desc(ddt_type_s* t, const DeviceLayout* dl, int op, const void* noncontig, const void* packed,
-                        int64_t count, ReqDesc* d, int max_lw) {
-    const Layout& L = t->layout;
-    std::memset(d, 0, sizeof(*d));
-    int64_t bytes = count * t->size;
-    int64_t ext = type_extent(t);
-    int w = L.align;
-    w = std::min(w, lowbit16((uint64_t)(uintptr_t)noncontig));
-    w = std::min(w, lowbit16((uint64_t)(uintptr_t)packed));
-    if (count > 1) w = std::min(w, lowbit16(uabs64(ext)));
+static int log2i(int w) {
     int lw = 0;
     while ((1 << lw) < w) lw++;
-    if (lw > max_lw) lw = max_lw;
+    return lw;
+}
+
+// Largest legal log2 vector width of one side (type layout over pointer p).
+static int side_lw(ddt_type_s* t, const void* p, int64_t count) {
+    int w = std::min(t->layout.align, lowbit16((uint64_t)(uintptr_t)p));
+    if (count > 1) w = std::min(w, lowbit16(uabs64(type_extent(t))));
+    return log2i(w);
+}
+
+// Fill the layout fields of `d` for `count` instances of t at `base_ptr`.
+static ddt_status_t layout_desc(ddt_type_s* t, const DeviceLayout* dl, const void* base_ptr, int64_t count, int lw,
+                                ReqDesc* d) {
+    const Layout& L = t->layout;
+    int64_t bytes = count * t->size;
+    int64_t ext = type_extent(t);
     uint64_t nvec = (uint64_t)bytes >> lw;
     if (nvec >= (1ull << 32)) {
         set_error("request too large for one descriptor (>= 2^32 vectors)");
         return DDT_ERR_UNSUPPORTED;
     }
-    d->noncontig = (uint64_t)(uintptr_t)noncontig;
-    d->packed = (uint64_t)(uintptr_t)packed;
+    d->ptr = (uint64_t)(uintptr_t)base_ptr;
     d->nvec = (uint32_t)nvec;
-    d->op = (uint8_t)op;
     d->lw = (uint8_t)lw;
     d->extent = ext;
     if (L.kind == DDT_LAYOUT_STRIDED) {
@@ -59,6 +72,7 @@ ddt_status_t build_desc(ddt_type_s* t, const DeviceLayout* dl, int op, const voi
         d->base = f.base;
         d->vps = make_div((uint32_t)(f.seg_len >> lw));
         if (f.dims.empty()) {
+            if (f.base == 0) d->kind = K_CONTIG;  // one contiguous run at the pointer itself
             d->ndim = 0;
             d->extent = 0;
         } else {
@@ -68,7 +82,7 @@ ddt_status_t build_desc(ddt_type_s* t, const DeviceLayout* dl, int op, const voi
                 return DDT_ERR_UNSUPPORTED;
             }
             d->ndim = (uint8_t)(D - 1);
-            // innermost first; the outermost dim is the final quotient
+            // innermost first; the outermost dim is the final quotient (no division)
             for (int k = 0; k < D - 1; k++) {
                 const Dim& x = f.dims[(size_t)(D - 1 - k)];
                 d->radix[k] = make_div((uint32_t)x.n);
@@ -94,29 +108,44 @@ ddt_status_t build_desc(ddt_type_s* t, const DeviceLayout* dl, int op, const voi
     return DDT_OK;
 }
 
-
-static int desc_lw_uncapped(ddt_type_s* t, const void* nc, const void* pk, int64_t count) {
-    int w = t->layout.align;
-    w = std::min(w, lowbit16((uint64_t)(uintptr_t)nc));
-    if (pk) w = std::min(w, lowbit16((uint64_t)(uintptr_t)pk));
-    if (count > 1) w = std::min(w, lowbit16(uabs64(type_extent(t))));
-    int lw = 0;
-    while ((1 << lw) < w) lw++;
-    return lw;
+static void contig_desc(const void* p, uint32_t nvec, int lw, ReqDesc* d) {
+    std::memset(d, 0, sizeof(*d));
+    d->ptr = (uint64_t)(uintptr_t)p;
+    d->nvec = nvec;
+    d->lw = (uint8_t)lw;
+    d->kind = K_CONTIG;
 }
 
-// DirectIPC: gather through the source layout and scatter
-// through the destination layout in one pass (no packed intermediate).  Both
-// descriptors share one vector width and vector count; `d` carries the items.
+ddt_status_t build_request(int op, ddt_type_s* t, const DeviceLayout* dl, const void* src, const void* dst,
+                           int64_t count, ReqDesc* s, ReqDesc* d) {
+    std::memset(s, 0, sizeof(*s));
+    std::memset(d, 0, sizeof(*d));
+    const void* nc = op == OP_PACK ? src : dst;  // the typed side
+    const void* pk = op == OP_PACK ? dst : src;  // the packed side
+    int lw = std::min(side_lw(t, nc, count), log2i(lowbit16((uint64_t)(uintptr_t)pk)));
+    ReqDesc lay, con;
+    std::memset(&lay, 0, sizeof(lay));
+    ddt_status_t st = layout_desc(t, dl, nc, count, lw, &lay);
+    if (st != DDT_OK) return st;
+    contig_desc(pk, lay.nvec, lw, &con);
+    *s = op == OP_PACK ? lay : con;
+    *d = op == OP_PACK ? con : lay;
+    s->op = (uint8_t)op;
+    d->op = (uint8_t)op;
+    return DDT_OK;
+}
+
 ddt_status_t build_direct(ddt_type_s* ts, const DeviceLayout* dls, const void* src, int64_t scount, ddt_type_s* td,
-                          const DeviceLayout* dld, void* dst, int64_t dcount, ReqDesc* d, ReqDesc* a) {
+                          const DeviceLayout* dld, void* dst, int64_t dcount, ReqDesc* s, ReqDesc* d) {
     if (scount * ts->size != dcount * td->size) return DDT_ERR_SIZE_MISMATCH;
-    int lw = std::min(desc_lw_uncapped(ts, src, nullptr, scount), desc_lw_uncapped(td, dst, nullptr, dcount));
-    ddt_status_t s = build_desc(ts, dls, OP_DIRECT, src, nullptr, scount, d, lw);
-    if (s != DDT_OK) return s;
-    s = build_desc(td, dld, OP_DIRECT, dst, nullptr, dcount, a, lw);
-    if (s != DDT_OK) return s;
-    if (d->nvec != a->nvec || d->lw != a->lw) return DDT_ERR_STATE;
+    std::memset(s, 0, sizeof(*s));
+    std::memset(d, 0, sizeof(*d));
+    int lw = std::min(side_lw(ts, src, scount), side_lw(td, dst, dcount));
+    ddt_status_t st = layout_desc(ts, dls, src, scount, lw, s);
+    if (st == DDT_OK) st = layout_desc(td, dld, dst, dcount, lw, d);
+    if (st != DDT_OK) return st;
+    if (s->nvec != d->nvec) return DDT_ERR_STATE;
+    s->op = d->op = OP_DIRECT;
     return DDT_OK;
 }
 

@@ -20,14 +20,19 @@ namespace ddt {
 
 constexpr int kMaxDims = 4;          // closed-form strided dims per layout (R7)
 constexpr int kThreads = 256;        // threads per CTA of the fused kernel
-constexpr int kUnroll = 4;           // vectors per thread per item (loads in flight)
-constexpr int kItemVecs = kThreads * kUnroll;  // vectors per work item
+constexpr int kUnroll = 4;           // max vectors per thread per item (loads in flight)
+constexpr int kItemVecs = kThreads * kUnroll;  // max vectors per work item
+// A batch picks ub in {1, 2, 4} vectors per thread per item: small batches use
+// smaller items so that their work spreads over all 148 SMs (latency-bound
+// regime), large batches use kUnroll for memory-level parallelism.
 
-// PACK: gather non-contiguous -> packed; UNPACK: packed -> scatter;
-// DIRECT: non-contiguous -> non-contiguous with a second layout (the paper's
-// DirectIPC op), used for self messages of a halo exchange.
+// Every request is a (source, destination) pair of descriptors: vector v is
+// loaded through the source layout and stored through the destination layout.
+// PACK: typed source -> contiguous destination; UNPACK: contiguous -> typed;
+// DIRECT: typed -> typed (the paper's DirectIPC op; self
+// messages of a halo exchange).  K_CONTIG is the packed side (offset = v * w).
 enum DescOp : uint8_t { OP_PACK = 0, OP_UNPACK = 1, OP_DIRECT = 2 };
-enum DescKind : uint8_t { K_STRIDED = 0, K_UNIFORM32 = 1, K_UNIFORM64 = 2, K_GENERAL = 3 };
+enum DescKind : uint8_t { K_STRIDED = 0, K_UNIFORM32 = 1, K_UNIFORM64 = 2, K_GENERAL = 3, K_CONTIG = 4 };
 
 // Unsigned 32-bit division by a runtime constant d via a 64-bit reciprocal:
 // q = umulhi64(n, ceil(2^64 / d)) is exact for n, d < 2^32 (error < 1/d);
@@ -39,8 +44,8 @@ struct DivU32 {
 };
 
 struct alignas(16) ReqDesc {
-    uint64_t noncontig;     // non-contiguous side (pack: source, unpack / direct-aux: destination)
-    uint64_t packed;        // contiguous side     (pack: destination, unpack: source)
+    uint64_t ptr;           // base pointer of this side (MPI buffer address or packed buffer)
+    uint64_t pad0;
     uint32_t nvec;          // vectors in the request (count*size / w), < 2^32
     uint8_t op;             // DescOp
     uint8_t kind;           // DescKind
@@ -57,7 +62,7 @@ struct alignas(16) ReqDesc {
     uint64_t prefix;        // general: int64 exclusive packed prefix (nseg + 1 entries)
     uint32_t list_n;        // general: number of segments per instance
     uint32_t uid_lo;        // low bits of the request UID (debug / tracing)
-    uint32_t aux;           // DIRECT: index of the destination-layout descriptor in aux[]
+    uint32_t aux;           // source descriptors: index of the destination descriptor in aux[]
     uint32_t pad2;
 };
 
@@ -71,7 +76,7 @@ struct alignas(16) XInfo {
 };
 
 // Header of a device batch table:
-//   BatchHeader | uint32 prefix[nreq + 1] (16 B padded) | ReqDesc[nreq] | ReqDesc aux[naux] | XInfo[nreq]?
+//   BatchHeader | uint32 prefix[nreq + 1] (16 B padded) | ReqDesc src[nreq] | ReqDesc dst[naux] | XInfo[nreq]?
 struct alignas(16) BatchHeader {
     uint32_t nreq;
     uint32_t total_items;
@@ -79,7 +84,8 @@ struct alignas(16) BatchHeader {
     uint32_t aux_offset;
     uint32_t xinfo_offset;  // 0 = no exchange info
     uint32_t naux;
-    uint32_t pad[2];
+    uint32_t ub;            // vectors per thread per item (1, 2 or 4)
+    uint32_t pad;
 };
 
 // A small batch carried in the kernel parameters.

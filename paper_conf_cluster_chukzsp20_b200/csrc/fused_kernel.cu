@@ -42,8 +42,9 @@ __device__ __forceinline__ uint32_t divu(uint32_t n, const DivU32& d) {
 // NC: read-only data for the kernel's lifetime -> non-coherent path, no L1
 // allocation.  !NC: data another agent writes during the kernel (P2P window)
 // -> ld.global.cg (L2, coherent).
-template <bool NC>
-__device__ __forceinline__ uint4 ld_vec(const uint8_t* p, int lw) {
+template <bool NC, int LW>
+__device__ __forceinline__ uint4 ld_vec(const uint8_t* p, int lw_rt) {
+    const int lw = LW >= 0 ? LW : lw_rt;  // compile-time width folds the switch
     uint4 r = make_uint4(0, 0, 0, 0);
     switch (lw) {
     case 4:
@@ -82,7 +83,9 @@ __device__ __forceinline__ uint4 ld_vec(const uint8_t* p, int lw) {
     return r;
 }
 
-__device__ __forceinline__ void st_vec(uint8_t* p, int lw, const uint4& r) {
+template <int LW>
+__device__ __forceinline__ void st_vec(uint8_t* p, int lw_rt, const uint4& r) {
+    const int lw = LW >= 0 ? LW : lw_rt;
     switch (lw) {
     case 4: asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(r.x), "r"(r.y), "r"(r.z), "r"(r.w) : "memory"); break;
     case 3: asm volatile("st.global.v2.u32 [%0], {%1,%2};" ::"l"(p), "r"(r.x), "r"(r.y) : "memory"); break;
@@ -93,9 +96,12 @@ __device__ __forceinline__ void st_vec(uint8_t* p, int lw, const uint4& r) {
 }
 
 // Byte offset (relative to the non-contiguous pointer) of vector v.
+// SONLY: the batch holds closed-form strided layouts only (list paths compiled out).
+template <int LW, bool SONLY>
 __device__ __forceinline__ int64_t vec_offset(const ReqDesc& d, uint32_t v) {
-    const int lw = d.lw;
-    if (d.kind == K_STRIDED) {
+    const int lw = LW >= 0 ? LW : d.lw;
+    if (d.kind == K_CONTIG) return (int64_t)v << lw;  // the packed side
+    if (SONLY || d.kind == K_STRIDED) {
         uint32_t s = divu(v, d.vps);
         uint32_t within = v - s * d.vps.d;
         int64_t off = d.base + ((int64_t)within << lw);
@@ -106,6 +112,8 @@ __device__ __forceinline__ int64_t vec_offset(const ReqDesc& d, uint32_t v) {
             s = q;
         }
         return off + (int64_t)s * d.extent;
+    } else if constexpr (SONLY) {
+        return 0;
     } else if (d.kind != K_GENERAL) {
         uint32_t s = divu(v, d.vps);
         uint32_t within = v - s * d.vps.d;
@@ -130,46 +138,30 @@ __device__ __forceinline__ int64_t vec_offset(const ReqDesc& d, uint32_t v) {
     }
 }
 
-// One work item: kItemVecs vectors starting at v0.  COH: the packed side of an
-// unpack is written by another GPU during this kernel.
-template <bool COH>
-__device__ __forceinline__ void run_desc(const ReqDesc& d, const ReqDesc& a, uint32_t v0) {
-    const uint32_t nvec = d.nvec;
-    const int lw = d.lw;
-    uint8_t* nc = reinterpret_cast<uint8_t*>(d.noncontig);
-    uint8_t* pk = reinterpret_cast<uint8_t*>(d.packed);
+// One work item: kItemVecs vectors starting at v0, loaded through the source
+// descriptor S and stored through the destination descriptor D (one code path
+// for pack, unpack and DirectIPC).  coh: the source is written by another GPU
+// during this kernel (P2P window) -> L2-coherent loads instead of the
+// non-coherent read-only path.
+template <int LW, bool SONLY>
+__device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uint32_t v0, bool coh, int ub) {
+    const uint32_t nvec = S.nvec;
+    const int lw = LW >= 0 ? LW : S.lw;
+    const uint8_t* src = reinterpret_cast<const uint8_t*>(S.ptr);
+    uint8_t* dst = reinterpret_cast<uint8_t*>(D.ptr);
     uint4 buf[kUnroll];
-    if (d.op == OP_UNPACK) {
 #pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
-            uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-            if (v < nvec) buf[u] = ld_vec<!COH>(pk + ((uint64_t)v << lw), lw);
+    for (int u = 0; u < kUnroll; u++) {
+        uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+        if (u < ub && v < nvec) {
+            const uint8_t* p = src + vec_offset<LW, SONLY>(S, v);
+            buf[u] = coh ? ld_vec<false, LW>(p, lw) : ld_vec<true, LW>(p, lw);
         }
-#pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
-            uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-            if (v < nvec) st_vec(nc + vec_offset(d, v), lw, buf[u]);
-        }
-        return;
     }
 #pragma unroll
     for (int u = 0; u < kUnroll; u++) {
         uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-        if (v < nvec) buf[u] = ld_vec<true>(nc + vec_offset(d, v), lw);
-    }
-    if (d.op == OP_PACK) {
-#pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
-            uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-            if (v < nvec) st_vec(pk + ((uint64_t)v << lw), lw, buf[u]);
-        }
-    } else {  // OP_DIRECT: scatter through the destination layout
-        uint8_t* dn = reinterpret_cast<uint8_t*>(a.noncontig);
-#pragma unroll
-        for (int u = 0; u < kUnroll; u++) {
-            uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-            if (v < nvec) st_vec(dn + vec_offset(a, v), lw, buf[u]);
-        }
+        if (u < ub && v < nvec) st_vec<LW>(dst + vec_offset<LW, SONLY>(D, v), lw, buf[u]);
     }
 }
 
@@ -185,7 +177,7 @@ __device__ __forceinline__ uint32_t find_request(const uint32_t* prefix, uint32_
 }
 
 struct TableView {
-    uint32_t nreq, total;
+    uint32_t nreq, total, ub;
     const uint32_t* prefix;
     const ReqDesc* descs;
     const ReqDesc* aux;
@@ -197,6 +189,7 @@ __device__ __forceinline__ TableView view_of(const uint8_t* t) {
     TableView v;
     v.nreq = h->nreq;
     v.total = h->total_items;
+    v.ub = h->ub;
     v.prefix = reinterpret_cast<const uint32_t*>(t + sizeof(BatchHeader));
     v.descs = reinterpret_cast<const ReqDesc*>(t + h->desc_offset);
     v.aux = reinterpret_cast<const ReqDesc*>(t + h->aux_offset);
@@ -209,6 +202,7 @@ __device__ __forceinline__ TableView view_of(const ParamBatch<CAP>& p) {
     TableView v;
     v.nreq = p.h.nreq;
     v.total = p.h.total_items;
+    v.ub = p.h.ub;
     v.prefix = p.prefix;
     v.descs = p.descs;
     v.aux = p.aux;
@@ -245,7 +239,7 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // items in increasing order, so a CTA only ever waits after finishing all of
 // its own pack items; with grid <= resident CTAs nothing waits on work that
 // cannot run (deadlock freedom without a global ticket).
-template <bool XCHG>
+template <bool XCHG, int LW, bool SONLY>
 __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int* err_flag, uint64_t timeout_ns) {
     __shared__ ReqDesc sd;
     __shared__ ReqDesc sa;
@@ -267,21 +261,22 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
             __syncthreads();  // every warp is done with the previous descriptor
             copy_words(&sd, tv.descs + r, kWords, 0);
             if constexpr (XCHG) copy_words(&sx, tv.xinfo + r, kXWords, 32);
+            copy_words(&sa, tv.aux + r, kWords, 64);  // destination descriptor (aux[r], see HostBatch::add)
             __syncthreads();
-            if (sd.op == OP_DIRECT) {
-                copy_words(&sa, tv.aux + sd.aux, kWords, 0);
-                __syncthreads();
-            }
             if constexpr (XCHG) {
-                if (sx.parity_stride) {
-                    if (threadIdx.x == 0) sd.packed += (epoch & 1ull) * (uint64_t)sx.parity_stride;
+                if (sx.parity_stride) {  // double-buffered window: pack writes it, unpack reads it
+                    if (threadIdx.x == 0) {
+                        const uint64_t off = (epoch & 1ull) * (uint64_t)sx.parity_stride;
+                        if (sd.op == OP_PACK) sa.ptr += off;
+                        else sd.ptr += off;
+                    }
                     __syncthreads();
                 }
             }
             cur_first = tv.prefix[r];
             cur = r;
         }
-        const uint32_t v0 = (item - cur_first) * (uint32_t)kItemVecs;
+        const uint32_t v0 = (item - cur_first) * (uint32_t)(kThreads * tv.ub);
         if constexpr (XCHG) {
             if (sd.op == OP_UNPACK && sx.flag) {
                 if (threadIdx.x == 0) {
@@ -302,11 +297,11 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
                     s_ok = ok;
                 }
                 __syncthreads();
-                if (s_ok) run_desc<true>(sd, sa, v0);
+                if (s_ok) run_desc<LW, SONLY>(sd, sa, v0, true, (int)tv.ub);
                 continue;
             }
         }
-        run_desc<false>(sd, sa, v0);
+        run_desc<LW, SONLY>(sd, sa, v0, false, (int)tv.ub);
         if constexpr (XCHG) {
             if (sd.op == OP_PACK && sx.flag) {
                 __syncthreads();  // the CTA's peer stores precede thread 0's release
@@ -339,24 +334,32 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
     }
 }
 
+// Kernel instances.  Variant V: 0 = generic (any kind, runtime width);
+// 1 + lw = closed-form strided layouts only, vector width 2^lw fixed at
+// compile time -- a compact kernel for halo plans and dense batches (a cold
+// SM fetches a few KB of code instead of the generic ~80 KB).
+template <int V> struct VarT { static constexpr int LW = V == 0 ? -1 : V - 1; static constexpr bool SONLY = V != 0; };
+
+template <int V>
 __global__ void __launch_bounds__(kThreads) ddt_fused_dev(const uint8_t* __restrict__ table) {
-    fused_body<false>(view_of(table), nullptr, nullptr, 0);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY>(view_of(table), nullptr, nullptr, 0);
 }
 
-template <int CAP>
+template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
-    fused_body<false>(view_of(pb), nullptr, nullptr, 0);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY>(view_of(pb), nullptr, nullptr, 0);
 }
 
+template <int V>
 __global__ void __launch_bounds__(kThreads)
     ddt_exchange_dev(const uint8_t* __restrict__ table, XCtrl* ctrl, int* err_flag, uint64_t timeout_ns) {
-    fused_body<true>(view_of(table), ctrl, err_flag, timeout_ns);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY>(view_of(table), ctrl, err_flag, timeout_ns);
 }
 
-template <int CAP>
+template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads)
     ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, XCtrl* ctrl, int* err_flag, uint64_t timeout_ns) {
-    fused_body<true>(view_of(pb), ctrl, err_flag, timeout_ns);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY>(view_of(pb), ctrl, err_flag, timeout_ns);
 }
 
 // ------------------------------------------------------------------ host side
@@ -371,15 +374,12 @@ int device_sm_count(int device) {
 }
 
 template <class K>
-static int resident_ctas(K kernel, int* cache) {
-    if (*cache == 0) {
-        int b = 0;
-        if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, kThreads, 0) != cudaSuccess || b <= 0) b = 1;
-        *cache = b;
-    }
+static int resident_ctas(K kernel) {
+    int b = 0;
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, kThreads, 0) != cudaSuccess || b <= 0) b = 1;
     int dev = 0;
     cudaGetDevice(&dev);
-    return *cache * device_sm_count(dev);
+    return b * device_sm_count(dev);
 }
 
 static uint32_t grid_for(uint32_t total, int resident, int grid_cap) {
@@ -388,42 +388,69 @@ static uint32_t grid_for(uint32_t total, int resident, int grid_cap) {
     return total < cap ? total : cap;
 }
 
-// form: 1 = ParamBatch<kParamSmall>, 2 = ParamBatch<kParamLarge>, 3 = device table
-int launch_fused_form(int form, const void* param_or_table, uint32_t total_items, void* stream, int grid_cap) {
-    if (total_items == 0) return 0;
-    static int occ_dev = 0, occ_s = 0, occ_l = 0;
-    cudaStream_t s = (cudaStream_t)stream;
+template <int V>
+static void launch_fused_v(int form, const void* src, uint32_t total, cudaStream_t s, int grid_cap) {
+    static int res[4] = {0, 0, 0, 0};
     if (form == 1) {
-        uint32_t g = grid_for(total_items, resident_ctas(ddt_fused_param<kParamSmall>, &occ_s), grid_cap);
-        ddt_fused_param<kParamSmall><<<g, kThreads, 0, s>>>(*reinterpret_cast<const ParamBatch<kParamSmall>*>(param_or_table));
+        if (!res[1]) res[1] = resident_ctas(ddt_fused_param<kParamSmall, V>);
+        ddt_fused_param<kParamSmall, V><<<grid_for(total, res[1], grid_cap), kThreads, 0, s>>>(
+            *reinterpret_cast<const ParamBatch<kParamSmall>*>(src));
     } else if (form == 2) {
-        uint32_t g = grid_for(total_items, resident_ctas(ddt_fused_param<kParamLarge>, &occ_l), grid_cap);
-        ddt_fused_param<kParamLarge><<<g, kThreads, 0, s>>>(*reinterpret_cast<const ParamBatch<kParamLarge>*>(param_or_table));
+        if (!res[2]) res[2] = resident_ctas(ddt_fused_param<kParamLarge, V>);
+        ddt_fused_param<kParamLarge, V><<<grid_for(total, res[2], grid_cap), kThreads, 0, s>>>(
+            *reinterpret_cast<const ParamBatch<kParamLarge>*>(src));
     } else {
-        uint32_t g = grid_for(total_items, resident_ctas(ddt_fused_dev, &occ_dev), grid_cap);
-        ddt_fused_dev<<<g, kThreads, 0, s>>>(reinterpret_cast<const uint8_t*>(param_or_table));
+        if (!res[3]) res[3] = resident_ctas(ddt_fused_dev<V>);
+        ddt_fused_dev<V><<<grid_for(total, res[3], grid_cap), kThreads, 0, s>>>(reinterpret_cast<const uint8_t*>(src));
+    }
+}
+
+template <int V>
+static void launch_exchange_v(int form, const void* src, uint32_t total, XCtrl* c, int* err, uint64_t timeout_ns,
+                              cudaStream_t s, int grid_cap) {
+    static int res[4] = {0, 0, 0, 0};
+    if (form == 1) {
+        if (!res[1]) res[1] = resident_ctas(ddt_exchange_param<kParamSmall, V>);
+        ddt_exchange_param<kParamSmall, V><<<grid_for(total, res[1], grid_cap), kThreads, 0, s>>>(
+            *reinterpret_cast<const ParamBatch<kParamSmall>*>(src), c, err, timeout_ns);
+    } else if (form == 2) {
+        if (!res[2]) res[2] = resident_ctas(ddt_exchange_param<kParamLarge, V>);
+        ddt_exchange_param<kParamLarge, V><<<grid_for(total, res[2], grid_cap), kThreads, 0, s>>>(
+            *reinterpret_cast<const ParamBatch<kParamLarge>*>(src), c, err, timeout_ns);
+    } else {
+        if (!res[3]) res[3] = resident_ctas(ddt_exchange_dev<V>);
+        ddt_exchange_dev<V><<<grid_for(total, res[3], grid_cap), kThreads, 0, s>>>(
+            reinterpret_cast<const uint8_t*>(src), c, err, timeout_ns);
+    }
+}
+
+// form: 1 = ParamBatch<kParamSmall>, 2 = ParamBatch<kParamLarge>, 3 = device table
+int launch_fused_form(int form, int variant, const void* src, uint32_t total_items, void* stream, int grid_cap) {
+    if (total_items == 0) return 0;
+    cudaStream_t s = (cudaStream_t)stream;
+    switch (variant) {
+    case 1: launch_fused_v<1>(form, src, total_items, s, grid_cap); break;
+    case 2: launch_fused_v<2>(form, src, total_items, s, grid_cap); break;
+    case 3: launch_fused_v<3>(form, src, total_items, s, grid_cap); break;
+    case 4: launch_fused_v<4>(form, src, total_items, s, grid_cap); break;
+    case 5: launch_fused_v<5>(form, src, total_items, s, grid_cap); break;
+    default: launch_fused_v<0>(form, src, total_items, s, grid_cap); break;
     }
     return (int)cudaGetLastError();
 }
 
-int launch_exchange_form(int form, const void* param_or_table, uint32_t total_items, void* ctrl, int* err_flag_dev,
+int launch_exchange_form(int form, int variant, const void* src, uint32_t total_items, void* ctrl, int* err_flag_dev,
                          uint64_t timeout_ns, void* stream, int grid_cap) {
     if (total_items == 0) return 0;
-    static int occ_dev = 0, occ_s = 0, occ_l = 0;
     cudaStream_t s = (cudaStream_t)stream;
     XCtrl* c = reinterpret_cast<XCtrl*>(ctrl);
-    if (form == 1) {
-        uint32_t g = grid_for(total_items, resident_ctas(ddt_exchange_param<kParamSmall>, &occ_s), grid_cap);
-        ddt_exchange_param<kParamSmall><<<g, kThreads, 0, s>>>(
-            *reinterpret_cast<const ParamBatch<kParamSmall>*>(param_or_table), c, err_flag_dev, timeout_ns);
-    } else if (form == 2) {
-        uint32_t g = grid_for(total_items, resident_ctas(ddt_exchange_param<kParamLarge>, &occ_l), grid_cap);
-        ddt_exchange_param<kParamLarge><<<g, kThreads, 0, s>>>(
-            *reinterpret_cast<const ParamBatch<kParamLarge>*>(param_or_table), c, err_flag_dev, timeout_ns);
-    } else {
-        uint32_t g = grid_for(total_items, resident_ctas(ddt_exchange_dev, &occ_dev), grid_cap);
-        ddt_exchange_dev<<<g, kThreads, 0, s>>>(reinterpret_cast<const uint8_t*>(param_or_table), c, err_flag_dev,
-                                                timeout_ns);
+    switch (variant) {
+    case 1: launch_exchange_v<1>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
+    case 2: launch_exchange_v<2>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
+    case 3: launch_exchange_v<3>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
+    case 4: launch_exchange_v<4>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
+    case 5: launch_exchange_v<5>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
+    default: launch_exchange_v<0>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
     }
     return (int)cudaGetLastError();
 }

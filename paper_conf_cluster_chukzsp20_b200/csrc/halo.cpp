@@ -141,11 +141,11 @@ ddt_status_t upload(const std::vector<uint8_t>& host, void** dev) {
 
 // Small batches ride in the kernel parameters (captured into the graph node);
 // larger ones are uploaded once as a device table.
-ddt_status_t make_table(const HostBatch& b, Launchable& l) {
-    make_launchable(b, true, l);
+ddt_status_t make_table(const HostBatch& b, Launchable& l, int sm_count) {
+    make_launchable(b, true, l, sm_count);
     if (l.form != 3) return DDT_OK;
     std::vector<uint8_t> host(device_table_bytes(b));
-    write_device_table(host.data(), b);
+    write_device_table(host.data(), b, l.ub);
     return upload(host, &l.dev);
 }
 
@@ -433,11 +433,17 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     }
 
     // ---- build the device work tables
-    auto desc_for = [&](ddt_type_s* t, int op, const void* nc, const void* pk, int64_t count, ReqDesc* d) -> ddt_status_t {
+    // pack: typed send buffer -> packed slot; unpack: packed slot -> typed recv buffer
+    auto add_req = [&](HostBatch& b, ddt_type_s* t, int op, const void* src, const void* dst, int64_t count,
+                       uint32_t* items) -> ddt_status_t {
         DeviceLayout* dl = nullptr;
         ddt_status_t s2 = type_device_layout(t, h->device, &dl);
+        ReqDesc sd, dd;
+        if (s2 == DDT_OK) s2 = build_request(op, t, dl, src, dst, count, &sd, &dd);
         if (s2 != DDT_OK) return s2;
-        return build_desc(t, dl, op, nc, pk, count, d);
+        b.add(sd, dd);
+        if (items) *items = desc_items(sd);
+        return DDT_OK;
     };
     // Self messages never touch a staging buffer or window: one DirectIPC
     // descriptor gathers the send layout and scatters straight into the
@@ -454,9 +460,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         ReqDesc d, a;
         if (s2 == DDT_OK) s2 = build_direct(s.type, dls, s.buf, s.count, r.type, dld, r.buf, r.count, &d, &a);
         if (s2 != DDT_OK) return s2;
-        d.aux = (uint32_t)b.aux.size();
-        b.aux.push_back(a);
-        b.descs.push_back(d);
+        b.add(d, a);
         if (with_x) b.xinfo.push_back(XInfo{});
         return DDT_OK;
     };
@@ -515,19 +519,16 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                 continue;
             }
             char* dst = (char*)h->send_stage + region[s.peer] + (match[(size_t)i]->data_off - span[s.peer].first);
-            ReqDesc d;
-            st = desc_for(s.type, OP_PACK, s.buf, dst, s.count, &d);
-            packb.descs.push_back(d);
+            st = add_req(packb, s.type, OP_PACK, s.buf, dst, s.count, nullptr);
         }
         for (int i = 0; i < nrecv && st == DDT_OK; i++) {
             const auto& r = recvs[i];
             if (r.count * r.type->size == 0 || r.peer == c->rank) continue;
-            ReqDesc d;
-            st = desc_for(r.type, OP_UNPACK, r.buf, (char*)h->recv_stage + RL.data_off[(size_t)i], r.count, &d);
-            unpackb.descs.push_back(d);
+            st = add_req(unpackb, r.type, OP_UNPACK, (char*)h->recv_stage + RL.data_off[(size_t)i], r.buf, r.count,
+                         nullptr);
         }
-        if (st == DDT_OK && !packb.descs.empty()) st = make_table(packb, h->pack_l);
-        if (st == DDT_OK && !unpackb.descs.empty()) st = make_table(unpackb, h->unpack_l);
+        if (st == DDT_OK && !packb.descs.empty()) st = make_table(packb, h->pack_l, queue_sm_count(q));
+        if (st == DDT_OK && !unpackb.descs.empty()) st = make_table(unpackb, h->unpack_l, queue_sm_count(q));
         h->launches = (packb.descs.empty() ? 0 : 1) + (unpackb.descs.empty() ? 0 : 1);
     } else {
         // P2P: one kernel; items ordered remote packs, self directs, then the
@@ -540,14 +541,13 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             if (s.count * s.type->size == 0 || s.peer == c->rank) continue;
             const Directory& d = dirs[(size_t)s.peer];
             char* win = (char*)c->peer_windows[s.peer];
-            ReqDesc rd;
-            st = desc_for(s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, &rd);
+            uint32_t items = 0;
+            st = add_req(xb, s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, &items);
             XInfo x{};
             x.flag = (uint64_t)(uintptr_t)(win + 8 * match[(size_t)i]->flag_idx);
             x.counter = npack++;
-            x.nitems = desc_items(rd);
+            x.nitems = items;
             x.parity_stride = d.parity_stride;
-            xb.descs.push_back(rd);
             xb.xinfo.push_back(x);
         }
         for (int i = 0; i < nsend && st == DDT_OK; i++) {
@@ -558,15 +558,20 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         for (int i = 0; i < nrecv && st == DDT_OK; i++) {
             const auto& r = recvs[i];
             if (r.count * r.type->size == 0 || r.peer == c->rank) continue;
-            ReqDesc rd;
-            st = desc_for(r.type, OP_UNPACK, r.buf, mywin + RL.flags_bytes + RL.data_off[(size_t)i], r.count, &rd);
+            st = add_req(xb, r.type, OP_UNPACK, mywin + RL.flags_bytes + RL.data_off[(size_t)i], r.buf, r.count,
+                         nullptr);
             XInfo x{};
             x.flag = (uint64_t)(uintptr_t)(mywin + 8 * RL.flag_idx[(size_t)i]);
             x.parity_stride = RL.parity_stride;
-            xb.descs.push_back(rd);
             xb.xinfo.push_back(x);
         }
-        if (st == DDT_OK && !xb.descs.empty()) st = make_table(xb, h->x_l);
+        if (st == DDT_OK && !xb.descs.empty()) {
+            // completion-counter targets use the batch's item size
+            const int ub = choose_ub(xb, queue_sm_count(q));
+            for (size_t i = 0; i < xb.descs.size(); i++)
+                if (xb.descs[i].op == OP_PACK) xb.xinfo[i].nitems = desc_items(xb.descs[i], ub);
+            st = make_table(xb, h->x_l, queue_sm_count(q));
+        }
         size_t ctrl_bytes = sizeof(XCtrl) + sizeof(unsigned long long) * std::max<size_t>(npack, 1);
         if (st == DDT_OK) {
             cudaError_t e = cudaMalloc(&h->ctrl, ctrl_bytes);

@@ -37,8 +37,8 @@ struct ddt_queue_s {
         ddt_type_s* t;
         ddt_type_s* t2;  // DIRECT destination type (else nullptr)
         int64_t bytes;
-        ReqDesc desc;    // built at enqueue (O(1)); flush only serializes
-        ReqDesc aux;     // DIRECT destination layout
+        ReqDesc desc;    // source descriptor, built at enqueue (O(1)); flush only serializes
+        ReqDesc aux;     // destination descriptor
     };
     struct Batch {
         int64_t first, end;  // uid range
@@ -124,7 +124,7 @@ int64_t claim(ddt_queue_s* q) {
 }
 
 int64_t commit_req(ddt_queue_s* q, int op, ddt_type_s* t, ddt_type_s* t2, int64_t bytes, const ReqDesc& d,
-                   const ReqDesc* a) {
+                   const ReqDesc& a) {
     int64_t uid = q->tail++;
     auto& r = q->ring[(size_t)(uid % q->capacity)];
     r.uid = uid;
@@ -136,7 +136,7 @@ int64_t commit_req(ddt_queue_s* q, int op, ddt_type_s* t, ddt_type_s* t2, int64_
     r.bytes = bytes;
     r.desc = d;
     r.desc.uid_lo = (uint32_t)uid;
-    if (a) r.aux = *a;
+    r.aux = a;
     q->stats.requests++;
     return uid;
 }
@@ -150,19 +150,18 @@ int64_t enqueue(ddt_queue_s* q, int op, ddt_type_s* t, const void* src, int64_t 
     if (op == OP_UNPACK && bytes > 0 && t->layout.overlaps) return DDT_ERR_OVERLAP;
     int64_t c = claim(q);
     if (c < 0) return c;
-    ReqDesc desc;
-    std::memset(&desc, 0, sizeof(desc));
+    ReqDesc sd, dd;
+    std::memset(&sd, 0, sizeof(sd));
+    std::memset(&dd, 0, sizeof(dd));
     if (bytes > 0) {
         DeviceGuard g(q->device);
         DeviceLayout* dl = nullptr;
         ddt_status_t s = type_device_layout(t, q->device, &dl);
         if (s != DDT_OK) return s;
-        const void* nc = op == OP_PACK ? src : dst;
-        const void* pk = op == OP_PACK ? dst : src;
-        s = build_desc(t, dl, op, nc, pk, count, &desc);
+        s = build_request(op, t, dl, src, dst, count, &sd, &dd);
         if (s != DDT_OK) return s;
     }
-    return commit_req(q, op, t, nullptr, bytes, desc, nullptr);
+    return commit_req(q, op, t, nullptr, bytes, sd, dd);
 }
 
 ddt_status_t ensure_host_slot(ddt_queue_s* q, size_t bytes, ddt_queue_s::HostSlot** out) {
@@ -196,12 +195,7 @@ int64_t gather_pending(ddt_queue_s* q) {
     for (int64_t u = q->flushed; u < q->tail; u++) {
         auto& r = q->ring[(size_t)(u % q->capacity)];
         if (r.bytes == 0) continue;
-        ReqDesc d = r.desc;
-        if (r.op == OP_DIRECT) {
-            d.aux = (uint32_t)b.aux.size();
-            b.aux.push_back(r.aux);
-        }
-        b.descs.push_back(d);
+        b.add(r.desc, r.aux);
         moved += r.bytes;
     }
     return moved;
@@ -287,7 +281,7 @@ int64_t ddt_direct_enqueue(ddt_queue_t q, ddt_type_t src_type, const void* src, 
         if (s == DDT_OK) s = build_direct(src_type, dls, src, src_count, dst_type, dld, dst, dst_count, &d, &a);
         if (s != DDT_OK) return s;
     }
-    return commit_req(q, OP_DIRECT, src_type, dst_type, bytes, d, &a);
+    return commit_req(q, OP_DIRECT, src_type, dst_type, bytes, d, a);
 }
 
 int32_t ddt_flush(ddt_queue_t q) {
@@ -299,13 +293,13 @@ int32_t ddt_flush(ddt_queue_t q) {
     int32_t nflushed = (int32_t)(q->tail - q->flushed);
     if (!q->scratch.descs.empty()) {
         Launchable& L = q->launch;
-        make_launchable(q->scratch, true, L);
+        make_launchable(q->scratch, true, L, q->sm_count);
         if (L.form == 3) {
             size_t tb = device_table_bytes(q->scratch);
             ddt_queue_s::HostSlot* slot = nullptr;
             ddt_status_t s = ensure_host_slot(q, tb, &slot);
             if (s != DDT_OK) return q->sticky = s;
-            write_device_table(slot->p, q->scratch);
+            write_device_table(slot->p, q->scratch, L.ub);
             if (q->dev_cap < tb) {
                 if (q->dev_table) cudaFree(q->dev_table);  // synchronizes: old table no longer in use
                 size_t cap = std::max<size_t>(tb, 64 << 10);
@@ -405,10 +399,10 @@ ddt_status_t ddt_plan_create(ddt_queue_t q, ddt_plan_t* out) {
             }
     }
     if (!q->scratch.descs.empty()) {
-        make_launchable(q->scratch, true, p->launch);
+        make_launchable(q->scratch, true, p->launch, q->sm_count);
         if (p->launch.form == 3) {
             std::vector<uint8_t> host(device_table_bytes(q->scratch));
-            write_device_table(host.data(), q->scratch);
+            write_device_table(host.data(), q->scratch, p->launch.ub);
             cudaError_t e = cudaMalloc(&p->launch.dev, host.size());
             if (e == cudaSuccess) e = cudaMemcpy(p->launch.dev, host.data(), host.size(), cudaMemcpyHostToDevice);
             if (e != cudaSuccess) {

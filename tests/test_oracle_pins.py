@@ -176,7 +176,7 @@ def test_indexed_matches_concatenation(data):
         lb = ub = 0
     assert t.extent() == (lb, ub - lb)
     assert t.size == sum(bl) * esz
-    src = random_bytes(200, 9)
+    src = random_bytes(256, 9)
     off = 80
     got = oracle.pack(t, src, src_offset=off)
     parts = [src[off + s: off + s + b * esz] for s, b in zip(starts, bl)]
