@@ -212,23 +212,30 @@ typedef struct {
 } ddt_recv_t;
 
 /* Communication context.  nranks == 1 needs neither NCCL nor windows (every
- * message is a self message).  DDT_XCHG_NCCL needs nccl_comm (an ncclComm_t
- * from ddt_nccl_comm_create).  DDT_XCHG_P2P needs peer_windows[nranks] (device
- * pointers, valid on this device, to every rank's window -- this rank's own
- * included -- each of `window_bytes` >= ddt_halo_window_bytes()) and, for
- * nranks > 1, nccl_comm for the one-time metadata exchange at create.       */
+ * message is a self message).  The one-time plan metadata exchange (directory
+ * of tags / sizes / window offsets, and an agreed status) uses host_allgather
+ * when given -- any process group, e.g. torch.distributed over gloo or NCCL --
+ * else NCCL.  DDT_XCHG_NCCL needs nccl_comm (an ncclComm_t from
+ * ddt_nccl_comm_create) for its data path.  DDT_XCHG_P2P needs peer_windows
+ * [nranks] (device pointers, valid on this device, to every rank's window --
+ * this rank's own included -- each >= ddt_halo_window_bytes() bytes).
+ * host_allgather(ctx, send, bytes, recv) must gather `bytes` bytes from every
+ * rank into recv[nranks * bytes] in rank order and return 0 (collective). */
+typedef int32_t (*ddt_allgather_fn)(void* ctx, const void* send, int64_t bytes, void* recv);
 typedef struct {
     int32_t rank, nranks;
     void* nccl_comm;
     void* const* peer_windows;
     int64_t window_bytes;
+    ddt_allgather_fn host_allgather;
+    void* host_ctx;
 } ddt_comm_t;
 
 /* Bytes of window a rank needs for DDT_XCHG_P2P with the given receives. */
 ddt_status_t ddt_halo_window_bytes(int32_t nrecv, const ddt_recv_t* recvs, int64_t* bytes);
 /* Build the plan: validates, matches sizes with the peers (one metadata
- * exchange over NCCL when nranks > 1), allocates staging, builds the device
- * work tables once.  Collective over all ranks of the comm.
+ * exchange when nranks > 1), allocates staging, builds the device work tables
+ * once.  Collective over all ranks of the comm.
  * Errors: DDT_ERR_ARG, DDT_ERR_STATE, DDT_ERR_SIZE_MISMATCH, DDT_ERR_NCCL,
  * DDT_ERR_CUDA, DDT_ERR_NOMEM, DDT_ERR_OVERLAP.                              */
 ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* comm, int32_t nsend, const ddt_send_t* sends,

@@ -34,9 +34,12 @@ class ddt_recv_t(ctypes.Structure):
     _fields_ = [("peer", I32), ("tag", I32), ("type", P), ("buf", P), ("count", I64)]
 
 
+ALLGATHER_FN = ctypes.CFUNCTYPE(I32, P, P, I64, P)
+
+
 class ddt_comm_t(ctypes.Structure):
     _fields_ = [("rank", I32), ("nranks", I32), ("nccl_comm", P), ("peer_windows", ctypes.POINTER(P)),
-                ("window_bytes", I64)]
+                ("window_bytes", I64), ("host_allgather", ALLGATHER_FN), ("host_ctx", P)]
 
 
 class ddt_queue_stats_t(ctypes.Structure):

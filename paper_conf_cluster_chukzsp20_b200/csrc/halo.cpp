@@ -95,6 +95,8 @@ struct ddt_halo_s {
     cudaStream_t stream = nullptr;
     int rank = 0, nranks = 1, mode = DDT_XCHG_NCCL;
     void* comm = nullptr;
+    ddt_allgather_fn ag = nullptr;  // host all-gather for plan metadata (else NCCL)
+    void* ag_ctx = nullptr;
     std::vector<ddt_send_t> sends;
     std::vector<ddt_recv_t> recvs;
     // NCCL mode
@@ -224,8 +226,50 @@ ddt_status_t exchange_directories(ddt_halo_s* h, const std::vector<std::vector<i
     return DDT_OK;
 }
 
+// Host path: every rank all-gathers one blob = concat over destination p of
+// (len_p, directory_p...); rank r keeps section r of every peer's blob.
+ddt_status_t exchange_directories_host(ddt_halo_s* h, const std::vector<std::vector<int64_t>>& out,
+                                       std::vector<std::vector<int64_t>>& in) {
+    const int P = h->nranks;
+    std::vector<int64_t> blob;
+    for (int p = 0; p < P; p++) {
+        blob.push_back((int64_t)out[(size_t)p].size());
+        blob.insert(blob.end(), out[(size_t)p].begin(), out[(size_t)p].end());
+    }
+    int64_t mine = (int64_t)blob.size();
+    std::vector<int64_t> sizes((size_t)P);
+    if (h->ag(h->ag_ctx, &mine, 8, sizes.data()) != 0) {
+        set_error("host all-gather failed (sizes)");
+        return DDT_ERR_ARG;
+    }
+    int64_t mx = *std::max_element(sizes.begin(), sizes.end());
+    blob.resize((size_t)mx, 0);
+    std::vector<int64_t> all((size_t)(mx * P));
+    if (h->ag(h->ag_ctx, blob.data(), mx * 8, all.data()) != 0) {
+        set_error("host all-gather failed (directories)");
+        return DDT_ERR_ARG;
+    }
+    in.assign((size_t)P, {});
+    for (int q = 0; q < P; q++) {
+        const int64_t* b = all.data() + (size_t)q * (size_t)mx;
+        int64_t pos = 0;
+        for (int p = 0; p < P; p++) {
+            int64_t len = b[pos++];
+            if (p == h->rank) in[(size_t)q].assign(b + pos, b + pos + len);
+            pos += len;
+        }
+    }
+    return DDT_OK;
+}
+
 ddt_status_t agree(ddt_halo_s* h, ddt_status_t mine) {
     if (h->nranks == 1) return mine;
+    if (h->ag) {
+        std::vector<int32_t> all((size_t)h->nranks);
+        int32_t v = mine;
+        if (h->ag(h->ag_ctx, &v, 4, all.data()) != 0) return DDT_ERR_ARG;
+        return *std::min_element(all.begin(), all.end());
+    }
     const NcclApi* n = nccl();
     if (!n) return DDT_ERR_UNSUPPORTED;
     int32_t* d = nullptr;
@@ -319,7 +363,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     if (!q || !c || !out || nsend < 0 || nrecv < 0 || (nsend && !sends) || (nrecv && !recvs)) return DDT_ERR_ARG;
     if (mode != DDT_XCHG_NCCL && mode != DDT_XCHG_P2P) return DDT_ERR_ARG;
     if (c->nranks < 1 || c->rank < 0 || c->rank >= c->nranks) return DDT_ERR_ARG;
-    if (c->nranks > 1 && !c->nccl_comm) return DDT_ERR_ARG;
+    if (c->nranks > 1 && !c->nccl_comm && !c->host_allgather) return DDT_ERR_ARG;  // no metadata path
+    if (c->nranks > 1 && mode == DDT_XCHG_NCCL && !c->nccl_comm) return DDT_ERR_ARG;
     if (mode == DDT_XCHG_P2P && (!c->peer_windows || c->window_bytes <= 0)) return DDT_ERR_ARG;
     if (queue_sticky(q) != DDT_OK) return queue_sticky(q);
     // validate messages
@@ -359,6 +404,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     h->nranks = c->nranks;
     h->mode = mode;
     h->comm = c->nccl_comm;
+    h->ag = c->host_allgather;
+    h->ag_ctx = c->host_ctx;
     h->sends.assign(sends, sends + nsend);
     h->recvs.assign(recvs, recvs + nrecv);
     for (auto& s : h->sends) type_retain(s.type);
@@ -389,7 +436,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     }
     ddt_status_t st = DDT_OK;
     if (P > 1) {
-        st = exchange_directories(h, dir_out, dir_in);
+        st = h->ag ? exchange_directories_host(h, dir_out, dir_in) : exchange_directories(h, dir_out, dir_in);
         if (st != DDT_OK) {
             free_halo(h);
             return st;

@@ -1,23 +1,52 @@
 """Halo exchange plans (Alg 3, §IV-B) and the
 communicator plumbing under them.  Marshalling only (csrc/halo.cpp,
 csrc/comm.cpp); torch.distributed is used solely to broadcast the NCCL unique
-id and to all-gather CUDA-IPC window handles."""
+id, to all-gather CUDA-IPC window handles and, as a host all-gather callback,
+to carry the one-time plan metadata."""
 from __future__ import annotations
 
 import ctypes
 
-from ._abi import (lib, check, P, ddt_send_t, ddt_recv_t, ddt_comm_t, DDT_XCHG_NCCL, DDT_XCHG_P2P)
+from ._abi import (lib, check, P, ddt_send_t, ddt_recv_t, ddt_comm_t, ALLGATHER_FN, DDT_XCHG_NCCL,
+                   DDT_XCHG_P2P)
 from .queue import ptr_of
+
+
+def torch_allgather(group=None):
+    """A host all-gather over a torch.distributed group (gloo or NCCL): the
+    plan-metadata path of ddt_comm_t (plumbing, never the data path)."""
+    import torch.distributed as dist
+
+    def gather(send: bytes) -> list:
+        out = [None] * dist.get_world_size(group)
+        dist.all_gather_object(out, send, group=group)
+        return out
+    return gather
+
+
+def _c_allgather(gather):
+    def cb(ctx, send, nbytes, recv):
+        try:
+            parts = gather(ctypes.string_at(send, nbytes))
+            for i, b in enumerate(parts):
+                assert len(b) == nbytes
+                ctypes.memmove(recv + i * nbytes, b, nbytes)
+            return 0
+        except Exception:
+            return -1
+    return ALLGATHER_FN(cb)
 
 
 class Comm:
     """rank / nranks, an NCCL communicator (nranks > 1) and, for the P2P mode,
     the device pointers of every rank's receive window."""
 
-    def __init__(self, rank: int = 0, nranks: int = 1, device: int = 0, nccl_comm=None, group=None):
+    def __init__(self, rank: int = 0, nranks: int = 1, device: int = 0, nccl_comm=None, group=None, gather=None):
         self.rank, self.nranks, self.device = int(rank), int(nranks), int(device)
         self.nccl_comm = nccl_comm
         self.group = group
+        self.gather = gather        # python all-gather of bytes (metadata plumbing)
+        self._cb = _c_allgather(gather) if gather is not None else None
         self.window = None          # own window (device pointer)
         self.window_bytes = 0
         self.peer_windows = None    # ctypes array of device pointers (own included)
@@ -28,13 +57,15 @@ class Comm:
         return Comm(0, 1, device)
 
     @staticmethod
-    def from_torch(device: int, group=None) -> "Comm":
-        """One process per GPU under torch.distributed: creates an NCCL
-        communicator of the same ranks (unique id broadcast by the group)."""
+    def from_torch(device: int, group=None, nccl: bool = True) -> "Comm":
+        """One process per GPU under torch.distributed: plan metadata travels by
+        host all-gather over the group; with nccl=True an NCCL communicator of
+        the same ranks is created too (unique id broadcast by the group) for the
+        NCCL-mode data path."""
         import torch.distributed as dist
         rank, n = dist.get_rank(group), dist.get_world_size(group)
-        c = Comm(rank, n, device, group=group)
-        if n > 1:
+        c = Comm(rank, n, device, group=group, gather=torch_allgather(group) if n > 1 else None)
+        if n > 1 and nccl:
             uid = ctypes.create_string_buffer(128)
             if rank == 0:
                 check(lib().ddt_nccl_unique_id(uid), "ddt_nccl_unique_id")
@@ -57,9 +88,8 @@ class Comm:
         ptrs = [0] * self.nranks
         ptrs[self.rank] = ptr.value
         if self.nranks > 1:
-            import torch.distributed as dist
-            allh = [None] * self.nranks
-            dist.all_gather_object(allh, (bytes(handle.raw), int(nbytes)), group=self.group)
+            import pickle
+            allh = [pickle.loads(b) for b in self.gather(pickle.dumps((bytes(handle.raw), int(nbytes))))]
             for p, (h, nb) in enumerate(allh):
                 if p == self.rank:
                     continue
@@ -77,6 +107,8 @@ class Comm:
         c.nccl_comm = self.nccl_comm.value if isinstance(self.nccl_comm, P) else self.nccl_comm
         c.peer_windows = ctypes.cast(self.peer_windows, ctypes.POINTER(P)) if self.peer_windows else None
         c.window_bytes = self.window_bytes
+        if self._cb is not None:
+            c.host_allgather = self._cb
         return c
 
     def close(self):
