@@ -187,6 +187,21 @@ ddt_status_t ddt_plan_create(ddt_queue_t q, ddt_plan_t* out);
 ddt_status_t ddt_plan_launch(ddt_plan_t p);
 ddt_status_t ddt_plan_destroy(ddt_plan_t p);
 
+/* Scheduler trigger (2) of §IV-C: once the pending requests hold
+ * >= `bytes` packed bytes, the enqueue that crossed the threshold also flushes
+ * (the paper's fusion threshold; ~512 KB on V100, to be re-tuned on B200).
+ * 0 (the default) = launch only on explicit ddt_flush / ddt_wait (trigger (1),
+ * the synchronisation point).  Errors: DDT_ERR_ARG. */
+ddt_status_t ddt_queue_set_flush_threshold(ddt_queue_t q, int64_t bytes);
+/* Scheduler (3) per request: when enabled, the GPU thread that
+ * finishes a request's last work item writes its response status into
+ * host-mapped memory, so ddt_query reports DDT_COMPLETED for that request as
+ * soon as it is done -- before the rest of its fused batch -- without any host
+ * synchronisation.  Default off (batch-level completion by CUDA event; the
+ * per-item bookkeeping costs one atomic per work item).  Only between batches
+ * (DDT_ERR_STATE if requests are pending). */
+ddt_status_t ddt_queue_set_response_flags(ddt_queue_t q, int32_t enable);
+
 /* Counters since queue creation: requests enqueued, fused kernel launches,
  * flushes, packed bytes moved (pack + unpack).                              */
 typedef struct {

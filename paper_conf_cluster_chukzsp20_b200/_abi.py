@@ -73,6 +73,8 @@ PROTOTYPES = {
     "ddt_query": (I32, [P, I64, I32P]),
     "ddt_wait": (I32, [P]),
     "ddt_queue_get_stats": (I32, [P, ctypes.POINTER(ddt_queue_stats_t)]),
+    "ddt_queue_set_flush_threshold": (I32, [P, I64]),
+    "ddt_queue_set_response_flags": (I32, [P, I32]),
     "ddt_plan_create": (I32, [P, ctypes.POINTER(P)]),
     "ddt_plan_launch": (I32, [P]),
     "ddt_plan_destroy": (I32, [P]),

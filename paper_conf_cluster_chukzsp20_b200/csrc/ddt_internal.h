@@ -84,6 +84,9 @@ struct ddt_type_s {
     bool committed = false;
     ddt::Layout layout;
     std::map<int, ddt::DeviceLayout> dev;  // device ordinal -> device cache
+    // lock-free fast path of type_device_layout: the last (device, cache) pair
+    std::atomic<int> fast_dev{-1};
+    std::atomic<ddt::DeviceLayout*> fast_dl{nullptr};
 };
 
 namespace ddt {

@@ -65,18 +65,42 @@ static ddt_status_t layout_desc(ddt_type_s* t, const DeviceLayout* dl, const voi
     d->lw = (uint8_t)lw;
     d->extent = ext;
     if (L.kind == DDT_LAYOUT_STRIDED) {
-        Form f = L.form;
-        f.dims.insert(f.dims.begin(), Dim{count, ext});
-        normalize(f);
+        // dims = [(count, extent)] ++ layout dims, normalised without heap
+        // allocation (the same rules as normalize(): drop unit dims, fold a
+        // contiguous innermost dim into the segment, merge chained dims)
+        Dim dims[kMaxDims + 2];
+        int D = 0;
+        int64_t seg = L.form.seg_len;
+        if (count != 1) dims[D++] = Dim{count, ext};
+        for (const Dim& x : L.form.dims)
+            if (x.n != 1) dims[D++] = x;
+        bool changed = true;
+        while (changed) {
+            changed = false;
+            if (D > 0 && dims[D - 1].stride == seg) {
+                seg *= dims[D - 1].n;
+                D--;
+                changed = true;
+                continue;
+            }
+            for (int k = 0; k + 1 < D; k++) {
+                if (dims[k].stride == dims[k + 1].n * dims[k + 1].stride) {
+                    dims[k + 1].n *= dims[k].n;
+                    for (int j = k; j + 1 < D; j++) dims[j] = dims[j + 1];
+                    D--;
+                    changed = true;
+                    break;
+                }
+            }
+        }
         d->kind = K_STRIDED;
-        d->base = f.base;
-        d->vps = make_div((uint32_t)(f.seg_len >> lw));
-        if (f.dims.empty()) {
-            if (f.base == 0) d->kind = K_CONTIG;  // one contiguous run at the pointer itself
+        d->base = L.form.base;
+        d->vps = make_div((uint32_t)(seg >> lw));
+        if (D == 0) {
+            if (d->base == 0) d->kind = K_CONTIG;  // one contiguous run at the pointer itself
             d->ndim = 0;
             d->extent = 0;
         } else {
-            int D = (int)f.dims.size();
             if (D - 1 > kMaxDims) {
                 set_error("strided layout with too many dims after count folding");
                 return DDT_ERR_UNSUPPORTED;
@@ -84,11 +108,11 @@ static ddt_status_t layout_desc(ddt_type_s* t, const DeviceLayout* dl, const voi
             d->ndim = (uint8_t)(D - 1);
             // innermost first; the outermost dim is the final quotient (no division)
             for (int k = 0; k < D - 1; k++) {
-                const Dim& x = f.dims[(size_t)(D - 1 - k)];
+                const Dim& x = dims[D - 1 - k];
                 d->radix[k] = make_div((uint32_t)x.n);
                 d->stride[k] = x.stride;
             }
-            d->extent = f.dims[0].stride;
+            d->extent = dims[0].stride;
         }
     } else if (L.kind == DDT_LAYOUT_UNIFORM_LIST) {
         d->kind = L.off32 ? K_UNIFORM32 : K_UNIFORM64;

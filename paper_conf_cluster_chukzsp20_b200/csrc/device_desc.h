@@ -45,7 +45,7 @@ struct DivU32 {
 
 struct alignas(16) ReqDesc {
     uint64_t ptr;           // base pointer of this side (MPI buffer address or packed buffer)
-    uint64_t pad0;
+    uint64_t resp;          // source desc: host-mapped u32 response-status slot, 0 = none
     uint32_t nvec;          // vectors in the request (count*size / w), < 2^32
     uint8_t op;             // DescOp
     uint8_t kind;           // DescKind
@@ -63,7 +63,10 @@ struct alignas(16) ReqDesc {
     uint32_t list_n;        // general: number of segments per instance
     uint32_t uid_lo;        // low bits of the request UID (debug / tracing)
     uint32_t aux;           // source descriptors: index of the destination descriptor in aux[]
-    uint32_t pad2;
+    uint32_t resp_val;      // value written to *resp when the request's last item is done
+    uint64_t done_ctr;      // device u32 counter of finished items (reset by the finishing CTA)
+    uint32_t nitems;        // items of this request in its batch (set at flush)
+    uint32_t pad3;
 };
 
 // Exchange-only side info of a descriptor (fused P2P halo kernel).

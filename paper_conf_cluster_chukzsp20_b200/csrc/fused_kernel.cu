@@ -9,9 +9,9 @@
 //
 // B200 design: pure HBM-bound byte movement, no tensor
 // cores.  The host builds a work table (exclusive prefix sum of per-request
-// item counts); CTA b walks items b, b + gridDim.x, ... in
+// item counts); CTA b walks its contiguous range of items in
 // increasing order (grid <= resident CTAs on the 148 SMs), finds its request
-// with a binary search of the prefix, caches the descriptor in shared memory
+// with a binary search of the prefix, caches the descriptors in shared memory
 // and moves kItemVecs vectors of the request's packed stream.  Thread i of the
 // CTA takes vectors v0 + i + u*kThreads, so the packed side is perfectly
 // coalesced and the strided side is coalesced within each segment.  The vector
@@ -255,7 +255,12 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
     constexpr int kWords = (int)(sizeof(ReqDesc) / 16);
     constexpr int kXWords = (int)(sizeof(XInfo) / 16);
     uint32_t cur = 0xffffffffu, cur_first = 0;
-    for (uint32_t item = blockIdx.x; item < tv.total; item += gridDim.x) {
+    // blocked assignment: CTA b owns items [b*per, (b+1)*per) -- consecutive
+    // items usually share a request, so descriptors are (re)loaded rarely
+    const uint32_t per = (tv.total + gridDim.x - 1) / gridDim.x;
+    const uint32_t first = blockIdx.x * per;
+    const uint32_t last = min(tv.total, first + per);
+    for (uint32_t item = first; item < last; item++) {
         const uint32_t r = find_request(tv.prefix, tv.nreq, item);
         if (r != cur) {
             __syncthreads();  // every warp is done with the previous descriptor
@@ -302,6 +307,20 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
             }
         }
         run_desc<LW, SONLY>(sd, sa, v0, false, (int)tv.ub);
+        if constexpr (!XCHG) {
+            if (sd.resp) {  // scheduler (3): the CTA finishing the request's last item signals it
+                __syncthreads();
+                if (threadIdx.x == 0) {
+                    __threadfence();
+                    unsigned int* ctr = reinterpret_cast<unsigned int*>(sd.done_ctr);
+                    if (atomicAdd(ctr, 1u) + 1u == sd.nitems) {
+                        *ctr = 0u;
+                        __threadfence_system();
+                        *reinterpret_cast<volatile unsigned int*>(sd.resp) = sd.resp_val;
+                    }
+                }
+            }
+        }
         if constexpr (XCHG) {
             if (sd.op == OP_PACK && sx.flag) {
                 __syncthreads();  // the CTA's peer stores precede thread 0's release

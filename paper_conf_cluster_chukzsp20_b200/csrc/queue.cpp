@@ -66,6 +66,14 @@ struct ddt_queue_s {
     int sm_count = 148;
     HostBatch scratch;
     Launchable launch;
+    // §IV-C trigger (2): flush once the pending requests hold >= threshold bytes (0 = off)
+    int64_t threshold = 0;
+    int64_t pending_bytes = 0;
+    // scheduler (3) per request: GPU-written response status (host-mapped) + item counters
+    bool resp_on = false;
+    uint32_t* resp_host = nullptr;
+    uint32_t* resp_dev = nullptr;
+    uint32_t* done_ctr = nullptr;
 };
 
 namespace {
@@ -137,7 +145,15 @@ int64_t commit_req(ddt_queue_s* q, int op, ddt_type_s* t, ddt_type_s* t2, int64_
     r.desc = d;
     r.desc.uid_lo = (uint32_t)uid;
     r.aux = a;
+    if (q->resp_on && bytes > 0) {
+        size_t slot = (size_t)(uid % q->capacity);
+        r.desc.resp = (uint64_t)(uintptr_t)(q->resp_dev + slot);
+        r.desc.resp_val = (uint32_t)(uid + 1);
+        r.desc.done_ctr = (uint64_t)(uintptr_t)(q->done_ctr + slot);
+    }
     q->stats.requests++;
+    q->pending_bytes += bytes;
+    if (q->threshold > 0 && q->pending_bytes >= q->threshold) ddt_flush(q);  // errors are sticky
     return uid;
 }
 
@@ -154,7 +170,6 @@ int64_t enqueue(ddt_queue_s* q, int op, ddt_type_s* t, const void* src, int64_t 
     std::memset(&sd, 0, sizeof(sd));
     std::memset(&dd, 0, sizeof(dd));
     if (bytes > 0) {
-        DeviceGuard g(q->device);
         DeviceLayout* dl = nullptr;
         ddt_status_t s = type_device_layout(t, q->device, &dl);
         if (s != DDT_OK) return s;
@@ -198,6 +213,11 @@ int64_t gather_pending(ddt_queue_s* q) {
         b.add(r.desc, r.aux);
         moved += r.bytes;
     }
+    if (q->resp_on) {  // the finishing CTA compares its count with the request's item count
+        int ub = choose_ub(b, q->sm_count);
+        for (auto& d : b.descs) d.nitems = desc_items(d, ub);
+    }
+    q->pending_bytes = 0;
     return moved;
 }
 
@@ -246,8 +266,37 @@ ddt_status_t ddt_queue_destroy(ddt_queue_t q) {
             if (s.ev) cudaEventDestroy(s.ev);
         }
         if (q->dev_table) cudaFree(q->dev_table);
+        if (q->resp_host) cudaFreeHost(q->resp_host);
+        if (q->done_ctr) cudaFree(q->done_ctr);
     }
     delete q;
+    return DDT_OK;
+}
+
+ddt_status_t ddt_queue_set_flush_threshold(ddt_queue_t q, int64_t bytes) {
+    if (!q || bytes < 0) return DDT_ERR_ARG;
+    q->threshold = bytes;
+    if (bytes > 0 && q->pending_bytes >= bytes) {
+        int32_t f = ddt_flush(q);
+        if (f < 0) return f;
+    }
+    return DDT_OK;
+}
+
+ddt_status_t ddt_queue_set_response_flags(ddt_queue_t q, int32_t enable) {
+    if (!q) return DDT_ERR_ARG;
+    if (q->flushed != q->tail) return DDT_ERR_STATE;  // only between batches
+    if (enable && !q->resp_host) {
+        DeviceGuard g(q->device);
+        size_t n = (size_t)q->capacity;
+        cudaError_t e = cudaHostAlloc((void**)&q->resp_host, n * 4, cudaHostAllocMapped);
+        if (e == cudaSuccess) e = cudaHostGetDevicePointer((void**)&q->resp_dev, q->resp_host, 0);
+        if (e == cudaSuccess) e = cudaMalloc(&q->done_ctr, n * 4);
+        if (e == cudaSuccess) e = cudaMemset(q->done_ctr, 0, n * 4);
+        if (e != cudaSuccess) return cuda_fail("response flags", e);
+        std::memset(q->resp_host, 0, n * 4);
+    }
+    q->resp_on = enable != 0;
     return DDT_OK;
 }
 
@@ -274,7 +323,6 @@ int64_t ddt_direct_enqueue(ddt_queue_t q, ddt_type_t src_type, const void* src, 
     std::memset(&d, 0, sizeof(d));
     std::memset(&a, 0, sizeof(a));
     if (bytes > 0) {
-        DeviceGuard g(q->device);
         DeviceLayout *dls = nullptr, *dld = nullptr;
         ddt_status_t s = type_device_layout(src_type, q->device, &dls);
         if (s == DDT_OK) s = type_device_layout(dst_type, q->device, &dld);
@@ -340,6 +388,12 @@ ddt_status_t ddt_query(ddt_queue_t q, int64_t uid, int32_t* state) {
     }
     auto& r = q->ring[(size_t)(uid % q->capacity)];
     if (r.bytes == 0) {
+        *state = DDT_COMPLETED;
+        return q->sticky;
+    }
+    // response status written by the GPU for this very request
+    if (r.desc.resp && uid < q->flushed &&
+        *reinterpret_cast<volatile uint32_t*>(q->resp_host + uid % q->capacity) == (uint32_t)(uid + 1)) {
         *state = DDT_COMPLETED;
         return q->sticky;
     }

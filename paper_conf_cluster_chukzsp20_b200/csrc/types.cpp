@@ -582,12 +582,33 @@ static ddt_status_t flatten(ddt_type_s* t) {
 }
 
 ddt_status_t type_device_layout(ddt_type_s* t, int device, DeviceLayout** out) {
+    // strided layouts carry everything in the descriptor: nothing to upload
+    static DeviceLayout none;
+    if (t->layout.kind == DDT_LAYOUT_STRIDED || t->layout.kind == DDT_LAYOUT_EMPTY) {
+        *out = &none;
+        return DDT_OK;
+    }
+    if (t->fast_dev.load(std::memory_order_acquire) == device) {
+        *out = t->fast_dl.load(std::memory_order_acquire);
+        if (*out) return DDT_OK;
+    }
     std::lock_guard<std::mutex> g(t->mu);
     auto it = t->dev.find(device);
     if (it != t->dev.end()) {
         *out = &it->second;
+        t->fast_dl.store(&it->second, std::memory_order_release);
+        t->fast_dev.store(device, std::memory_order_release);
         return DDT_OK;
     }
+    int prev_dev = -1;  // uploads go to `device` (callers may run with another current device)
+    cudaGetDevice(&prev_dev);
+    if (prev_dev != device) cudaSetDevice(device);
+    struct Restore {
+        int d;
+        ~Restore() {
+            if (d >= 0) cudaSetDevice(d);
+        }
+    } restore{prev_dev};
     DeviceLayout dl;
     const Layout& L = t->layout;
     cudaError_t e = cudaSuccess;
@@ -619,6 +640,8 @@ ddt_status_t type_device_layout(ddt_type_s* t, int device, DeviceLayout** out) {
     }
     auto r = t->dev.emplace(device, dl);
     *out = &r.first->second;
+    t->fast_dl.store(&r.first->second, std::memory_order_release);
+    t->fast_dev.store(device, std::memory_order_release);
     return DDT_OK;
 }
 

@@ -38,7 +38,8 @@ class Queue:
         self.stream = stream
         handle = int(stream.cuda_stream) if hasattr(stream, "cuda_stream") else int(stream)
         out = P()
-        check(lib().ddt_queue_create(self.device, ctypes.c_void_p(handle), int(capacity), ctypes.byref(out)),
+        self._lib = lib()
+        check(self._lib.ddt_queue_create(self.device, ctypes.c_void_p(handle), int(capacity), ctypes.byref(out)),
               "ddt_queue_create")
         self._h = out
 
@@ -48,13 +49,13 @@ class Queue:
 
     def pack(self, t, src, count: int, dst_packed) -> int:
         """Scheduler (1): enqueue a packing request; returns its uid."""
-        return check(lib().ddt_pack_enqueue(self._h, t.handle, ctypes.c_void_p(ptr_of(src)), int(count),
-                                            ctypes.c_void_p(ptr_of(dst_packed))), "ddt_pack_enqueue")
+        rc = self._lib.ddt_pack_enqueue(self._h, t.handle, ptr_of(src), count, ptr_of(dst_packed))
+        return rc if rc >= 0 else check(rc, "ddt_pack_enqueue")
 
     def unpack(self, t, src_packed, count: int, dst) -> int:
         """Scheduler (1): enqueue an unpacking request; returns its uid."""
-        return check(lib().ddt_unpack_enqueue(self._h, t.handle, ctypes.c_void_p(ptr_of(src_packed)), int(count),
-                                              ctypes.c_void_p(ptr_of(dst))), "ddt_unpack_enqueue")
+        rc = self._lib.ddt_unpack_enqueue(self._h, t.handle, ptr_of(src_packed), count, ptr_of(dst))
+        return rc if rc >= 0 else check(rc, "ddt_unpack_enqueue")
 
     def direct(self, src_type, src, src_count: int, dst_type, dst, dst_count: int) -> int:
         """Enqueue a DirectIPC request: gather through src_type, scatter through
@@ -70,7 +71,8 @@ class Queue:
 
     def flush(self) -> int:
         """Scheduler (2): one fused launch for every pending request."""
-        return check(lib().ddt_flush(self._h), "ddt_flush")
+        rc = self._lib.ddt_flush(self._h)
+        return rc if rc >= 0 else check(rc, "ddt_flush")
 
     def query(self, uid: int) -> str:
         """Scheduler (4): 'pending' | 'busy' | 'completed'."""
@@ -80,6 +82,14 @@ class Queue:
 
     def wait(self):
         check(lib().ddt_wait(self._h), "ddt_wait")
+
+    def set_flush_threshold(self, nbytes: int):
+        """Auto-flush once pending requests hold >= nbytes (§IV-C); 0 = off."""
+        check(self._lib.ddt_queue_set_flush_threshold(self._h, int(nbytes)), "ddt_queue_set_flush_threshold")
+
+    def set_response_flags(self, enable: bool = True):
+        """GPU-written per-request completion."""
+        check(self._lib.ddt_queue_set_response_flags(self._h, 1 if enable else 0), "ddt_queue_set_response_flags")
 
     def stats(self) -> dict:
         s = ddt_queue_stats_t()

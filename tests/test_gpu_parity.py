@@ -307,3 +307,59 @@ def test_plan_replay(ddt, q, n):
         for i in range(n):
             assert_bytes_equal(got[i], oracle.pack(o, hs[i]), f"plan it={it} req={i}")
     plan.destroy()
+
+
+# --------------------------------------------------------------- scheduler triggers / response status
+def test_auto_flush_threshold(ddt):
+    """§IV-C trigger (2): the enqueue that makes the pending bytes reach the
+    threshold launches the batch; the results are unchanged."""
+    import torch
+    q2 = ddt.Queue()
+    spec, fp = config5_spec(65536)
+    o = oracle.Type(spec)
+    t = ddt.Type.from_spec(spec)
+    hs = random_bytes(8 * fp, 77).reshape(8, fp)
+    src = torch.from_numpy(hs).cuda()
+    dst = torch.zeros((8, 65536), dtype=torch.uint8, device="cuda")
+    q2.set_flush_threshold(3 * 65536)
+    uids = [q2.pack(t, src[i], 1, dst[i]) for i in range(8)]
+    st = q2.stats()
+    assert st["flushes"] == 2 and st["launches"] == 2  # after requests 3 and 6
+    assert q2.query(uids[7]) == "pending" and q2.query(uids[0]) in ("busy", "completed")
+    q2.wait()
+    assert q2.stats()["launches"] == 3
+    got = host(dst)
+    for i in range(8):
+        assert_bytes_equal(got[i], oracle.pack(o, hs[i]), f"threshold req {i}")
+    q2.destroy()
+
+
+def test_gpu_written_response_status(ddt):
+    """Scheduler (3) per request: a small request fused ahead of a
+    1 GiB request reports COMPLETED while the batch is still running."""
+    import torch
+    q3 = ddt.Queue()
+    q3.set_response_flags(True)
+    small_spec, sfp = config5_spec(4096)
+    big_spec, bfp = config5_spec(64 << 20)
+    ts, tb = ddt.Type.from_spec(small_spec), ddt.Type.from_spec(big_spec)
+    hs = random_bytes(sfp, 5)
+    s_src = torch.from_numpy(hs).cuda()
+    s_dst = torch.zeros(4096, dtype=torch.uint8, device="cuda")
+    b_src = torch.zeros((16, bfp), dtype=torch.uint8, device="cuda")
+    b_dst = torch.zeros((16, 64 << 20), dtype=torch.uint8, device="cuda")
+    torch.cuda.synchronize()
+    u_small = q3.pack(ts, s_src, 1, s_dst)
+    u_big = [q3.pack(tb, b_src[i], 1, b_dst[i]) for i in range(16)]
+    q3.flush()
+    early = False
+    stream = torch.cuda.current_stream()
+    for _ in range(200000):
+        if q3.query(u_small) == "completed":
+            early = not stream.query()
+            break
+    q3.wait()
+    assert all(q3.query(u) == "completed" for u in [u_small] + u_big)
+    assert early, "the small request's response status did not arrive before its batch finished"
+    assert_bytes_equal(host(s_dst), oracle.pack(oracle.Type(small_spec), hs), "response-flag batch")
+    q3.destroy()
