@@ -111,6 +111,7 @@ struct ddt_halo_s {
     int* err_dev = nullptr;
     uint64_t timeout_ns = 10ull * 1000 * 1000 * 1000;
     int grid_cap = 0;
+    bool x_flags = false;         // P2P plan has remote messages (flags); else the plain fused kernel runs
     // graph replay
     bool use_graph = false;
     cudaGraphExec_t gexec = nullptr;
@@ -312,7 +313,8 @@ void free_halo(ddt_halo_s* h) {
 
 ddt_status_t record_exchange(ddt_halo_s* h) {
     if (h->mode == DDT_XCHG_P2P) {
-        int e = launch_exchange(h->x_l, h->ctrl, h->err_dev, h->timeout_ns, h->stream, h->grid_cap);
+        int e = h->x_flags ? launch_exchange(h->x_l, h->ctrl, h->err_dev, h->timeout_ns, h->stream, h->grid_cap)
+                           : launch_fused(h->x_l, h->stream, h->grid_cap);  // self messages only: no signalling
         if (e) return cuda_fail("exchange kernel launch", e);
         return DDT_OK;
     }
@@ -612,6 +614,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             x.parity_stride = RL.parity_stride;
             xb.xinfo.push_back(x);
         }
+        for (const auto& x : xb.xinfo) h->x_flags |= x.flag != 0;
         if (st == DDT_OK && !xb.descs.empty()) {
             // completion-counter targets use the batch's item size
             const int ub = choose_ub(xb, queue_sm_count(q));
