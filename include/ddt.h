@@ -71,8 +71,12 @@ enum ddt_layout_kind { DDT_LAYOUT_EMPTY = 0, DDT_LAYOUT_STRIDED = 1, DDT_LAYOUT_
 /* Exchange modes. */
 enum ddt_xchg_mode {
     DDT_XCHG_NCCL = 0,  /* fused pack -> grouped ncclSend/ncclRecv per peer -> fused unpack */
-    DDT_XCHG_P2P = 1    /* ONE kernel: pack straight into peers' windows over NVLink,
+    DDT_XCHG_P2P = 1,   /* ONE kernel: pack straight into peers' windows over NVLink,
                            release a per-message flag, unpack each message on arrival */
+    DDT_XCHG_P2P_DIRECT = 2  /* ONE kernel, pack-free (DirectIPC): gather the
+                           send layout and scatter straight into the peer's receive layout
+                           through a CUDA-IPC mapping of its buffer, after the peer's
+                           "ready" flag; needs closed-form (strided) receive types */
 };
 
 typedef struct ddt_type_s* ddt_type_t;   /* opaque, library-owned, immutable after commit */

@@ -18,7 +18,7 @@ request list and launched by ``flush`` as one fused kernel (§IV-A, P:185-230);
 from __future__ import annotations
 
 from ._abi import (DDTError, lib, check, LAYOUT_KINDS, BASE_CODES, STATE_NAMES,  # noqa: F401
-                   DDT_XCHG_NCCL, DDT_XCHG_P2P, DDT_PENDING, DDT_BUSY, DDT_COMPLETED)
+                   DDT_XCHG_NCCL, DDT_XCHG_P2P, DDT_XCHG_P2P_DIRECT, DDT_PENDING, DDT_BUSY, DDT_COMPLETED)
 from .types import Type  # noqa: F401
 from .queue import Queue, Plan  # noqa: F401
 from .halo import Halo, Comm  # noqa: F401

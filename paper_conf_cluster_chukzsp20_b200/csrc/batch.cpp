@@ -87,11 +87,16 @@ static void to_param(const HostBatch& b, Launchable& out) {
 // The compact kernel variant applies when every source and destination
 // descriptor is closed-form (strided or contiguous) with one vector width.
 static int batch_variant(const HostBatch& b) {
-    if (b.descs.empty()) return 0;
-    int lw = b.descs[0].lw;
+    int lw = -1;
+    for (const ReqDesc& d : b.descs)
+        if (d.nvec) {
+            lw = d.lw;
+            break;
+        }
+    if (lw < 0) return 0;
     for (const auto* v : {&b.descs, &b.aux})
         for (const ReqDesc& d : *v)
-            if ((d.kind != K_STRIDED && d.kind != K_CONTIG) || d.lw != lw) return 0;
+            if (d.nvec && ((d.kind != K_STRIDED && d.kind != K_CONTIG) || d.lw != lw)) return 0;
     return 1 + lw;
 }
 

@@ -60,6 +60,28 @@ const NcclApi* nccl() {
     return g_nccl.ok ? &g_nccl : nullptr;
 }
 
+ddt_status_t alloc_base(const void* p, void** base) {
+    using GetRange = int (*)(unsigned long long*, size_t*, unsigned long long);
+    static GetRange fn = [] {
+        void* h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_NOLOAD);
+        if (!h) h = dlopen("libcuda.so.1", RTLD_NOW);
+        return h ? (GetRange)dlsym(h, "cuMemGetAddressRange_v2") : (GetRange) nullptr;
+    }();
+    if (!fn) {
+        set_error("cuMemGetAddressRange unavailable");
+        return DDT_ERR_UNSUPPORTED;
+    }
+    unsigned long long b = 0;
+    size_t sz = 0;
+    int r = fn(&b, &sz, (unsigned long long)(uintptr_t)p);
+    if (r != 0) {
+        set_error("cuMemGetAddressRange failed (" + std::to_string(r) + ")");
+        return DDT_ERR_CUDA;
+    }
+    *base = (void*)(uintptr_t)b;
+    return DDT_OK;
+}
+
 ddt_status_t nccl_fail(const char* what, int r) {
     const NcclApi* n = nccl();
     std::string m = std::string(what) + ": nccl error " + std::to_string(r);

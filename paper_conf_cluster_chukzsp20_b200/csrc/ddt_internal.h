@@ -103,10 +103,15 @@ ddt_status_t build_request(int op, ddt_type_s* t, const DeviceLayout* dl, const 
                            int64_t count, ReqDesc* s, ReqDesc* d);
 ddt_status_t build_direct(ddt_type_s* ts, const DeviceLayout* dls, const void* src, int64_t scount, ddt_type_s* td,
                           const DeviceLayout* dld, void* dst, int64_t dcount, ReqDesc* s, ReqDesc* d);
+ddt_status_t build_typed(ddt_type_s* t, const DeviceLayout* dl, const void* p, int64_t count, ReqDesc* d);
+ddt_status_t rescale_desc(ReqDesc* d, int lw);
+// Base address of the device allocation containing p (CUDA driver, for IPC).
+ddt_status_t alloc_base(const void* p, void** base);
 // Items of a descriptor at ub vectors per thread per item.
 inline uint32_t desc_items(const ReqDesc& d, int ub = kUnroll) {
     uint64_t per = (uint64_t)kThreads * (uint64_t)ub;
-    return (uint32_t)((d.nvec + per - 1) / per);
+    uint64_t n = (d.nvec + per - 1) / per;
+    return n ? (uint32_t)n : 1u;  // a data-free (signal / wait) request still owns one item
 }
 
 // A batch on the host: source descriptors (items come from these), their

@@ -173,4 +173,26 @@ ddt_status_t build_direct(ddt_type_s* ts, const DeviceLayout* dls, const void* s
     return DDT_OK;
 }
 
+// A typed descriptor at its own largest legal width (pack-free remote
+// transfers: the receiver publishes its destination side, the sender
+// rescales both sides to their common width).
+ddt_status_t build_typed(ddt_type_s* t, const DeviceLayout* dl, const void* p, int64_t count, ReqDesc* d) {
+    std::memset(d, 0, sizeof(*d));
+    return layout_desc(t, dl, p, count, side_lw(t, p, count), d);
+}
+
+// Re-express a closed-form descriptor at a smaller vector width.
+ddt_status_t rescale_desc(ReqDesc* d, int lw) {
+    if (lw > d->lw) return DDT_ERR_ARG;
+    if (d->kind != K_STRIDED && d->kind != K_CONTIG) return DDT_ERR_UNSUPPORTED;
+    const int sh = d->lw - lw;
+    uint64_t nvec = (uint64_t)d->nvec << sh;
+    uint64_t vps = (uint64_t)d->vps.d << sh;
+    if (nvec >= (1ull << 32) || vps >= (1ull << 32)) return DDT_ERR_UNSUPPORTED;
+    d->nvec = (uint32_t)nvec;
+    if (d->kind == K_STRIDED) d->vps = make_div((uint32_t)vps);
+    d->lw = (uint8_t)lw;
+    return DDT_OK;
+}
+
 }  // namespace ddt

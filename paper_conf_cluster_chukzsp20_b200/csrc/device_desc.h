@@ -31,7 +31,7 @@ constexpr int kItemVecs = kThreads * kUnroll;  // max vectors per work item
 // PACK: typed source -> contiguous destination; UNPACK: contiguous -> typed;
 // DIRECT: typed -> typed (the paper's DirectIPC op; self
 // messages of a halo exchange).  K_CONTIG is the packed side (offset = v * w).
-enum DescOp : uint8_t { OP_PACK = 0, OP_UNPACK = 1, OP_DIRECT = 2 };
+enum DescOp : uint8_t { OP_PACK = 0, OP_UNPACK = 1, OP_DIRECT = 2, OP_SIGNAL = 3 };  // SIGNAL: ready / wait items, no data
 enum DescKind : uint8_t { K_STRIDED = 0, K_UNIFORM32 = 1, K_UNIFORM64 = 2, K_GENERAL = 3, K_CONTIG = 4 };
 
 // Unsigned 32-bit division by a runtime constant d via a 64-bit reciprocal:
@@ -70,12 +70,20 @@ struct alignas(16) ReqDesc {
 };
 
 // Exchange-only side info of a descriptor (fused P2P halo kernel).
+// Per item of request r:  [wait] -> move the data -> [signal].
+//   remote pack   : signal = the peer's flag for this message
+//   unpack        : wait   = own flag of the message (written by the sender)
+//   remote direct : wait   = own "ready" slot of the peer (the peer entered this
+//                   exchange, its ghosts are free), signal = the peer's done flag
+//   ready         : no data; signal = own slot in the peer's ready array
+//   wait          : no data; wait = own done flag of an incoming direct message
+// Flags hold the exchange epoch (monotonic, never reset).
 struct alignas(16) XInfo {
-    uint64_t flag;          // pack: peer's flag slot; unpack: own flag slot (u64 epoch); 0 = none
-    uint32_t counter;       // pack: index of the per-message completion counter
-    uint32_t nitems;        // pack: items of the message (counter target = epoch * nitems)
-    int64_t parity_stride;  // window half size: iteration e uses half (e & 1)
-    int64_t pad;
+    uint64_t signal;        // release `epoch` here once every item of the message moved, 0 = none
+    uint64_t wait;          // acquire-wait until *wait >= epoch before moving, 0 = none
+    uint32_t counter;       // multi-item messages: index of the completion counter
+    uint32_t nitems;        // items of the message (signal when all are done)
+    int64_t parity_stride;  // window half size: the window side moves by (epoch & 1) * stride
 };
 
 // Header of a device batch table:

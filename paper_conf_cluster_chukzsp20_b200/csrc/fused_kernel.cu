@@ -282,10 +282,11 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
             cur = r;
         }
         const uint32_t v0 = (item - cur_first) * (uint32_t)(kThreads * tv.ub);
+        bool run = true;
         if constexpr (XCHG) {
-            if (sd.op == OP_UNPACK && sx.flag) {
+            if (sx.wait) {  // acquire: the peer's data / ready signal has arrived
                 if (threadIdx.x == 0) {
-                    const uint64_t* flag = reinterpret_cast<const uint64_t*>(sx.flag);
+                    const uint64_t* flag = reinterpret_cast<const uint64_t*>(sx.wait);
                     int ok = 1;
                     if (ld_acquire_sys(flag) < epoch) {
                         const uint64_t t0 = globaltimer();
@@ -302,11 +303,10 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
                     s_ok = ok;
                 }
                 __syncthreads();
-                if (s_ok) run_desc<LW, SONLY>(sd, sa, v0, true, (int)tv.ub);
-                continue;
+                run = s_ok != 0;
             }
         }
-        run_desc<LW, SONLY>(sd, sa, v0, false, (int)tv.ub);
+        if (run) run_desc<LW, SONLY>(sd, sa, v0, XCHG && sd.op == OP_UNPACK, (int)tv.ub);
         if constexpr (!XCHG) {
             if (sd.resp) {  // scheduler (3): the CTA finishing the request's last item signals it
                 __syncthreads();
@@ -322,17 +322,17 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
             }
         }
         if constexpr (XCHG) {
-            if (sd.op == OP_PACK && sx.flag) {
-                __syncthreads();  // the CTA's peer stores precede thread 0's release
+            if (sx.signal) {  // release once every item of the message has moved
+                __syncthreads();  // the CTA's (peer) stores precede thread 0's release
                 if (threadIdx.x == 0) {
-                    if (sx.nitems == 1) {
-                        st_release_sys(reinterpret_cast<uint64_t*>(sx.flag), epoch);
+                    if (sx.nitems <= 1) {
+                        st_release_sys(reinterpret_cast<uint64_t*>(sx.signal), epoch);
                     } else {
                         __threadfence_system();
                         unsigned long long old = atomicAdd_system(&ctrl->counters[sx.counter], 1ull);
                         if (old + 1ull == epoch * (unsigned long long)sx.nitems) {
                             __threadfence_system();
-                            st_release_sys(reinterpret_cast<uint64_t*>(sx.flag), epoch);
+                            st_release_sys(reinterpret_cast<uint64_t*>(sx.signal), epoch);
                         }
                     }
                 }

@@ -46,6 +46,7 @@ struct RecvLayout {
     std::vector<int> order;          // recv indices sorted by (peer, tag)
     std::vector<int64_t> data_off;   // per recv index: offset inside one parity half
     std::vector<int> flag_idx;       // per recv index
+    int64_t ready_off = 0;           // byte offset of the per-sender "ready" slots (pack-free mode)
     int64_t flags_bytes = 0, parity_stride = 0, window_bytes = 0;
 };
 
@@ -67,7 +68,10 @@ RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs) {
         L.flag_idx[(size_t)i] = (int)k;
         off += bytes;
     }
-    L.flags_bytes = round_up(std::max<int64_t>(8 * (int64_t)nrecv, 8), 256);
+    int64_t nready = 0;  // one slot per possible sender rank
+    for (int i = 0; i < nrecv; i++) nready = std::max<int64_t>(nready, (int64_t)recvs[i].peer + 1);
+    L.ready_off = 8 * (int64_t)nrecv;
+    L.flags_bytes = round_up(std::max<int64_t>(8 * ((int64_t)nrecv + nready), 8), 256);
     L.parity_stride = round_up(std::max<int64_t>(off, 16), 256);
     L.window_bytes = L.flags_bytes + 2 * L.parity_stride;
     return L;
@@ -75,11 +79,17 @@ RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs) {
 
 struct DirEntry {
     int64_t tag, bytes, data_off, flag_idx;
+    // pack-free mode: where the receive buffer lives and how it is laid out
+    int64_t ipc[8];      // cudaIpcMemHandle_t of the buffer's allocation
+    int64_t alloc_off;   // buffer address - allocation base
+    ReqDesc desc;        // receiver's typed descriptor (ptr = 0), at its widest legal width
 };
 struct Directory {  // what a receiver tells one sender
-    int64_t parity_stride = 0, data_base = 0;
+    int64_t parity_stride = 0, data_base = 0, ready_base = 0, direct = 0;
     std::vector<DirEntry> e;  // sorted by tag
 };
+constexpr int kDescWords = (int)(sizeof(ReqDesc) / 8);
+static_assert(sizeof(cudaIpcMemHandle_t) == 64, "IPC handle size");
 
 struct Xfer {
     int peer;
@@ -112,6 +122,7 @@ struct ddt_halo_s {
     uint64_t timeout_ns = 10ull * 1000 * 1000 * 1000;
     int grid_cap = 0;
     bool x_flags = false;         // P2P plan has remote messages (flags); else the plain fused kernel runs
+    std::vector<void*> ipc_opened;  // peers' receive buffers mapped for pack-free writes
     // graph replay
     bool use_graph = false;
     cudaGraphExec_t gexec = nullptr;
@@ -286,14 +297,31 @@ ddt_status_t agree(ddt_halo_s* h, ddt_status_t mine) {
     return res;
 }
 
+// [n, parity_stride, data_base, ready_base, direct] then n entries of
+// [tag, bytes, data_off, flag_idx] (+ [ipc x8, alloc_off, desc x kDescWords] if direct)
 Directory parse_dir(const std::vector<int64_t>& v) {
     Directory d;
-    if (v.size() < 3) return d;
+    if (v.size() < 5) return d;
     int64_t n = v[0];
     d.parity_stride = v[1];
     d.data_base = v[2];
-    for (int64_t i = 0; i < n && (size_t)(3 + 4 * i + 3) < v.size(); i++)
-        d.e.push_back({v[(size_t)(3 + 4 * i)], v[(size_t)(4 + 4 * i)], v[(size_t)(5 + 4 * i)], v[(size_t)(6 + 4 * i)]});
+    d.ready_base = v[3];
+    d.direct = v[4];
+    size_t pos = 5;
+    const size_t stride = 4 + (d.direct ? 9 + kDescWords : 0);
+    for (int64_t i = 0; i < n && pos + stride <= v.size(); i++, pos += stride) {
+        DirEntry e{};
+        e.tag = v[pos];
+        e.bytes = v[pos + 1];
+        e.data_off = v[pos + 2];
+        e.flag_idx = v[pos + 3];
+        if (d.direct) {
+            std::memcpy(e.ipc, &v[pos + 4], 64);
+            e.alloc_off = v[pos + 12];
+            std::memcpy(&e.desc, &v[pos + 13], sizeof(ReqDesc));
+        }
+        d.e.push_back(e);
+    }
     return d;
 }
 
@@ -306,13 +334,14 @@ void free_halo(ddt_halo_s* h) {
     cudaFree(h->x_l.dev);
     cudaFree(h->ctrl);
     if (h->err_host) cudaFreeHost(h->err_host);
+    for (void* p : h->ipc_opened) cudaIpcCloseMemHandle(p);
     for (auto& s : h->sends) type_release(s.type);
     for (auto& r : h->recvs) type_release(r.type);
     delete h;
 }
 
 ddt_status_t record_exchange(ddt_halo_s* h) {
-    if (h->mode == DDT_XCHG_P2P) {
+    if (h->mode != DDT_XCHG_NCCL) {
         int e = h->x_flags ? launch_exchange(h->x_l, h->ctrl, h->err_dev, h->timeout_ns, h->stream, h->grid_cap)
                            : launch_fused(h->x_l, h->stream, h->grid_cap);  // self messages only: no signalling
         if (e) return cuda_fail("exchange kernel launch", e);
@@ -363,11 +392,13 @@ ddt_status_t ddt_halo_window_bytes(int32_t nrecv, const ddt_recv_t* recvs, int64
 ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, const ddt_send_t* sends, int32_t nrecv,
                              const ddt_recv_t* recvs, int32_t mode, ddt_halo_t* out) {
     if (!q || !c || !out || nsend < 0 || nrecv < 0 || (nsend && !sends) || (nrecv && !recvs)) return DDT_ERR_ARG;
-    if (mode != DDT_XCHG_NCCL && mode != DDT_XCHG_P2P) return DDT_ERR_ARG;
+    if (mode != DDT_XCHG_NCCL && mode != DDT_XCHG_P2P && mode != DDT_XCHG_P2P_DIRECT) return DDT_ERR_ARG;
+    const bool p2p = mode != DDT_XCHG_NCCL;
+    const bool direct = mode == DDT_XCHG_P2P_DIRECT;
     if (c->nranks < 1 || c->rank < 0 || c->rank >= c->nranks) return DDT_ERR_ARG;
     if (c->nranks > 1 && !c->nccl_comm && !c->host_allgather) return DDT_ERR_ARG;  // no metadata path
     if (c->nranks > 1 && mode == DDT_XCHG_NCCL && !c->nccl_comm) return DDT_ERR_ARG;
-    if (mode == DDT_XCHG_P2P && (!c->peer_windows || c->window_bytes <= 0)) return DDT_ERR_ARG;
+    if (p2p && (!c->peer_windows || c->window_bytes <= 0)) return DDT_ERR_ARG;
     if (queue_sticky(q) != DDT_OK) return queue_sticky(q);
     // validate messages
     std::map<std::pair<int, int>, int> seen_s, seen_r;
@@ -386,7 +417,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         if (r.count * r.type->size > 0 && r.type->layout.overlaps) return DDT_ERR_OVERLAP;
         if (!seen_r.emplace(std::make_pair(r.peer, r.tag), i).second) return DDT_ERR_ARG;
     }
-    if (mode == DDT_XCHG_P2P) {  // symmetric pattern required by the parity double buffering
+    if (p2p) {  // symmetric pattern required by the parity double buffering / ready handshake
         for (auto& kv : seen_s)
             if (kv.first.first != c->rank) {
                 bool back = false;
@@ -416,7 +447,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
 
     // ---- receive layout and directories (receiver -> each sender)
     RecvLayout RL = layout_recvs(nrecv, recvs);
-    if (mode == DDT_XCHG_P2P && c->window_bytes < RL.window_bytes) {
+    if (p2p && c->window_bytes < RL.window_bytes) {
         free_halo(h);
         set_error("window smaller than ddt_halo_window_bytes()");
         return DDT_ERR_ARG;
@@ -428,12 +459,40 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         for (int k : RL.order)
             if (recvs[k].peer == p) mine.push_back(k);
         auto& v = dir_out[(size_t)p];
-        v = {(int64_t)mine.size(), RL.parity_stride, RL.flags_bytes};
+        const bool dmsg = direct && p != c->rank;
+        v = {(int64_t)mine.size(), RL.parity_stride, RL.flags_bytes, RL.ready_off, dmsg ? 1 : 0};
         for (int k : mine) {
             v.push_back(recvs[k].tag);
             v.push_back(recvs[k].count * recvs[k].type->size);
             v.push_back(RL.data_off[(size_t)k]);
             v.push_back(RL.flag_idx[(size_t)k]);
+            if (!dmsg) continue;
+            // pack-free: publish the receive buffer (IPC handle + offset) and its layout
+            int64_t words[9 + kDescWords] = {0};
+            ReqDesc d;
+            DeviceLayout* dl = nullptr;
+            void* base = nullptr;
+            cudaIpcMemHandle_t ih;
+            ddt_status_t s2 = type_device_layout(recvs[k].type, h->device, &dl);
+            if (s2 == DDT_OK) s2 = build_typed(recvs[k].type, dl, recvs[k].buf, recvs[k].count, &d);
+            if (s2 == DDT_OK && d.kind != K_STRIDED && d.kind != K_CONTIG) {
+                set_error("pack-free exchange needs closed-form (strided) receive types");
+                s2 = DDT_ERR_UNSUPPORTED;
+            }
+            if (s2 == DDT_OK) s2 = alloc_base(recvs[k].buf, &base);
+            if (s2 == DDT_OK) {
+                cudaError_t e = cudaIpcGetMemHandle(&ih, base);
+                if (e != cudaSuccess) s2 = cuda_fail("cudaIpcGetMemHandle(recv buffer)", e);
+            }
+            if (s2 != DDT_OK) {
+                free_halo(h);
+                return s2;
+            }
+            d.ptr = 0;
+            std::memcpy(words, &ih, 64);
+            words[8] = (int64_t)((const char*)recvs[k].buf - (const char*)base);
+            std::memcpy(words + 9, &d, sizeof(ReqDesc));
+            v.insert(v.end(), words, words + 9 + kDescWords);
         }
     }
     ddt_status_t st = DDT_OK;
@@ -580,22 +639,40 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         if (st == DDT_OK && !unpackb.descs.empty()) st = make_table(unpackb, h->unpack_l, queue_sm_count(q));
         h->launches = (packb.descs.empty() ? 0 : 1) + (unpackb.descs.empty() ? 0 : 1);
     } else {
-        // P2P: one kernel; items ordered remote packs, self directs, then the
-        // unpacks that wait on flags (deadlock-freedom order, fused_kernel.cu)
+        // P2P: one kernel.  Item order = deadlock-freedom order (fused_kernel.cu):
+        // items that never wait first (ready signals, remote packs, self directs),
+        // then pack-free remote directs (wait for the peer's ready flag), then the
+        // items that wait for data (unpacks / completion waits).
         HostBatch xb;
         char* mywin = (char*)c->peer_windows[c->rank];
         uint32_t npack = 0;
-        for (int i = 0; i < nsend && st == DDT_OK; i++) {
+        ReqDesc none;
+        std::memset(&none, 0, sizeof(none));
+        none.kind = K_CONTIG;
+        none.op = OP_SIGNAL;
+        std::vector<int> rpeers;  // remote peers we receive from (== send to: symmetric)
+        for (int i = 0; i < nrecv; i++)
+            if (recvs[i].peer != c->rank && recvs[i].count * recvs[i].type->size > 0) rpeers.push_back(recvs[i].peer);
+        std::sort(rpeers.begin(), rpeers.end());
+        rpeers.erase(std::unique(rpeers.begin(), rpeers.end()), rpeers.end());
+        if (direct) {  // "ready": this rank entered the exchange, its ghosts may be overwritten
+            for (int p : rpeers) {
+                XInfo x{};
+                x.signal = (uint64_t)(uintptr_t)((char*)c->peer_windows[p] + dirs[(size_t)p].ready_base + 8 * c->rank);
+                x.nitems = 1;
+                xb.add(none, none);
+                xb.xinfo.push_back(x);
+            }
+        }
+        for (int i = 0; i < nsend && st == DDT_OK && !direct; i++) {
             const auto& s = sends[i];
             if (s.count * s.type->size == 0 || s.peer == c->rank) continue;
             const Directory& d = dirs[(size_t)s.peer];
             char* win = (char*)c->peer_windows[s.peer];
-            uint32_t items = 0;
-            st = add_req(xb, s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, &items);
+            st = add_req(xb, s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, nullptr);
             XInfo x{};
-            x.flag = (uint64_t)(uintptr_t)(win + 8 * match[(size_t)i]->flag_idx);
+            x.signal = (uint64_t)(uintptr_t)(win + 8 * match[(size_t)i]->flag_idx);
             x.counter = npack++;
-            x.nitems = items;
             x.parity_stride = d.parity_stride;
             xb.xinfo.push_back(x);
         }
@@ -604,22 +681,57 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             if (s.count * s.type->size == 0 || s.peer != c->rank) continue;
             st = add_direct(xb, s, recvs[self_recv(s.tag)], true);
         }
+        for (int i = 0; i < nsend && st == DDT_OK && direct; i++) {
+            const auto& s = sends[i];
+            if (s.count * s.type->size == 0 || s.peer == c->rank) continue;
+            const DirEntry& e = *match[(size_t)i];
+            cudaIpcMemHandle_t ih;
+            std::memcpy(&ih, e.ipc, 64);
+            void* mapped = nullptr;
+            cudaError_t ce = cudaIpcOpenMemHandle(&mapped, ih, cudaIpcMemLazyEnablePeerAccess);
+            if (ce != cudaSuccess) {
+                st = cuda_fail("cudaIpcOpenMemHandle(peer recv buffer)", ce);
+                break;
+            }
+            h->ipc_opened.push_back(mapped);
+            ReqDesc sd, dd = e.desc;
+            dd.ptr = (uint64_t)(uintptr_t)((char*)mapped + e.alloc_off);
+            DeviceLayout* dl = nullptr;
+            st = type_device_layout(s.type, h->device, &dl);
+            if (st == DDT_OK) st = build_typed(s.type, dl, s.buf, s.count, &sd);
+            const int lw = std::min<int>(sd.lw, dd.lw);
+            if (st == DDT_OK && sd.lw != lw) st = rescale_desc(&sd, lw);
+            if (st == DDT_OK && dd.lw != lw) st = rescale_desc(&dd, lw);
+            if (st == DDT_OK && sd.nvec != dd.nvec) st = DDT_ERR_SIZE_MISMATCH;
+            if (st != DDT_OK) break;
+            sd.op = dd.op = OP_DIRECT;
+            xb.add(sd, dd);
+            XInfo x{};
+            x.signal = (uint64_t)(uintptr_t)((char*)c->peer_windows[s.peer] + 8 * e.flag_idx);
+            x.wait = (uint64_t)(uintptr_t)(mywin + RL.ready_off + 8 * s.peer);
+            x.counter = npack++;
+            xb.xinfo.push_back(x);
+        }
         for (int i = 0; i < nrecv && st == DDT_OK; i++) {
             const auto& r = recvs[i];
             if (r.count * r.type->size == 0 || r.peer == c->rank) continue;
-            st = add_req(xb, r.type, OP_UNPACK, mywin + RL.flags_bytes + RL.data_off[(size_t)i], r.buf, r.count,
-                         nullptr);
             XInfo x{};
-            x.flag = (uint64_t)(uintptr_t)(mywin + 8 * RL.flag_idx[(size_t)i]);
-            x.parity_stride = RL.parity_stride;
+            x.wait = (uint64_t)(uintptr_t)(mywin + 8 * RL.flag_idx[(size_t)i]);
+            if (direct) {  // the data lands by itself; wait for its completion flag
+                xb.add(none, none);
+            } else {
+                st = add_req(xb, r.type, OP_UNPACK, mywin + RL.flags_bytes + RL.data_off[(size_t)i], r.buf, r.count,
+                             nullptr);
+                x.parity_stride = RL.parity_stride;
+            }
             xb.xinfo.push_back(x);
         }
-        for (const auto& x : xb.xinfo) h->x_flags |= x.flag != 0;
+        for (const auto& x : xb.xinfo) h->x_flags |= x.signal != 0 || x.wait != 0;
         if (st == DDT_OK && !xb.descs.empty()) {
             // completion-counter targets use the batch's item size
             const int ub = choose_ub(xb, queue_sm_count(q));
             for (size_t i = 0; i < xb.descs.size(); i++)
-                if (xb.descs[i].op == OP_PACK) xb.xinfo[i].nitems = desc_items(xb.descs[i], ub);
+                if (xb.xinfo[i].signal) xb.xinfo[i].nitems = desc_items(xb.descs[i], ub);
             st = make_table(xb, h->x_l, queue_sm_count(q));
         }
         size_t ctrl_bytes = sizeof(XCtrl) + sizeof(unsigned long long) * std::max<size_t>(npack, 1);

@@ -8,7 +8,7 @@ from __future__ import annotations
 import ctypes
 
 from ._abi import (lib, check, P, ddt_send_t, ddt_recv_t, ddt_comm_t, ALLGATHER_FN, DDT_XCHG_NCCL,
-                   DDT_XCHG_P2P)
+                   DDT_XCHG_P2P, DDT_XCHG_P2P_DIRECT)
 from .queue import ptr_of
 
 
@@ -135,15 +135,17 @@ def _msgs(items, cls):
 class Halo:
     """A persistent exchange plan.  sends / recvs: lists of
     (peer, tag, Type, buffer, count); a send to (peer, tag) matches the peer's
-    receive from (this rank, tag)."""
+    receive from (this rank, tag).  mode: "nccl" (fused pack -> NCCL send/recv
+    -> fused unpack), "p2p" (one kernel through peers' windows) or
+    "p2p_direct" (one pack-free kernel writing peers' receive buffers)."""
 
     def __init__(self, queue, comm: Comm, sends, recvs, mode: str = "nccl", graph: bool = True):
         self.queue, self.comm = queue, comm
         self._keep = [m[2] for m in sends] + [m[2] for m in recvs]
         s_arr = _msgs(sends, ddt_send_t)
         r_arr = _msgs(recvs, ddt_recv_t)
-        self.mode = DDT_XCHG_P2P if mode == "p2p" else DDT_XCHG_NCCL
-        if self.mode == DDT_XCHG_P2P and comm.window is None:
+        self.mode = {"nccl": DDT_XCHG_NCCL, "p2p": DDT_XCHG_P2P, "p2p_direct": DDT_XCHG_P2P_DIRECT}[mode]
+        if self.mode != DDT_XCHG_NCCL and comm.window is None:
             nb = ctypes.c_int64()
             check(lib().ddt_halo_window_bytes(len(recvs), r_arr, ctypes.byref(nb)), "ddt_halo_window_bytes")
             comm.setup_windows(nb.value)

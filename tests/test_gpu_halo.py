@@ -69,7 +69,7 @@ def _check(arrs, local, dirs, before=None):
         assert np.all(h.view(np.uint8).reshape(h.shape + (8,))[rest] == 0xA5)
 
 
-@pytest.mark.parametrize("mode", ["nccl", "p2p"])
+@pytest.mark.parametrize("mode", ["nccl", "p2p", "p2p_direct"])
 @pytest.mark.parametrize("graph", [False, True])
 @pytest.mark.parametrize("local,dirs,nvars,cfg", [
     ((5, 6, 7), ALL_DIRS, 2, 4),

@@ -17,7 +17,7 @@ from mp_util import free_port, init  # noqa: E402
 pytestmark = pytest.mark.gpu
 
 
-def _worker(rank, world, port, dirs_name, iters, q):
+def _worker(rank, world, port, dirs_name, iters, mode, q):
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     ok = False
     try:
@@ -50,7 +50,7 @@ def _worker(rank, world, port, dirs_name, iters, q):
         recvs = [(m["recv_peer"], m["recv_tag"], T(m["recv_spec"]), arrs[m["var"]], 1) for m in msgs]
         comm = ddt.Comm.from_torch(0, nccl=False)
         qq = ddt.Queue()
-        h = ddt.Halo(qq, comm, sends, recvs, mode="p2p", graph=(iters % 2 == 0))
+        h = ddt.Halo(qq, comm, sends, recvs, mode=mode, graph=(iters % 2 == 0))
         ok = True
         gm = ghost_mask(local, dirs)
         for it in range(iters):
@@ -80,13 +80,15 @@ def _worker(rank, world, port, dirs_name, iters, q):
 
 
 @pytest.mark.timeout(600)
-@pytest.mark.parametrize("world,dirs_name,iters", [(2, "faces", 3), (2, "all", 4), (4, "all", 3), (8, "faces", 2)])
-def test_p2p_exchange_multiprocess_one_gpu(world, dirs_name, iters):
+@pytest.mark.parametrize("world,dirs_name,iters,mode", [(2, "faces", 3, "p2p"), (2, "all", 4, "p2p"), (4, "all", 3, "p2p"),
+                                                       (8, "faces", 2, "p2p"), (2, "all", 4, "p2p_direct"),
+                                                       (4, "all", 3, "p2p_direct"), (8, "faces", 2, "p2p_direct")])
+def test_p2p_exchange_multiprocess_one_gpu(world, dirs_name, iters, mode):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, dirs_name, iters, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, dirs_name, iters, mode, q)) for r in range(world)]
     for p in procs:
         p.start()
     res = {}
