@@ -313,7 +313,7 @@ def main():
     ap.add_argument("--steps", type=int, default=500)
     ap.add_argument("--warmup", type=int, default=50)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--mode", default="auto", choices=["auto", "p2p", "nccl"])
+    ap.add_argument("--mode", default="auto", choices=["auto", "p2p", "p2p_direct", "nccl"])
     ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0)
     args = ap.parse_args()
@@ -398,7 +398,12 @@ def main():
     flush_buf = torch.empty(L2_FLUSH_BYTES, dtype=torch.uint8, device="cuda")
 
     results = {}
-    modes = ["p2p", "nccl"] if args.mode == "auto" else [args.mode]
+    # N = 1: every message is a self message (one DirectIPC launch in every mode);
+    # N > 1: the three data paths differ -- measure all, report the fastest
+    if args.mode == "auto":
+        modes = ["nccl", "p2p"] if not dist_on else ["p2p_direct", "p2p", "nccl"]
+    else:
+        modes = [args.mode]
     for mode in modes:
         try:
             # plan metadata: host all-gather over the process group; NCCL comm
@@ -429,7 +434,7 @@ def main():
     alg_bytes = wl.alg_bytes
     step_s = best["mean_ms"] / 1e3
     achieved = alg_bytes / step_s / 1e9
-    kname = "ddt_exchange_*" if best_mode == "p2p" else "ddt_fused_*"
+    kname = "ddt_exchange_*" if (best_mode != "nccl" and dist_on) else "ddt_fused_*"
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
             "frac": round(achieved / hbm, 4), "traffic": traffic_from_profiles(kname, "configs[1]"),
             "kernel": kname, "alg_bytes_per_launch": alg_bytes,
