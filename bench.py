@@ -133,10 +133,11 @@ class HaloWorkload:
         self.S = sum(T(m["send_spec"]).size for m in msgs)                      # packed bytes out per rank
         self.S_remote = sum(T(m["send_spec"]).size for m in msgs if m["peer"] != rank)
         self.S_self = self.S - self.S_remote
-        # minimum HBM bytes per rank per step: a self message is one DirectIPC
+        # algorithmic HBM bytes per rank per step: a self message is one DirectIPC
         # gather->scatter (read S + write S); a remote one is packed (read + write),
-        # lands in the receiver's window and is unpacked there (read + write)
-        self.alg_bytes = 2 * self.S_self + 4 * self.S_remote
+        # lands in the receiver's window and is unpacked there (read + write), or,
+        # pack-free (p2p_direct), gathered and scattered once (read S + write S)
+        self.alg_bytes = 2 * self.S_self + (2 if mode == "p2p_direct" else 4) * self.S_remote
         self.nmsgs = len(msgs)
         self.launches = self.halo.launches_per_exchange
         self.array_bytes = sum(a.numel() * 8 for a in self.arrs)
