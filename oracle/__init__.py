@@ -29,6 +29,8 @@ Spec tuples (the neutral input language both sides parse independently):
     ("indexed", blocklens, displs, old)
     ("hindexed", blocklens, displs_bytes, old)
     ("subarray", sizes, subsizes, starts, "C"|"F", old)
+    ("struct", blocklens, displs_bytes, [old_0, old_1, ...])
+    ("resized", old, lb, extent)
 
 Parity status: every function here is pinned by tests/test_oracle_pins.py
 (numpy slicing / as_strided / concatenation, closed forms, brute-force
@@ -78,6 +80,8 @@ def lib():
                 "orc_indexed": [I64, I64P, I64P, P],
                 "orc_hindexed": [I64, I64P, I64P, P],
                 "orc_subarray": [I, I64P, I64P, I64P, I, P],
+                "orc_struct": [I64, I64P, I64P, ctypes.POINTER(P)],
+                "orc_resized": [P, I64, I64],
             }.items():
                 f = getattr(L, name)
                 f.argtypes = args
@@ -135,6 +139,17 @@ class Type:
             self._keep += [a, b]
             f = L.orc_indexed if kind == "indexed" else L.orc_hindexed
             self.ptr = f(len(bl), a, b, old.ptr)
+        elif kind == "struct":
+            bl, d, olds = list(spec[1]), list(spec[2]), list(spec[3])
+            assert len(bl) == len(d) == len(olds)
+            kids = [self._child(o) for o in olds]
+            a, b = _arr(bl), _arr(d)
+            tp = (ctypes.c_void_p * max(1, len(kids)))(*[k.ptr for k in kids])
+            self._keep += [a, b, tp]
+            self.ptr = L.orc_struct(len(bl), a, b, tp)
+        elif kind == "resized":
+            old = self._child(spec[1])
+            self.ptr = L.orc_resized(old.ptr, int(spec[2]), int(spec[3]))
         elif kind == "subarray":
             sizes, subsizes, starts, order = spec[1], spec[2], spec[3], spec[4]
             old = self._child(spec[5])

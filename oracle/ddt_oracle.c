@@ -24,6 +24,10 @@
  *   indexed(n,B,D,old): for i<n, for j<B[i]: copy of old at (D[i]+j)*ext(old)
  *   hindexed(n,B,D,old):for i<n, for j<B[i]: copy of old at D[i] + j*ext(old)
  *   contiguous(n,old):  for i<n: copy of old at i*ext(old)
+ *   struct(n,B,D,T[]):  for i<n, for j<B[i]: copy of T[i] at D[i] + j*ext(T[i])
+ *                       (byte displacements; no alignment epsilon, DESIGN R2)
+ *   resized(old,lb,ex): the typemap of old with lb / extent set to (lb, ex)
+ *                       (MPI-3.1 §4.1.7); true bounds stay those of the entries
  *   subarray(nd,sizes,subsizes,starts,order,old): C order = dim 0 outermost,
  *     last dim fastest; Fortran = dim nd-1 outermost, dim 0 fastest; element
  *     (i_0..i_{nd-1}) is a copy of old at
@@ -45,7 +49,7 @@
 #include <stdlib.h>
 #include <string.h>
 
-enum { OK_BASIC = 0, OK_CONTIG, OK_VECTOR, OK_HVECTOR, OK_INDEXED, OK_HINDEXED, OK_SUBARRAY };
+enum { OK_BASIC = 0, OK_CONTIG, OK_VECTOR, OK_HVECTOR, OK_INDEXED, OK_HINDEXED, OK_SUBARRAY, OK_STRUCT, OK_RESIZED };
 
 typedef struct orc_type {
     int kind;
@@ -56,6 +60,8 @@ typedef struct orc_type {
     int ndims, order;
     int64_t sizes[16], subsizes[16], starts[16];
     struct orc_type *old;
+    struct orc_type **types;        /* struct: one oldtype per block */
+    int64_t rlb, rextent;           /* resized */
 } orc_type;
 
 /* ---------------------------------------------------------------- builders */
@@ -120,11 +126,25 @@ orc_type *orc_subarray(int ndims, const int64_t *sizes, const int64_t *subsizes,
     return t;
 }
 
+orc_type *orc_struct(int64_t n, const int64_t *bl, const int64_t *displs_bytes, orc_type **types) {
+    orc_type *t = orc_blocks(OK_STRUCT, n, bl, displs_bytes, NULL);
+    t->types = (orc_type **)malloc(sizeof(orc_type *) * (size_t)(n > 0 ? n : 1));
+    for (int64_t i = 0; i < n; i++) t->types[i] = types[i];
+    return t;
+}
+
+orc_type *orc_resized(orc_type *old, int64_t lb, int64_t extent) {
+    orc_type *t = orc_new(OK_RESIZED);
+    t->old = old; t->rlb = lb; t->rextent = extent;
+    return t;
+}
+
 /* The oracle never frees shared oldtypes; tests build small trees. */
 void orc_free(orc_type *t) {
     if (!t) return;
     free(t->blocklens);
     free(t->displs);
+    free(t->types);
     free(t);
 }
 
@@ -174,6 +194,16 @@ static void orc_walk(const orc_type *t, int64_t base, orc_emit_fn emit, void *ct
                 orc_walk(t->old, base + t->displs[i] + j * e, emit, ctx);
         return;
     }
+    case OK_STRUCT:
+        for (int64_t i = 0; i < t->nblocks; i++) {
+            int64_t e = orc_extent(t->types[i]);
+            for (int64_t j = 0; j < t->blocklens[i]; j++)
+                orc_walk(t->types[i], base + t->displs[i] + j * e, emit, ctx);
+        }
+        return;
+    case OK_RESIZED:
+        orc_walk(t->old, base, emit, ctx);
+        return;
     case OK_SUBARRAY: {
         /* Odometer over the subsizes box.  C order: last dim fastest.
          * Fortran order: dim 0 fastest. */
@@ -260,6 +290,29 @@ static int orc_bounds(const orc_type *t, int64_t *lb, int64_t *ub) {
         if (total == 0 || !nonempty_old) { *lb = 0; *ub = 0; return 0; }
         *lb = 0;
         *ub = prod * (oub - olb);
+        return 1;
+    }
+    if (t->kind == OK_RESIZED) {
+        /* explicit bounds; a type without entries still contributes none (R3) */
+        int64_t olb, oub;
+        int nonempty_old = orc_bounds(t->old, &olb, &oub);
+        *lb = t->rlb;
+        *ub = t->rlb + t->rextent;
+        return nonempty_old;
+    }
+    if (t->kind == OK_STRUCT) {
+        orc_bacc b = {0, 0, 0};
+        for (int64_t i = 0; i < t->nblocks; i++) {
+            int64_t olb, oub;
+            if (!orc_bounds(t->types[i], &olb, &oub)) continue;
+            int64_t e = oub - olb;
+            for (int64_t j = 0; j < t->blocklens[i]; j++) {
+                int64_t d = t->displs[i] + j * e;
+                orc_bacc_add(&b, d + olb, d + oub);
+            }
+        }
+        if (!b.any) { *lb = 0; *ub = 0; return 0; }
+        *lb = b.lo; *ub = b.hi;
         return 1;
     }
     int64_t olb, oub;

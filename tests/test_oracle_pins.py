@@ -350,3 +350,64 @@ def test_oracle_exchange_matches_np_pad_wrap(P, faces_only):
             rest = ~gm
             rest[1:-1, 1:-1, 1:-1] = False
             assert np.all(got[rest] == 0xA5A5A5A5A5A5A5A5)
+
+
+# ------------------------------------------------------------ struct / resized (MPI-3.1 §4.1.2, §4.1.7)
+_NP = {"double": "<f8", "float": "<f4", "int32": "<i4", "int64": "<i8", "byte": "u1"}
+
+
+@HSET
+@given(st.data())
+def test_struct_matches_numpy_structured_dtype(data):
+    """A struct of basic blocks is a numpy structured dtype with explicit field
+    offsets: packing `count` instances copies the fields, in field order, of
+    consecutive records of itemsize = extent (numpy implements the same
+    field-by-name copy)."""
+    n = data.draw(st.integers(1, 4))
+    names, formats, offsets, bl, d, olds = [], [], [], [], [], []
+    pos = data.draw(st.integers(0, 8))
+    for i in range(n):
+        base = data.draw(st.sampled_from(["double", "float", "int32", "byte"]))
+        esz = oracle.BASIC_SIZES[base]
+        b = data.draw(st.integers(1, 3))
+        pos = (pos + esz - 1) // esz * esz
+        names.append(f"f{i}")
+        formats.append((_NP[base], (b,)))
+        offsets.append(pos)
+        bl.append(b), d.append(pos), olds.append(("basic", base))
+        pos += b * esz + data.draw(st.integers(0, 12))
+    perm = data.draw(st.permutations(range(n)))          # typemap order != address order
+    spec = ("struct", [bl[i] for i in perm], [d[i] for i in perm], [olds[i] for i in perm])
+    t = oracle.Type(spec)
+    lo = min(d)
+    hi = max(off + bb * oracle.BASIC_SIZES[o[1]] for off, bb, o in zip(d, bl, olds))
+    assert t.extent() == (lo, hi - lo)
+    count = data.draw(st.integers(1, 3))
+    # numpy record layout: the MPI buffer address is the record start minus lb
+    rec = np.dtype({"names": names, "formats": formats, "offsets": [o - lo for o in offsets], "itemsize": hi - lo})
+    src = random_bytes(rec.itemsize * count + 16, 21)
+    arr = np.frombuffer(src[: rec.itemsize * count].tobytes(), dtype=rec)
+    packed_dt = np.dtype([(names[i], formats[i]) for i in perm])
+    expect = np.empty(count, dtype=packed_dt)
+    for i in perm:
+        expect[names[i]] = arr[names[i]]
+    got = oracle.pack(t, np.concatenate([src, np.zeros(64, np.uint8)]), count, src_offset=-lo)
+    np.testing.assert_array_equal(got, expect.view(np.uint8))
+
+
+@HSET
+@given(c=st.integers(1, 4), b=st.integers(1, 3), stride=st.integers(3, 6), lb=st.integers(-16, 16),
+       extra=st.integers(0, 64), count=st.integers(1, 4))
+def test_resized_steps_instances_by_the_new_extent(c, b, stride, lb, extra, count):
+    inner = ("vector", c, b, stride, ("basic", "double"))
+    E = ((c - 1) * stride + b) * 8 + extra
+    t = oracle.Type(("resized", inner, lb, E))
+    assert t.extent() == (lb, E)
+    assert t.true_extent() == oracle.Type(inner).true_extent()
+    src = random_bytes(E * count + 512, 8)
+    got = oracle.pack(t, src, count)
+    view = np.lib.stride_tricks.as_strided(src, shape=(count, c, b, 8), strides=(E, stride * 8, 8, 1))
+    np.testing.assert_array_equal(got, view.reshape(-1))
+    # a resized oldtype sets the copy spacing of its parent
+    v = oracle.Type(("contiguous", 3, ("resized", ("basic", "double"), 0, 24)))
+    assert v.typemap()[0].tolist() == [0, 24, 48]
