@@ -104,6 +104,21 @@ ddt_status_t ddt_create_indexed(int64_t count, const int64_t* blocklens, const i
 /* hindexed: as indexed with displacements in BYTES (need not be multiples of the element size, R20) */
 ddt_status_t ddt_create_hindexed(int64_t count, const int64_t* blocklens, const int64_t* displs_bytes,
                                  ddt_type_t old, ddt_type_t* out);
+/* indexed_block / hindexed_block: every block has `blocklen` elements (MPI-3.1 §4.1.2) */
+ddt_status_t ddt_create_indexed_block(int64_t count, int64_t blocklen, const int64_t* displs, ddt_type_t old,
+                                      ddt_type_t* out);
+ddt_status_t ddt_create_hindexed_block(int64_t count, int64_t blocklen, const int64_t* displs_bytes, ddt_type_t old,
+                                       ddt_type_t* out);
+/* struct: block i = blocklens[i] copies of types[i] at byte displacement
+ * displs_bytes[i] (+ j * extent(types[i])).  Heterogeneous blocks (e.g. the
+ * paper's struct-on-indexed specfem3D_cm layout).  No alignment epsilon
+ * is added to the upper bound (reading R2): use ddt_create_resized to pad. */
+ddt_status_t ddt_create_struct(int64_t count, const int64_t* blocklens, const int64_t* displs_bytes,
+                               const ddt_type_t* types, ddt_type_t* out);
+/* resized (MPI-3.1 §4.1.7): the typemap of `old` with lb / extent replaced;
+ * instances of a count and copies inside parent types step by `extent`.
+ * extent >= 0.  A type without entries still contributes no bounds (R3). */
+ddt_status_t ddt_create_resized(ddt_type_t old, int64_t lb, int64_t extent, ddt_type_t* out);
 /* subarray (MPI-3.1 §4.1.3): 1 <= ndims <= 16, 1 <= subsizes[k] <= sizes[k],
  * 0 <= starts[k] <= sizes[k]-subsizes[k]; result has lb 0 and extent prod(sizes)*ext(old). */
 ddt_status_t ddt_create_subarray(int ndims, const int64_t* sizes, const int64_t* subsizes,

@@ -54,6 +54,10 @@ PROTOTYPES = {
     "ddt_create_hvector": (I32, [I64, I64, I64, P, ctypes.POINTER(P)]),
     "ddt_create_indexed": (I32, [I64, I64P, I64P, P, ctypes.POINTER(P)]),
     "ddt_create_hindexed": (I32, [I64, I64P, I64P, P, ctypes.POINTER(P)]),
+    "ddt_create_indexed_block": (I32, [I64, I64, I64P, P, ctypes.POINTER(P)]),
+    "ddt_create_hindexed_block": (I32, [I64, I64, I64P, P, ctypes.POINTER(P)]),
+    "ddt_create_struct": (I32, [I64, I64P, I64P, ctypes.POINTER(P), ctypes.POINTER(P)]),
+    "ddt_create_resized": (I32, [P, I64, I64, ctypes.POINTER(P)]),
     "ddt_create_subarray": (I32, [ctypes.c_int, I64P, I64P, I64P, ctypes.c_int, P, ctypes.POINTER(P)]),
     "ddt_commit": (I32, [P]),
     "ddt_free": (I32, [ctypes.POINTER(P)]),

@@ -18,7 +18,7 @@ const char* last_error();
 ddt_status_t cuda_fail(const char* what, int cuda_err);
 
 // ---------------------------------------------------------------- types
-enum TypeKind { T_BASIC, T_CONTIG, T_VECTOR, T_HVECTOR, T_INDEXED, T_HINDEXED, T_SUBARRAY };
+enum TypeKind { T_BASIC, T_CONTIG, T_VECTOR, T_HVECTOR, T_INDEXED, T_HINDEXED, T_SUBARRAY, T_STRUCT, T_RESIZED };
 
 // A closed-form strided description of the typemap's contiguous segments:
 // segment (i_0..i_{D-1}) (outermost first, typemap order = row-major over the
@@ -71,6 +71,7 @@ struct ddt_type_s {
     int ndims = 0, order = 0;
     std::vector<int64_t> sizes, subsizes, starts;
     ddt_type_s* old = nullptr;
+    std::vector<ddt_type_s*> types;                // struct: one oldtype per block (retained)
     std::atomic<int64_t> refs{1};
 
     // closed-form properties (computed at construction)

@@ -103,9 +103,12 @@ void type_release(ddt_type_s* t) {
     if (!t || t->predefined) return;
     if (t->refs.fetch_sub(1) == 1) {
         ddt_type_s* old = t->old;
+        std::vector<ddt_type_s*> kids;
+        kids.swap(t->types);
         free_device_layouts(t);
         delete t;
         type_release(old);
+        for (ddt_type_s* k : kids) type_release(k);
     }
 }
 
@@ -247,6 +250,57 @@ static void derive_subarray(ddt_type_s* t) {
     }
 }
 
+// struct: block i = blocklens[i] copies of types[i] at displs[i] + j*ext(types[i])
+// (byte displacements, MPI-3.1 §4.1.2; no alignment epsilon, reading R2).
+static void derive_struct(ddt_type_s* t) {
+    bool any = false;
+    int64_t lb = 0, ub = 0, tlb = 0, tub = 0;
+    t->size = 0;
+    for (size_t i = 0; i < t->blocklens.size(); i++) {
+        const ddt_type_s* o = t->types[i];
+        int64_t B = t->blocklens[i];
+        t->size += B * o->size;
+        if (B <= 0 || !o->nonempty) continue;
+        int64_t E = type_extent(o), d = t->displs[i];
+        int64_t blo = d + o->lb, bhi = d + (B - 1) * E + o->ub;
+        int64_t tlo = d + o->true_lb, thi = d + (B - 1) * E + o->true_ub;
+        if (!any || blo < lb) lb = blo;
+        if (!any || bhi > ub) ub = bhi;
+        if (!any || tlo < tlb) tlb = tlo;
+        if (!any || thi > tub) tub = thi;
+        any = true;
+    }
+    t->nonempty = any;
+    if (!any) {
+        t->lb = t->ub = t->true_lb = t->true_ub = 0;
+        t->has_form = true;
+        t->form = Form();
+        return;
+    }
+    t->lb = lb;
+    t->ub = ub;
+    t->true_lb = tlb;
+    t->true_ub = tub;
+    // one non-empty block of a closed-form oldtype is itself closed-form
+    int nz = -1, cnt = 0;
+    for (size_t i = 0; i < t->blocklens.size(); i++)
+        if (t->blocklens[i] > 0 && t->types[i]->nonempty) {
+            nz = (int)i;
+            cnt++;
+        }
+    t->has_form = false;
+    if (cnt == 1 && t->types[(size_t)nz]->has_form) {
+        const ddt_type_s* o = t->types[(size_t)nz];
+        Form f;
+        f.base = t->displs[(size_t)nz] + o->form.base;
+        f.seg_len = o->form.seg_len;
+        f.dims.push_back({t->blocklens[(size_t)nz], type_extent(o)});
+        f.dims.insert(f.dims.end(), o->form.dims.begin(), o->form.dims.end());
+        t->has_form = normalize(f);
+        t->form = f;
+    }
+}
+
 }  // namespace ddt
 
 using namespace ddt;
@@ -336,6 +390,51 @@ ddt_status_t ddt_create_subarray(int ndims, const int64_t* sizes, const int64_t*
     return DDT_OK;
 }
 
+ddt_status_t ddt_create_indexed_block(int64_t count, int64_t blocklen, const int64_t* displs, ddt_type_t old,
+                                      ddt_type_t* out) {
+    if (count < 0 || blocklen < 0) return DDT_ERR_ARG;
+    std::vector<int64_t> bl((size_t)count, blocklen);
+    return create_indexed(T_INDEXED, count, bl.data(), displs, old, out);
+}
+
+ddt_status_t ddt_create_hindexed_block(int64_t count, int64_t blocklen, const int64_t* displs_bytes, ddt_type_t old,
+                                       ddt_type_t* out) {
+    if (count < 0 || blocklen < 0) return DDT_ERR_ARG;
+    std::vector<int64_t> bl((size_t)count, blocklen);
+    return create_indexed(T_HINDEXED, count, bl.data(), displs_bytes, old, out);
+}
+
+ddt_status_t ddt_create_struct(int64_t count, const int64_t* blocklens, const int64_t* displs_bytes,
+                               const ddt_type_t* types, ddt_type_t* out) {
+    if (!out || count < 0 || (count > 0 && (!blocklens || !displs_bytes || !types))) return DDT_ERR_ARG;
+    for (int64_t i = 0; i < count; i++)
+        if (blocklens[i] < 0 || !types[i]) return DDT_ERR_ARG;
+    auto* t = new ddt_type_s();
+    t->kind = T_STRUCT;
+    t->blocklens.assign(blocklens, blocklens + count);
+    t->displs.assign(displs_bytes, displs_bytes + count);
+    t->types.assign(types, types + count);
+    for (auto* k : t->types) type_retain(k);
+    derive_struct(t);
+    *out = t;
+    return DDT_OK;
+}
+
+ddt_status_t ddt_create_resized(ddt_type_t old, int64_t lb, int64_t extent, ddt_type_t* out) {
+    if (!out || !old || extent < 0) return DDT_ERR_ARG;
+    auto* t = new_derived(T_RESIZED, old);
+    t->size = old->size;
+    t->nonempty = old->nonempty;
+    t->lb = lb;
+    t->ub = lb + extent;
+    t->true_lb = old->true_lb;
+    t->true_ub = old->true_ub;
+    t->has_form = old->has_form;  // entries do not move, only the bounds
+    t->form = old->form;
+    *out = t;
+    return DDT_OK;
+}
+
 ddt_status_t ddt_free(ddt_type_t* t) {
     if (!t) return DDT_ERR_ARG;
     if (*t) type_release(*t);
@@ -396,8 +495,8 @@ static void enumerate(const ddt_type_s* t, int64_t base, F&& emit) {
         emit_form(t->form, base, emit);
         return;
     }
-    const ddt_type_s* o = t->old;
-    int64_t E = type_extent(o);
+    const ddt_type_s* o = t->old;  // null for struct (per-block oldtypes)
+    int64_t E = o ? type_extent(o) : 0;
     auto copy = [&](int64_t d) { enumerate(o, base + d, emit); };
     switch (t->kind) {
     case T_CONTIG:
@@ -426,6 +525,26 @@ static void enumerate(const ddt_type_s* t, int64_t base, F&& emit) {
                 if (normalize(f)) emit_form(f, base, emit);
             } else {
                 for (int64_t j = 0; j < B; j++) copy(d + j * E);
+            }
+        }
+        break;
+    case T_RESIZED:
+        enumerate(o, base, emit);
+        break;
+    case T_STRUCT:
+        for (size_t i = 0; i < t->blocklens.size(); i++) {
+            const ddt_type_s* k = t->types[i];
+            int64_t B = t->blocklens[i], Ek = type_extent(k);
+            if (B <= 0 || !k->nonempty) continue;
+            if (k->has_form) {
+                Form f;
+                f.base = t->displs[i] + k->form.base;
+                f.seg_len = k->form.seg_len;
+                f.dims.push_back({B, Ek});
+                f.dims.insert(f.dims.end(), k->form.dims.begin(), k->form.dims.end());
+                if (normalize(f)) emit_form(f, base, emit);
+            } else {
+                for (int64_t j = 0; j < B; j++) enumerate(k, base + t->displs[i] + j * Ek, emit);
             }
         }
         break;

@@ -64,6 +64,30 @@ class Type:
         return Type.indexed(blocklens, displs_bytes, old, hindexed=True)
 
     @staticmethod
+    def indexed_block(blocklen: int, displs, old: "Type", hindexed: bool = False) -> "Type":
+        d, dp = _i64arr(displs)
+        out = P()
+        f = lib().ddt_create_hindexed_block if hindexed else lib().ddt_create_indexed_block
+        check(f(int(d.size), int(blocklen), dp, old._h, ctypes.byref(out)), "ddt_create_(h)indexed_block")
+        return Type(out.value)
+
+    @staticmethod
+    def struct(blocklens, displs_bytes, types) -> "Type":
+        b, bp = _i64arr(blocklens)
+        d, dp = _i64arr(displs_bytes)
+        assert b.size == d.size == len(types)
+        arr = (ctypes.c_void_p * max(1, len(types)))(*[t._h.value for t in types])
+        out = P()
+        check(lib().ddt_create_struct(int(b.size), bp, dp, arr, ctypes.byref(out)), "ddt_create_struct")
+        return Type(out.value)
+
+    @staticmethod
+    def resized(old: "Type", lb: int, extent: int) -> "Type":
+        out = P()
+        check(lib().ddt_create_resized(old._h, int(lb), int(extent), ctypes.byref(out)), "ddt_create_resized")
+        return Type(out.value)
+
+    @staticmethod
     def subarray(sizes, subsizes, starts, order: str, old: "Type") -> "Type":
         s, sp = _i64arr(sizes)
         ss, ssp = _i64arr(subsizes)
@@ -100,6 +124,10 @@ class Type:
             return Type.hindexed(spec[1], spec[2], Type._build(spec[3]))
         if k == "subarray":
             return Type.subarray(spec[1], spec[2], spec[3], spec[4], Type._build(spec[5]))
+        if k == "struct":
+            return Type.struct(spec[1], spec[2], [Type._build(o) for o in spec[3]])
+        if k == "resized":
+            return Type.resized(Type._build(spec[1]), spec[2], spec[3])
         raise ValueError(f"unknown spec kind {k!r}")
 
     # ---------------------------------------------------------- lifecycle

@@ -80,7 +80,11 @@ def spec_strategy(depth=2):
                 lambda subs: st.tuples(st.just("subarray"), st.just(list(sizes)), st.just(list(subs)),
                                        st.tuples(*[st.integers(0, s - b) for s, b in zip(sizes, subs)]).map(list),
                                        st.sampled_from(["C", "F"]), children))))
-        return st.one_of(vec, hvec, cont, idx, hidx, sub)
+        strc = st.integers(1, 3).flatmap(lambda n: st.tuples(
+            st.just("struct"), st.lists(st.integers(0, 3), min_size=n, max_size=n),
+            st.lists(st.integers(-40, 80), min_size=n, max_size=n), st.lists(children, min_size=n, max_size=n)))
+        rsz = st.tuples(st.just("resized"), children, st.integers(-24, 24), st.integers(0, 96))
+        return st.one_of(vec, hvec, cont, idx, hidx, sub, strc, rsz)
 
     return st.recursive(base, extend, max_leaves=3)
 
