@@ -96,6 +96,7 @@ void type_release(ddt_type_s* t);
 // Upload list metadata to `device` if needed (caller has set the device).
 ddt_status_t type_device_layout(ddt_type_s* t, int device, DeviceLayout** out);
 inline int64_t type_extent(const ddt_type_s* t) { return t->ub - t->lb; }
+bool instances_overlap(ddt_type_s* t, int64_t count);  // R5 for unpack / direct destinations
 
 // ------------------------------------------------------------ kernels
 // One request -> (source, destination) descriptor pair (desc.cpp).

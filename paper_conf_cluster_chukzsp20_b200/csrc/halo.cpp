@@ -414,7 +414,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         if (!r.type || r.count < 0 || r.peer < 0 || r.peer >= c->nranks) return DDT_ERR_ARG;
         if (!r.type->committed) return DDT_ERR_STATE;
         if (r.count * r.type->size > 0 && !r.buf) return DDT_ERR_ARG;
-        if (r.count * r.type->size > 0 && r.type->layout.overlaps) return DDT_ERR_OVERLAP;
+        if (r.count * r.type->size > 0 && instances_overlap(r.type, r.count)) return DDT_ERR_OVERLAP;
         if (!seen_r.emplace(std::make_pair(r.peer, r.tag), i).second) return DDT_ERR_ARG;
     }
     if (p2p) {  // symmetric pattern required by the parity double buffering / ready handshake

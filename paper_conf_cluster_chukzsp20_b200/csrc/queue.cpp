@@ -163,7 +163,7 @@ int64_t enqueue(ddt_queue_s* q, int op, ddt_type_s* t, const void* src, int64_t 
     if (!t->committed) return DDT_ERR_STATE;
     int64_t bytes = count * t->size;
     if (bytes > 0 && (!src || !dst)) return DDT_ERR_ARG;
-    if (op == OP_UNPACK && bytes > 0 && t->layout.overlaps) return DDT_ERR_OVERLAP;
+    if (op == OP_UNPACK && bytes > 0 && instances_overlap(t, count)) return DDT_ERR_OVERLAP;
     int64_t c = claim(q);
     if (c < 0) return c;
     ReqDesc sd, dd;
@@ -316,7 +316,7 @@ int64_t ddt_direct_enqueue(ddt_queue_t q, ddt_type_t src_type, const void* src, 
     int64_t bytes = src_count * src_type->size;
     if (bytes != dst_count * dst_type->size) return DDT_ERR_SIZE_MISMATCH;
     if (bytes > 0 && (!src || !dst)) return DDT_ERR_ARG;
-    if (bytes > 0 && dst_type->layout.overlaps) return DDT_ERR_OVERLAP;
+    if (bytes > 0 && instances_overlap(dst_type, dst_count)) return DDT_ERR_OVERLAP;
     int64_t c = claim(q);
     if (c < 0) return c;
     ReqDesc d, a;

@@ -700,6 +700,26 @@ static ddt_status_t flatten(ddt_type_s* t) {
     return DDT_OK;
 }
 
+// Do `count` instances (instance k at k*extent) write any byte twice?  Within
+// one instance: the commit-time flag.  Across instances: impossible unless the
+// entries span more than the extent (only resized types can), then checked
+// exactly on the enumerated segments (bounded), else conservatively "yes".
+bool instances_overlap(ddt_type_s* t, int64_t count) {
+    if (t->layout.overlaps) return true;
+    if (count <= 1 || !t->nonempty) return false;
+    const int64_t ext = type_extent(t);
+    if (ext >= t->true_ub - t->true_lb) return false;
+    if (ext == 0) return true;  // every instance lands on the same bytes
+    std::vector<Seg> one;
+    enumerate(t, 0, [&](int64_t o, int64_t l) { one.push_back({o, l}); });
+    if ((int64_t)one.size() * count > ((int64_t)1 << 24)) return true;
+    std::vector<Seg> all;
+    all.reserve(one.size() * (size_t)count);
+    for (int64_t k = 0; k < count; k++)
+        for (const Seg& x : one) all.push_back({x.off + k * ext, x.len});
+    return segs_overlap(all);
+}
+
 ddt_status_t type_device_layout(ddt_type_s* t, int device, DeviceLayout** out) {
     // strided layouts carry everything in the descriptor: nothing to upload
     static DeviceLayout none;
