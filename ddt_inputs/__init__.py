@@ -56,6 +56,18 @@ def config3_spec(nblocks: int = 100_000, npoints: int = 1 << 20, s: int | None =
     return spec, 12 * npoints
 
 
+def config3_cm_spec(nblocks: int = 100_000, npoints: int = 1 << 20, s: int | None = None):
+    """specfem3D_cm-style struct-on-indexed layout (SURVEY
+    W2): three float field arrays of `npoints` each (x, y, z stored one after the
+    other), one indexed(1-float blocks at idx) type per component, combined by a
+    struct at the arrays' byte offsets.  Returns (spec, src_bytes)."""
+    rng = np.random.default_rng(seed(3, 7) if s is None else s)
+    idx = np.sort(rng.choice(npoints, size=nblocks, replace=False)).astype(np.int64).tolist()
+    comp = ("indexed", [1] * nblocks, idx, ("basic", "float"))
+    spec = ("struct", [1, 1, 1], [0, 4 * npoints, 8 * npoints], [comp, comp, comp])
+    return spec, 12 * npoints
+
+
 # ----------------------------------------------------------------- config 5
 def config5_spec(S: int):
     """BASELINE.json configs[4]: dense vector of doubles, block = min(S, 256 B),

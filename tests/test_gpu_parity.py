@@ -363,3 +363,26 @@ def test_gpu_written_response_status(ddt):
     assert early, "the small request's response status did not arrive before its batch finished"
     assert_bytes_equal(host(s_dst), oracle.pack(oracle.Type(small_spec), hs), "response-flag batch")
     q3.destroy()
+
+
+def test_config3_cm_struct_on_indexed_full(ddt, q):
+    """specfem3D_cm-style struct of three indexed float components (10^5 points
+    each over 2^20): pack and unpack bit-exact, one launch each."""
+    import torch
+    from ddt_inputs import config3_cm_spec
+    spec, nb = config3_cm_spec()
+    t = ddt.Type.from_spec(spec)
+    o = oracle.Type(spec)
+    src = random_bytes(nb, seed(3, 8))
+    d_src = cuda_bytes(src)
+    d_pk = torch.full((t.size,), SENTINEL, dtype=torch.uint8, device="cuda")
+    d_un = torch.full((nb,), SENTINEL, dtype=torch.uint8, device="cuda")
+    q.pack(t, d_src, 1, d_pk)
+    q.flush()
+    q.unpack(t, d_pk, 1, d_un)
+    q.wait()
+    exp = oracle.pack(o, src)
+    assert_bytes_equal(host(d_pk), exp, "config3-cm pack")
+    eu = np.full(nb, SENTINEL, np.uint8)
+    oracle.unpack(o, exp, eu)
+    assert_bytes_equal(host(d_un), eu, "config3-cm unpack")

@@ -411,3 +411,13 @@ def test_resized_steps_instances_by_the_new_extent(c, b, stride, lb, extra, coun
     # a resized oldtype sets the copy spacing of its parent
     v = oracle.Type(("contiguous", 3, ("resized", ("basic", "double"), 0, 24)))
     assert v.typemap()[0].tolist() == [0, 24, 48]
+
+
+def test_config3_cm_struct_on_indexed_matches_fancy_indexing():
+    from ddt_inputs import config3_cm_spec
+    spec, nb = config3_cm_spec(nblocks=2000, npoints=1 << 14)
+    t = oracle.Type(spec)
+    src = random_bytes(nb, 4)
+    f = src.view(np.float32).reshape(3, -1)
+    idx = np.array(spec[3][0][2])
+    np.testing.assert_array_equal(oracle.pack(t, src), np.concatenate([f[0][idx], f[1][idx], f[2][idx]]).view(np.uint8))

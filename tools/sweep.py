@@ -26,7 +26,8 @@ import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 import paper_conf_cluster_chukzsp20_b200 as ddt  # noqa: E402
-from ddt_inputs import config1_spec, config3_spec, config5_spec, CONFIG5_SIZES, CONFIG5_BATCHES  # noqa: E402
+from ddt_inputs import (config1_spec, config3_spec, config3_cm_spec, config5_spec, CONFIG5_SIZES,  # noqa: E402
+                        CONFIG5_BATCHES)
 
 FLUSH = None
 
@@ -86,11 +87,19 @@ def cfg1(reps):
 
 def cfg3(reps):
     res = []
-    for shuffled in (False, True):
-        spec, nb = config3_spec(shuffled=shuffled)
-        t = ddt.Type.from_spec(spec)
-        offs = np.array(spec[2], dtype=np.int64)
-        sectors = len(np.unique(np.concatenate([offs // 32, (offs + 11) // 32])))
+    for variant in ("sorted", "shuffled", "cm_struct"):
+        if variant == "cm_struct":
+            spec, nb = config3_cm_spec()
+            t = ddt.Type.from_spec(spec)
+            idx = np.array(spec[3][0][2], dtype=np.int64)
+            offs = np.concatenate([4 * idx + k * 4 * (1 << 20) for k in range(3)])
+            seglen = 4
+        else:
+            spec, nb = config3_spec(shuffled=(variant == "shuffled"))
+            t = ddt.Type.from_spec(spec)
+            offs = np.array(spec[2], dtype=np.int64)
+            seglen = 12
+        sectors = len(np.unique(np.concatenate([offs // 32, (offs + seglen - 1) // 32])))
         for B in (1, 16, 32):
             src = torch.randint(0, 255, (B, nb), dtype=torch.uint8, device="cuda")
             dst = torch.empty((B, t.size), dtype=torch.uint8, device="cuda")
@@ -101,7 +110,7 @@ def cfg3(reps):
             us = timed(plan.launch, reps)
             alg = 2 * t.size * B
             floor = (sectors * 32 + t.size) * B
-            res.append({"shuffled": shuffled, "B": B, "us": round(us, 2), "alg_gbs": round(alg / us / 1e3, 1),
+            res.append({"variant": variant, "B": B, "us": round(us, 2), "alg_gbs": round(alg / us / 1e3, 1),
                         "sector_floor_gbs_equiv": round(floor / us / 1e3, 1), "payload_bytes": t.size * B,
                         "sector_read_bytes": sectors * 32 * B})
             plan.destroy()
