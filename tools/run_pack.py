@@ -1,19 +1,26 @@
-"""Launch a configs[4] dense-pack plan N times (for ncu captures).
-usage: python tools/run_pack.py S B iters"""
+"""Launch a fused pack plan N times (for ncu captures).
+usage: python tools/run_pack.py S B iters          (configs[4] dense vector of S bytes, batch B)
+       python tools/run_pack.py cfg3 B iters       (configs[2] sparse hindexed, batch B)
+       python tools/run_pack.py cfg3cm B iters     (specfem3D_cm-style struct-on-indexed, batch B)"""
 import os
 import sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
 import paper_conf_cluster_chukzsp20_b200 as ddt  # noqa: E402
-from ddt_inputs import config5_spec  # noqa: E402
+from ddt_inputs import config5_spec, config3_spec, config3_cm_spec  # noqa: E402
 
-S, B, iters = (int(x) for x in sys.argv[1:4])
+what, B, iters = sys.argv[1], int(sys.argv[2]), int(sys.argv[3])
 torch.cuda.set_device(0)
-spec, fp = config5_spec(S)
+if what == "cfg3":
+    spec, fp = config3_spec()
+elif what == "cfg3cm":
+    spec, fp = config3_cm_spec()
+else:
+    spec, fp = config5_spec(int(what))
 t = ddt.Type.from_spec(spec)
 src = torch.empty((B, fp), dtype=torch.uint8, device="cuda")
 src.random_(0, 256)
-dst = torch.empty((B, S), dtype=torch.uint8, device="cuda")
+dst = torch.empty((B, t.size), dtype=torch.uint8, device="cuda")
 q = ddt.Queue()
 for b in range(B):
     q.pack(t, src[b], 1, dst[b])
@@ -21,4 +28,4 @@ plan = ddt.Plan(q)
 for _ in range(iters):
     plan.launch()
 torch.cuda.synchronize()
-print("ok", S, B, iters)
+print("ok", what, B, iters)
