@@ -19,7 +19,8 @@ KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "smsp__inst_executed.sum", "sm__cycles_active.max", "gpc__cycles_elapsed.max"]
 UNIT_SCALE = {"Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "byte": 1.0, "usecond": 1.0, "nsecond": 1e-3, "msecond": 1e3}
 summary, traffic = {}, {}
-for name, wl in [("full_cfg2", "configs[1]"), ("full_cfg4", "configs[3]"), ("full_cfg5", "configs[4]")]:
+for name, wl in [("full_cfg2", "configs[1]"), ("full_cfg3", "configs[2]"), ("full_cfg3cm", "configs[2]-cm"),
+                 ("full_cfg4", "configs[3]"), ("full_cfg5", "configs[4]")]:
     rep = os.path.join(src, name + ".ncu-rep")
     if not os.path.exists(rep):
         continue
