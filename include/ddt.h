@@ -280,6 +280,11 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* comm, int32_t nsen
  * launch.  `use_graph` != 0 replays a CUDA graph captured on first use.      */
 ddt_status_t ddt_exchange(ddt_halo_t h);
 ddt_status_t ddt_halo_set_graph(ddt_halo_t h, int32_t use_graph);
+/* Bound of every device-side flag wait of a P2P plan (default 10 s).  A wait
+ * that exceeds it abandons the message, sets a host-mapped error flag and
+ * the next ddt_exchange returns DDT_ERR_TIMEOUT (sticky) -- never a hang.
+ * Takes effect for launches issued afterwards (a captured graph is rebuilt). */
+ddt_status_t ddt_halo_set_timeout(ddt_halo_t h, int64_t timeout_ns);
 /* Kernel launches issued by the last ddt_exchange (graph replay counts the
  * kernels inside the graph). */
 ddt_status_t ddt_halo_launches_per_exchange(ddt_halo_t h, int32_t* launches);

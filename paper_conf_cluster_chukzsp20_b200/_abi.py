@@ -87,6 +87,7 @@ PROTOTYPES = {
                               ctypes.POINTER(ddt_recv_t), I32, ctypes.POINTER(P)]),
     "ddt_exchange": (I32, [P]),
     "ddt_halo_set_graph": (I32, [P, I32]),
+    "ddt_halo_set_timeout": (I32, [P, I64]),
     "ddt_halo_launches_per_exchange": (I32, [P, I32P]),
     "ddt_halo_destroy": (I32, [P]),
     "ddt_nccl_unique_id": (I32, [P]),

@@ -107,7 +107,9 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
     out.blob.clear();
     const char* force = getenv("DDT_FORCE_TABLE");  // experiments: always use the device-table form
     if (force && force[0] == '1') allow_param = false;
-    if (allow_param && n <= (size_t)kParamSmall) {
+    const char* large = getenv("DDT_FORCE_LARGE_PARAM");  // experiments: skip the small parameter form
+    const bool skip_small = large && large[0] == '1';
+    if (allow_param && n <= (size_t)kParamSmall && !skip_small) {
         out.form = 1;
         to_param<kParamSmall>(b, out);
     } else if (allow_param && n <= (size_t)kParamLarge) {

@@ -759,6 +759,16 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     return DDT_OK;
 }
 
+ddt_status_t ddt_halo_set_timeout(ddt_halo_t h, int64_t timeout_ns) {
+    if (!h || timeout_ns <= 0) return DDT_ERR_ARG;
+    h->timeout_ns = (uint64_t)timeout_ns;
+    if (h->gexec) {  // the old value is baked into the captured launch
+        cudaGraphExecDestroy(h->gexec);
+        h->gexec = nullptr;
+    }
+    return DDT_OK;
+}
+
 ddt_status_t ddt_halo_set_graph(ddt_halo_t h, int32_t use_graph) {
     if (!h) return DDT_ERR_ARG;
     h->use_graph = use_graph != 0;

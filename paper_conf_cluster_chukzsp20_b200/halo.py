@@ -159,6 +159,10 @@ class Halo:
     def exchange(self):
         check(lib().ddt_exchange(self._h), "ddt_exchange")
 
+    def set_timeout(self, seconds: float):
+        """Bound of the device-side flag waits (DDT_ERR_TIMEOUT instead of a hang)."""
+        check(lib().ddt_halo_set_timeout(self._h, int(seconds * 1e9)), "ddt_halo_set_timeout")
+
     @property
     def launches_per_exchange(self) -> int:
         v = ctypes.c_int32()
