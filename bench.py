@@ -295,6 +295,49 @@ def oracle_exchange_sample(local, dirs, nvars, P, budget_s):
     return el / n * 1e6, n
 
 
+def oracle_per_config(budget_s):
+    """The CPU oracle (plain C) on host copies of the other BASELINE configs'
+    layouts -- 1 thread, and a thread pool over a batch on every core of
+    os.sched_getaffinity(0) (ctypes releases the GIL).  Bounded samples;
+    reported beside the GPU numbers of tools/sweep.py, never a target."""
+    import oracle
+    from concurrent.futures import ThreadPoolExecutor
+    from ddt_inputs import config1_spec, config3_spec
+    ncores = len(os.sched_getaffinity(0))
+    res = {"cores_all": ncores,
+           "cpu_model": next((ln.split(":", 1)[1].strip() for ln in open("/proc/cpuinfo")
+                              if ln.startswith("model name")), "?")}
+
+    def rate(fn, nbytes, budget):
+        n, t0 = 0, time.perf_counter()
+        while time.perf_counter() - t0 < budget or n == 0:
+            fn()
+            n += 1
+        dt = (time.perf_counter() - t0) / n
+        return round(dt * 1e6, 2), round(nbytes / dt / 1e9, 4)
+
+    o1 = oracle.Type(config1_spec())
+    src = random_bytes(o1.footprint()[1] + 64, 1)
+    dst = np.zeros_like(src)
+    res["configs[0]_us_per_pack_unpack_1core"] = rate(lambda: oracle.unpack(o1, oracle.pack(o1, src), dst), 1024,
+                                                      budget_s / 3)[0]
+    spec, nb = config3_spec()
+    o3 = oracle.Type(spec)
+    srcs = [random_bytes(nb, 50 + i) for i in range(ncores)]
+    us, gbs = rate(lambda: oracle.pack(o3, srcs[0]), 2 * o3.size, budget_s / 3)
+    res["configs[2]_pack_1core"] = {"us": us, "alg_gbs": gbs}
+    with ThreadPoolExecutor(ncores) as ex:
+        us, gbs = rate(lambda: list(ex.map(lambda a: oracle.pack(o3, a), srcs)), 2 * o3.size * ncores, budget_s / 3)
+    res["configs[2]_pack_allcores"] = {"batch": ncores, "us": us, "alg_gbs": gbs}
+    spec, fp = config5_spec(1 << 20)
+    o5 = oracle.Type(spec)
+    srcs = [random_bytes(fp, 80 + i) for i in range(ncores)]
+    with ThreadPoolExecutor(ncores) as ex:
+        us, gbs = rate(lambda: list(ex.map(lambda a: oracle.pack(o5, a), srcs)), (2 << 20) * ncores, budget_s / 3)
+    res["configs[4]_S1MiB_pack_allcores"] = {"batch": ncores, "us": us, "alg_gbs": gbs}
+    return res
+
+
 def traffic_from_profiles(kernel: str, workload: str):
     """DRAM bytes read + written per launch of the step's kernel, from the
     committed ncu --set full capture (tools/capture_profiles.sh), or None."""
@@ -473,7 +516,8 @@ def main():
         us, n = oracle_exchange_sample(local, FACE_DIRS, 1, 1, args.cpu_budget)
         cpu = {"value": round(us, 2), "unit": "us/iter", "cores": 1, "kind": "oracle",
                "sample": f"{n} iterations of the configs[1] face exchange (pack + unpack of 6 faces, P=1) "
-                         f"over ~{args.cpu_budget:.0f} s, plain C oracle, 1 thread"}
+                         f"over ~{args.cpu_budget:.0f} s, plain C oracle, 1 thread",
+               "other_configs": oracle_per_config(max(3.0, args.cpu_budget / 2))}
 
     if rank == 0:
         line = {

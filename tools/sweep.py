@@ -170,57 +170,11 @@ def cfg5(reps, quick):
     return {"workload": "configs[4]", "cells": cells}
 
 
-# ------------------------------------------------------------------ CPU oracle
-def cpu_oracle(budget_s):
-    """The plain-C oracle on host copies of the same layouts (test
-    infrastructure as a reported baseline): 1 thread, and a thread pool over a
-    batch's requests on every core of os.sched_getaffinity(0) (ctypes releases
-    the GIL).  Bounded samples; transfers excluded."""
-    import oracle
-    from concurrent.futures import ThreadPoolExecutor
-    ncores = len(os.sched_getaffinity(0))
-    model = next((ln.split(":", 1)[1].strip() for ln in open("/proc/cpuinfo") if ln.startswith("model name")), "?")
-    res = {"cores": ncores, "cpu_model": model}
-
-    def rate(fn, nbytes_per_call, budget):
-        n, t0 = 0, time.perf_counter()
-        while time.perf_counter() - t0 < budget or n == 0:
-            fn()
-            n += 1
-        dt = (time.perf_counter() - t0) / n
-        return dt * 1e6, nbytes_per_call / dt / 1e9
-
-    o1 = oracle.Type(config1_spec())
-    lo, hi = o1.footprint()
-    src = np.random.default_rng(1).integers(0, 255, hi + 64, dtype=np.uint8)
-    dst = np.zeros_like(src)
-    us, _ = rate(lambda: oracle.unpack(o1, oracle.pack(o1, src), dst), 1024, budget_s / 4)
-    res["config1_us_per_iter_1core"] = round(us, 2)
-    spec, nb = config3_spec()
-    o3 = oracle.Type(spec)
-    srcs = [np.random.default_rng(i).integers(0, 255, nb, dtype=np.uint8) for i in range(ncores)]
-    us, gbs = rate(lambda: oracle.pack(o3, srcs[0]), 2 * o3.size, budget_s / 4)
-    res["config3_pack_1core"] = {"us": round(us, 1), "alg_gbs": round(gbs, 3)}
-    with ThreadPoolExecutor(ncores) as ex:
-        us, gbs = rate(lambda: list(ex.map(lambda a: oracle.pack(o3, a), srcs)), 2 * o3.size * ncores, budget_s / 4)
-    res["config3_pack_allcores"] = {"batch": ncores, "us": round(us, 1), "alg_gbs": round(gbs, 3)}
-    spec, fp = config5_spec(1 << 20)
-    o5 = oracle.Type(spec)
-    srcs = [np.random.default_rng(i).integers(0, 255, fp, dtype=np.uint8) for i in range(ncores)]
-    us, gbs = rate(lambda: oracle.pack(o5, srcs[0]), 2 << 20, budget_s / 4)
-    res["config5_S1MiB_pack_1core"] = {"us": round(us, 1), "alg_gbs": round(gbs, 3)}
-    with ThreadPoolExecutor(ncores) as ex:
-        us, gbs = rate(lambda: list(ex.map(lambda a: oracle.pack(o5, a), srcs)), (2 << 20) * ncores, budget_s / 4)
-    res["config5_S1MiB_pack_allcores"] = {"batch": ncores, "us": round(us, 1), "alg_gbs": round(gbs, 3)}
-    return res
-
-
 def main():
     global FLUSH
     ap = argparse.ArgumentParser()
     ap.add_argument("--reps", type=int, default=30)
     ap.add_argument("--quick", action="store_true")
-    ap.add_argument("--cpu-budget", type=float, default=20.0)
     args = ap.parse_args()
     torch.cuda.set_device(0)
     FLUSH = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
@@ -229,7 +183,6 @@ def main():
     out["config1"] = cfg1(args.reps)
     out["config3"] = cfg3(args.reps)
     out["config5"] = cfg5(args.reps, args.quick)
-    out["cpu_oracle"] = cpu_oracle(args.cpu_budget)
     out["wall_s"] = round(time.time() - t0, 1)
     print(json.dumps(out))
 
