@@ -15,8 +15,8 @@ L2 is flushed (a 256 MiB write) between timed steps and the flush is outside
 each step's CUDA-event pair.  value = mean per-step device time, max over ranks.
 
 Extra measurements on the same JSON line (rank 0):
-  pack_roofline  -- config 5 dense vector pack (S >= 1 MiB, B*S = 256 MiB and
-                    1 GiB cells): algorithmic bytes (read S + write S) / kernel
+  pack_roofline  -- config 5 dense vector pack (S >= 1 MiB, B*S = 1 GiB cells):
+                    algorithmic bytes (read S + write S) / kernel
                     time vs the measured HBM copy peak ("pack GB/s vs HBM peak")
   comb26         -- configs[3] COMB-style 26-neighbour exchange, 512^3 global
                     grid split over N ranks, 4 variables (104+104 messages)
@@ -222,7 +222,7 @@ def pack_roofline(ddt, torch, hbm_peak, reps=20):
     batches of B requests of S bytes; kernel time from CUDA events around a
     persistent plan launch (table already resident)."""
     cells = []
-    for S, B in [(1 << 20, 256), (4 << 20, 64), (64 << 20, 16)]:
+    for S, B in [(1 << 20, 1024), (4 << 20, 256), (64 << 20, 16)]:  # 1 GiB of packed bytes per launch
         spec, fp = config5_spec(S)
         t = ddt.Type.from_spec(spec)
         src = torch.empty((B, fp), dtype=torch.uint8, device="cuda")

@@ -28,6 +28,12 @@ static uint32_t fill_prefix(uint32_t* prefix, const std::vector<ReqDesc>& d, int
 
 static size_t pad16(size_t v) { return (v + 15) & ~(size_t)15; }
 
+// Item order (experiments: DDT_ITEM_ORDER=blocked); cyclic is the default.
+static uint32_t item_order_blocked() {
+    const char* e = getenv("DDT_ITEM_ORDER");
+    return (e && e[0] == 'b') ? 1u : 0u;
+}
+
 size_t device_table_bytes(const HostBatch& b) {
     size_t n = b.descs.size();
     size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
@@ -55,6 +61,7 @@ uint32_t write_device_table(void* dst, const HostBatch& b, int ub) {
     uint32_t items = fill_prefix(prefix, b.descs, ub);
     size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
     h->ub = (uint32_t)ub;
+    h->blocked = item_order_blocked();
     h->nreq = (uint32_t)n;
     h->total_items = items;
     h->desc_offset = (uint32_t)off;
@@ -77,6 +84,7 @@ static void to_param(const HostBatch& b, Launchable& out) {
     auto* p = reinterpret_cast<ParamBatch<CAP>*>(out.blob.data());
     p->h.nreq = (uint32_t)b.descs.size();
     p->h.ub = (uint32_t)out.ub;
+    p->h.blocked = item_order_blocked();
     p->h.total_items = fill_prefix(p->prefix, b.descs, out.ub);
     std::copy(b.descs.begin(), b.descs.end(), p->descs);
     std::copy(b.aux.begin(), b.aux.end(), p->aux);

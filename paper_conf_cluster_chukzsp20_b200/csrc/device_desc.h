@@ -96,7 +96,7 @@ struct alignas(16) BatchHeader {
     uint32_t xinfo_offset;  // 0 = no exchange info
     uint32_t naux;
     uint32_t ub;            // vectors per thread per item (1, 2 or 4)
-    uint32_t pad;
+    uint32_t blocked;       // item order: 0 = cyclic over CTAs, 1 = contiguous block per CTA
 };
 
 // A small batch carried in the kernel parameters.

@@ -177,7 +177,7 @@ __device__ __forceinline__ uint32_t find_request(const uint32_t* prefix, uint32_
 }
 
 struct TableView {
-    uint32_t nreq, total, ub;
+    uint32_t nreq, total, ub, blocked;
     const uint32_t* prefix;
     const ReqDesc* descs;
     const ReqDesc* aux;
@@ -190,6 +190,7 @@ __device__ __forceinline__ TableView view_of(const uint8_t* t) {
     v.nreq = h->nreq;
     v.total = h->total_items;
     v.ub = h->ub;
+    v.blocked = h->blocked;
     v.prefix = reinterpret_cast<const uint32_t*>(t + sizeof(BatchHeader));
     v.descs = reinterpret_cast<const ReqDesc*>(t + h->desc_offset);
     v.aux = reinterpret_cast<const ReqDesc*>(t + h->aux_offset);
@@ -203,6 +204,7 @@ __device__ __forceinline__ TableView view_of(const ParamBatch<CAP>& p) {
     v.nreq = p.h.nreq;
     v.total = p.h.total_items;
     v.ub = p.h.ub;
+    v.blocked = p.h.blocked;
     v.prefix = p.prefix;
     v.descs = p.descs;
     v.aux = p.aux;
@@ -255,12 +257,18 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
     constexpr int kWords = (int)(sizeof(ReqDesc) / 16);
     constexpr int kXWords = (int)(sizeof(XInfo) / 16);
     uint32_t cur = 0xffffffffu, cur_first = 0;
-    // blocked assignment: CTA b owns items [b*per, (b+1)*per) -- consecutive
-    // items usually share a request, so descriptors are (re)loaded rarely
-    const uint32_t per = (tv.total + gridDim.x - 1) / gridDim.x;
-    const uint32_t first = blockIdx.x * per;
-    const uint32_t last = min(tv.total, first + per);
-    for (uint32_t item = first; item < last; item++) {
+    // cyclic (default): CTA b takes items b, b + grid, ... -- at any moment the
+    // grid streams one contiguous window of each request (DRAM page locality);
+    // blocked: CTA b owns [b*per, (b+1)*per) -- fewer descriptor reloads.
+    // Both visit each CTA's items in increasing order (exchange deadlock freedom).
+    uint32_t first = blockIdx.x, last = tv.total, step = gridDim.x;
+    if (tv.blocked) {
+        const uint32_t per = (tv.total + gridDim.x - 1) / gridDim.x;
+        first = blockIdx.x * per;
+        last = min(tv.total, first + per);
+        step = 1;
+    }
+    for (uint32_t item = first; item < last; item += step) {
         const uint32_t r = find_request(tv.prefix, tv.nreq, item);
         if (r != cur) {
             __syncthreads();  // every warp is done with the previous descriptor
