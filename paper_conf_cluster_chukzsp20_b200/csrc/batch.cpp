@@ -108,10 +108,10 @@ static int batch_variant(const HostBatch& b) {
     return 1 + lw;
 }
 
-void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count) {
+void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count, int force_ub) {
     size_t n = std::max(b.descs.size(), b.aux.size());
     out.variant = batch_variant(b);
-    out.ub = choose_ub(b, sm_count);
+    out.ub = force_ub > 0 ? force_ub : choose_ub(b, sm_count);
     out.blob.clear();
     const char* force = getenv("DDT_FORCE_TABLE");  // experiments: always use the device-table form
     if (force && force[0] == '1') allow_param = false;

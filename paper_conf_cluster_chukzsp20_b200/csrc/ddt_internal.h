@@ -107,6 +107,8 @@ ddt_status_t build_direct(ddt_type_s* ts, const DeviceLayout* dls, const void* s
                           const DeviceLayout* dld, void* dst, int64_t dcount, ReqDesc* s, ReqDesc* d);
 ddt_status_t build_typed(ddt_type_s* t, const DeviceLayout* dl, const void* p, int64_t count, ReqDesc* d);
 ddt_status_t rescale_desc(ReqDesc* d, int lw);
+// Largest legal log2 vector width of one typed side (type layout over pointer p).
+int side_lw(ddt_type_s* t, const void* p, int64_t count);
 // Base address of the device allocation containing p (CUDA driver, for IPC).
 ddt_status_t alloc_base(const void* p, void** base);
 // Items of a descriptor at ub vectors per thread per item.
@@ -145,7 +147,8 @@ uint32_t write_device_table(void* dst, const HostBatch& b, int ub);
 // >= 2 items per SM, so latency-bound batches use every SM.
 int choose_ub(const HostBatch& b, int sm_count);
 // Param form if it fits (and allowed), else form 3 with `dev` left to the caller.
-void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count = 148);
+// force_ub > 0 fixes the item size (exchange plans: sender and receiver chunk alike).
+void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count = 148, int force_ub = 0);
 int launch_fused(const Launchable& l, void* stream, int grid_cap);
 int launch_exchange(const Launchable& l, void* ctrl, int* err_flag_dev, uint64_t timeout_ns, void* stream,
                     int grid_cap);

@@ -43,7 +43,7 @@ static int log2i(int w) {
 }
 
 // Largest legal log2 vector width of one side (type layout over pointer p).
-static int side_lw(ddt_type_s* t, const void* p, int64_t count) {
+int side_lw(ddt_type_s* t, const void* p, int64_t count) {
     int w = std::min(t->layout.align, lowbit16((uint64_t)(uintptr_t)p));
     if (count > 1) w = std::min(w, lowbit16(uabs64(type_extent(t))));
     return log2i(w);

@@ -84,7 +84,14 @@ struct alignas(16) XInfo {
     uint32_t counter;       // multi-item messages: index of the completion counter
     uint32_t nitems;        // items of the message (signal when all are done)
     int64_t parity_stride;  // window half size: the window side moves by (epoch & 1) * stride
+    uint32_t per_item;      // 1: item k signals / waits on flag k (sender and receiver chunk alike)
+    uint32_t fanout;        // per-message signal: number of consecutive flags to release (>= 1)
+    uint64_t pad;
 };
+// Exchange plans chunk every message in items of kThreads * kXchgUb vectors on
+// both sides, so a receiver's unpack item k depends only on the sender's pack
+// item k (per-chunk flags: unpack of a message overlaps its packing).
+constexpr int kXchgUb = 2;
 
 // Header of a device batch table:
 //   BatchHeader | uint32 prefix[nreq + 1] (16 B padded) | ReqDesc src[nreq] | ReqDesc dst[naux] | XInfo[nreq]?

@@ -294,7 +294,8 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
         if constexpr (XCHG) {
             if (sx.wait) {  // acquire: the peer's data / ready signal has arrived
                 if (threadIdx.x == 0) {
-                    const uint64_t* flag = reinterpret_cast<const uint64_t*>(sx.wait);
+                    const uint64_t* flag = reinterpret_cast<const uint64_t*>(sx.wait) +
+                                           (sx.per_item ? (item - cur_first) : 0u);
                     int ok = 1;
                     if (ld_acquire_sys(flag) < epoch) {
                         const uint64_t t0 = globaltimer();
@@ -330,17 +331,20 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
             }
         }
         if constexpr (XCHG) {
-            if (sx.signal) {  // release once every item of the message has moved
-                __syncthreads();  // the CTA's (peer) stores precede thread 0's release
+            if (sx.signal) {  // release: this chunk (per_item) or the whole message has moved
+                __syncthreads();  // the CTA's (peer) stores precede thread 0's release (cumulativity)
                 if (threadIdx.x == 0) {
-                    if (sx.nitems <= 1) {
-                        st_release_sys(reinterpret_cast<uint64_t*>(sx.signal), epoch);
+                    uint64_t* flag = reinterpret_cast<uint64_t*>(sx.signal);
+                    if (sx.per_item) {
+                        st_release_sys(flag + (item - cur_first), epoch);
+                    } else if (sx.nitems <= 1) {
+                        for (uint32_t k = 0; k < sx.fanout; k++) st_release_sys(flag + k, epoch);
                     } else {
                         __threadfence_system();
                         unsigned long long old = atomicAdd_system(&ctrl->counters[sx.counter], 1ull);
                         if (old + 1ull == epoch * (unsigned long long)sx.nitems) {
                             __threadfence_system();
-                            st_release_sys(reinterpret_cast<uint64_t*>(sx.signal), epoch);
+                            for (uint32_t k = 0; k < sx.fanout; k++) st_release_sys(flag + k, epoch);
                         }
                     }
                 }

@@ -23,6 +23,7 @@
 //   and tells each sender where its messages land; iterations can be replayed
 //   from a CUDA graph captured on first use.
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <map>
 #include <tuple>
@@ -45,7 +46,9 @@ int64_t round_up(int64_t v, int64_t a) { return (v + a - 1) / a * a; }
 struct RecvLayout {
     std::vector<int> order;          // recv indices sorted by (peer, tag)
     std::vector<int64_t> data_off;   // per recv index: offset inside one parity half
-    std::vector<int> flag_idx;       // per recv index
+    std::vector<int> flag_idx;       // per recv index: first of its per-chunk flag slots
+    std::vector<int> lw;             // per recv index: vector width of the unpack side
+    std::vector<int> nflags;         // per recv index: chunks (items at kXchgUb) of the message
     int64_t ready_off = 0;           // byte offset of the per-sender "ready" slots (pack-free mode)
     int64_t flags_bytes = 0, parity_stride = 0, window_bytes = 0;
 };
@@ -59,26 +62,33 @@ RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs) {
     });
     L.data_off.assign((size_t)nrecv, 0);
     L.flag_idx.assign((size_t)nrecv, 0);
-    int64_t off = 0;
+    L.lw.assign((size_t)nrecv, 0);
+    L.nflags.assign((size_t)nrecv, 1);
+    int64_t off = 0, nflag = 0;
+    const int64_t chunk = (int64_t)kThreads * kXchgUb;  // vectors per exchange item
     for (size_t k = 0; k < L.order.size(); k++) {
         int i = L.order[k];
         int64_t bytes = recvs[i].count * recvs[i].type->size;
         off = round_up(off, kAlign);
         L.data_off[(size_t)i] = off;
-        L.flag_idx[(size_t)i] = (int)k;
+        int lw = recvs[i].type->committed ? std::min(4, side_lw(recvs[i].type, recvs[i].buf, recvs[i].count)) : 0;
+        L.lw[(size_t)i] = lw;
+        L.nflags[(size_t)i] = (int)std::max<int64_t>(1, ((bytes >> lw) + chunk - 1) / chunk);
+        L.flag_idx[(size_t)i] = (int)nflag;
+        nflag += L.nflags[(size_t)i];
         off += bytes;
     }
     int64_t nready = 0;  // one slot per possible sender rank
     for (int i = 0; i < nrecv; i++) nready = std::max<int64_t>(nready, (int64_t)recvs[i].peer + 1);
-    L.ready_off = 8 * (int64_t)nrecv;
-    L.flags_bytes = round_up(std::max<int64_t>(8 * ((int64_t)nrecv + nready), 8), 256);
+    L.ready_off = 8 * nflag;
+    L.flags_bytes = round_up(std::max<int64_t>(8 * (nflag + nready), 8), 256);
     L.parity_stride = round_up(std::max<int64_t>(off, 16), 256);
     L.window_bytes = L.flags_bytes + 2 * L.parity_stride;
     return L;
 }
 
 struct DirEntry {
-    int64_t tag, bytes, data_off, flag_idx;
+    int64_t tag, bytes, data_off, flag_idx, lw, nflags;
     // pack-free mode: where the receive buffer lives and how it is laid out
     int64_t ipc[8];      // cudaIpcMemHandle_t of the buffer's allocation
     int64_t alloc_off;   // buffer address - allocation base
@@ -155,8 +165,8 @@ ddt_status_t upload(const std::vector<uint8_t>& host, void** dev) {
 
 // Small batches ride in the kernel parameters (captured into the graph node);
 // larger ones are uploaded once as a device table.
-ddt_status_t make_table(const HostBatch& b, Launchable& l, int sm_count) {
-    make_launchable(b, true, l, sm_count);
+ddt_status_t make_table(const HostBatch& b, Launchable& l, int sm_count, int force_ub = 0) {
+    make_launchable(b, true, l, sm_count, force_ub);
     if (l.form != 3) return DDT_OK;
     std::vector<uint8_t> host(device_table_bytes(b));
     write_device_table(host.data(), b, l.ub);
@@ -298,7 +308,7 @@ ddt_status_t agree(ddt_halo_s* h, ddt_status_t mine) {
 }
 
 // [n, parity_stride, data_base, ready_base, direct] then n entries of
-// [tag, bytes, data_off, flag_idx] (+ [ipc x8, alloc_off, desc x kDescWords] if direct)
+// [tag, bytes, data_off, flag_idx, lw, nflags] (+ [ipc x8, alloc_off, desc x kDescWords] if direct)
 Directory parse_dir(const std::vector<int64_t>& v) {
     Directory d;
     if (v.size() < 5) return d;
@@ -308,17 +318,19 @@ Directory parse_dir(const std::vector<int64_t>& v) {
     d.ready_base = v[3];
     d.direct = v[4];
     size_t pos = 5;
-    const size_t stride = 4 + (d.direct ? 9 + kDescWords : 0);
+    const size_t stride = 6 + (d.direct ? 9 + kDescWords : 0);
     for (int64_t i = 0; i < n && pos + stride <= v.size(); i++, pos += stride) {
         DirEntry e{};
         e.tag = v[pos];
         e.bytes = v[pos + 1];
         e.data_off = v[pos + 2];
         e.flag_idx = v[pos + 3];
+        e.lw = v[pos + 4];
+        e.nflags = v[pos + 5];
         if (d.direct) {
-            std::memcpy(e.ipc, &v[pos + 4], 64);
-            e.alloc_off = v[pos + 12];
-            std::memcpy(&e.desc, &v[pos + 13], sizeof(ReqDesc));
+            std::memcpy(e.ipc, &v[pos + 6], 64);
+            e.alloc_off = v[pos + 14];
+            std::memcpy(&e.desc, &v[pos + 15], sizeof(ReqDesc));
         }
         d.e.push_back(e);
     }
@@ -466,6 +478,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             v.push_back(recvs[k].count * recvs[k].type->size);
             v.push_back(RL.data_off[(size_t)k]);
             v.push_back(RL.flag_idx[(size_t)k]);
+            v.push_back(RL.lw[(size_t)k]);
+            v.push_back(RL.nflags[(size_t)k]);
             if (!dmsg) continue;
             // pack-free: publish the receive buffer (IPC handle + offset) and its layout
             int64_t words[9 + kDescWords] = {0};
@@ -543,14 +557,14 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     // ---- build the device work tables
     // pack: typed send buffer -> packed slot; unpack: packed slot -> typed recv buffer
     auto add_req = [&](HostBatch& b, ddt_type_s* t, int op, const void* src, const void* dst, int64_t count,
-                       uint32_t* items) -> ddt_status_t {
+                       int* lw) -> ddt_status_t {
         DeviceLayout* dl = nullptr;
         ddt_status_t s2 = type_device_layout(t, h->device, &dl);
         ReqDesc sd, dd;
         if (s2 == DDT_OK) s2 = build_request(op, t, dl, src, dst, count, &sd, &dd);
         if (s2 != DDT_OK) return s2;
         b.add(sd, dd);
-        if (items) *items = desc_items(sd);
+        if (lw) *lw = sd.lw;
         return DDT_OK;
     };
     // Self messages never touch a staging buffer or window: one DirectIPC
@@ -646,6 +660,12 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         HostBatch xb;
         char* mywin = (char*)c->peer_windows[c->rank];
         uint32_t npack = 0;
+        // test hook (never set in production): route self messages through the
+        // window + flag path instead of DirectIPC, so the single-GPU tests and
+        // benchmarks exercise and time the multi-GPU signalling protocol
+        const char* svw = getenv("DDT_SELF_VIA_WINDOW");
+        const bool self_window = !direct && svw && svw[0] == '1';
+        auto remote = [&](int peer) { return peer != c->rank || self_window; };
         ReqDesc none;
         std::memset(&none, 0, sizeof(none));
         none.kind = K_CONTIG;
@@ -660,25 +680,30 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                 XInfo x{};
                 x.signal = (uint64_t)(uintptr_t)((char*)c->peer_windows[p] + dirs[(size_t)p].ready_base + 8 * c->rank);
                 x.nitems = 1;
+                x.fanout = 1;
                 xb.add(none, none);
                 xb.xinfo.push_back(x);
             }
         }
         for (int i = 0; i < nsend && st == DDT_OK && !direct; i++) {
             const auto& s = sends[i];
-            if (s.count * s.type->size == 0 || s.peer == c->rank) continue;
+            if (s.count * s.type->size == 0 || !remote(s.peer)) continue;
             const Directory& d = dirs[(size_t)s.peer];
             char* win = (char*)c->peer_windows[s.peer];
-            st = add_req(xb, s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, nullptr);
+            int lw = 0;
+            st = add_req(xb, s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, &lw);
             XInfo x{};
             x.signal = (uint64_t)(uintptr_t)(win + 8 * match[(size_t)i]->flag_idx);
             x.counter = npack++;
             x.parity_stride = d.parity_stride;
+            // same vector width on both sides => identical chunking: per-chunk flags
+            x.per_item = lw == match[(size_t)i]->lw ? 1u : 0u;
+            x.fanout = (uint32_t)match[(size_t)i]->nflags;  // else: all of the receiver's flags at the end
             xb.xinfo.push_back(x);
         }
         for (int i = 0; i < nsend && st == DDT_OK; i++) {
             const auto& s = sends[i];
-            if (s.count * s.type->size == 0 || s.peer != c->rank) continue;
+            if (s.count * s.type->size == 0 || remote(s.peer)) continue;
             st = add_direct(xb, s, recvs[self_recv(s.tag)], true);
         }
         for (int i = 0; i < nsend && st == DDT_OK && direct; i++) {
@@ -710,29 +735,30 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             x.signal = (uint64_t)(uintptr_t)((char*)c->peer_windows[s.peer] + 8 * e.flag_idx);
             x.wait = (uint64_t)(uintptr_t)(mywin + RL.ready_off + 8 * s.peer);
             x.counter = npack++;
+            x.fanout = 1;
             xb.xinfo.push_back(x);
         }
         for (int i = 0; i < nrecv && st == DDT_OK; i++) {
             const auto& r = recvs[i];
-            if (r.count * r.type->size == 0 || r.peer == c->rank) continue;
+            if (r.count * r.type->size == 0 || !remote(r.peer)) continue;
             XInfo x{};
             x.wait = (uint64_t)(uintptr_t)(mywin + 8 * RL.flag_idx[(size_t)i]);
             if (direct) {  // the data lands by itself; wait for its completion flag
                 xb.add(none, none);
-            } else {
+            } else {  // unpack chunk k as soon as the sender's chunk k has landed
                 st = add_req(xb, r.type, OP_UNPACK, mywin + RL.flags_bytes + RL.data_off[(size_t)i], r.buf, r.count,
                              nullptr);
                 x.parity_stride = RL.parity_stride;
+                x.per_item = 1;
             }
             xb.xinfo.push_back(x);
         }
         for (const auto& x : xb.xinfo) h->x_flags |= x.signal != 0 || x.wait != 0;
         if (st == DDT_OK && !xb.descs.empty()) {
-            // completion-counter targets use the batch's item size
-            const int ub = choose_ub(xb, queue_sm_count(q));
+            // exchange plans chunk every message alike on both sides (kXchgUb)
             for (size_t i = 0; i < xb.descs.size(); i++)
-                if (xb.xinfo[i].signal) xb.xinfo[i].nitems = desc_items(xb.descs[i], ub);
-            st = make_table(xb, h->x_l, queue_sm_count(q));
+                if (xb.xinfo[i].signal) xb.xinfo[i].nitems = desc_items(xb.descs[i], kXchgUb);
+            st = make_table(xb, h->x_l, queue_sm_count(q), kXchgUb);
         }
         size_t ctrl_bytes = sizeof(XCtrl) + sizeof(unsigned long long) * std::max<size_t>(npack, 1);
         if (st == DDT_OK) {
