@@ -285,6 +285,12 @@ ddt_status_t ddt_halo_set_graph(ddt_halo_t h, int32_t use_graph);
  * the next ddt_exchange returns DDT_ERR_TIMEOUT (sticky) -- never a hang.
  * Takes effect for launches issued afterwards (a captured graph is rebuilt). */
 ddt_status_t ddt_halo_set_timeout(ddt_halo_t h, int64_t timeout_ns);
+/* Tracing: record one 48-byte record per work item of the fused
+ * P2P exchange kernel -- {u32 cta, item, request, op; u64 t_start, t_after_wait,
+ * t_after_data, t_after_signal} in %globaltimer ns -- into dev_records (device
+ * memory, `capacity` records; later records are dropped).  capacity 0 turns it
+ * off.  Resets the record counter.  DDT_ERR_STATE for NCCL-mode plans. */
+ddt_status_t ddt_halo_set_trace(ddt_halo_t h, void* dev_records, int64_t capacity);
 /* Kernel launches issued by the last ddt_exchange (graph replay counts the
  * kernels inside the graph). */
 ddt_status_t ddt_halo_launches_per_exchange(ddt_halo_t h, int32_t* launches);

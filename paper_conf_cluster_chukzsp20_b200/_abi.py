@@ -6,7 +6,8 @@ import os
 import threading
 
 HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(HERE, "libddt.so")
+# DDT_LIBDDT: load another build of the library (A/B experiments only)
+LIB_PATH = os.environ.get("DDT_LIBDDT") or os.path.join(HERE, "libddt.so")
 
 DDT_OK = 0
 ERRORS = {
@@ -88,6 +89,7 @@ PROTOTYPES = {
     "ddt_exchange": (I32, [P]),
     "ddt_halo_set_graph": (I32, [P, I32]),
     "ddt_halo_set_timeout": (I32, [P, I64]),
+    "ddt_halo_set_trace": (I32, [P, P, I64]),
     "ddt_halo_launches_per_exchange": (I32, [P, I32P]),
     "ddt_halo_destroy": (I32, [P]),
     "ddt_nccl_unique_id": (I32, [P]),

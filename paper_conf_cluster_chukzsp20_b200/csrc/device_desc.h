@@ -122,9 +122,19 @@ static_assert(sizeof(ParamBatch<kParamLarge>) <= 32000, "kernel parameter limit"
 // Control block of the fused exchange kernel (device memory, zeroed at create).
 struct XCtrl {
     unsigned int done;            // CTAs finished (reset by the last CTA to exit)
-    unsigned int pad;
+    unsigned int trace_n;         // trace records written (tracing on)
     unsigned long long epoch;     // completed exchanges
+    unsigned long long trace;     // device pointer to TraceRec[trace_cap], 0 = tracing off
+    unsigned long long trace_cap;
     unsigned long long counters[1];  // [nsend] monotonic per-message item counters
+};
+
+// One work item of the fused exchange kernel, %globaltimer stamps (ns):
+// t0 item start, t1 after its wait (== t0 if none), t2 after its data moved,
+// t3 after its signal (== t2 if none).
+struct TraceRec {
+    unsigned int cta, item, req, op;
+    unsigned long long t0, t1, t2, t3;
 };
 
 }  // namespace ddt

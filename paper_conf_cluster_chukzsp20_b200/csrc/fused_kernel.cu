@@ -224,6 +224,9 @@ __device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
     asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
+__device__ __forceinline__ void st_relaxed_sys(uint64_t* p, uint64_t v) {
+    asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 __device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
     asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
@@ -291,6 +294,10 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
         }
         const uint32_t v0 = (item - cur_first) * (uint32_t)(kThreads * tv.ub);
         bool run = true;
+        uint64_t tr0 = 0, tr1 = 0, tr2 = 0;
+        if constexpr (XCHG) {
+            if (ctrl->trace && threadIdx.x == 0) tr0 = globaltimer();
+        }
         if constexpr (XCHG) {
             if (sx.wait) {  // acquire: the peer's data / ready signal has arrived
                 if (threadIdx.x == 0) {
@@ -314,6 +321,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
                 __syncthreads();
                 run = s_ok != 0;
             }
+            if (ctrl->trace && threadIdx.x == 0) tr1 = globaltimer();
         }
         if (run) run_desc<LW, SONLY>(sd, sa, v0, XCHG && sd.op == OP_UNPACK, (int)tv.ub);
         if constexpr (!XCHG) {
@@ -331,6 +339,10 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
             }
         }
         if constexpr (XCHG) {
+            if (ctrl->trace) {
+                __syncthreads();
+                if (threadIdx.x == 0) tr2 = globaltimer();
+            }
             if (sx.signal) {  // release: this chunk (per_item) or the whole message has moved
                 __syncthreads();  // the CTA's (peer) stores precede thread 0's release (cumulativity)
                 if (threadIdx.x == 0) {
@@ -338,15 +350,30 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
                     if (sx.per_item) {
                         st_release_sys(flag + (item - cur_first), epoch);
                     } else if (sx.nitems <= 1) {
-                        for (uint32_t k = 0; k < sx.fanout; k++) st_release_sys(flag + k, epoch);
+                        __threadfence_system();
+                        for (uint32_t k = 0; k < sx.fanout; k++) st_relaxed_sys(flag + k, epoch);
                     } else {
                         __threadfence_system();
                         unsigned long long old = atomicAdd_system(&ctrl->counters[sx.counter], 1ull);
                         if (old + 1ull == epoch * (unsigned long long)sx.nitems) {
-                            __threadfence_system();
-                            for (uint32_t k = 0; k < sx.fanout; k++) st_release_sys(flag + k, epoch);
+                            __threadfence_system();  // one release for all of the message's flags
+                            for (uint32_t k = 0; k < sx.fanout; k++) st_relaxed_sys(flag + k, epoch);
                         }
                     }
+                }
+            }
+            if (ctrl->trace && threadIdx.x == 0) {
+                unsigned int slot = atomicAdd(&ctrl->trace_n, 1u);
+                if (slot < ctrl->trace_cap) {
+                    TraceRec* t = reinterpret_cast<TraceRec*>(ctrl->trace) + slot;
+                    t->cta = blockIdx.x;
+                    t->item = item;
+                    t->req = cur;
+                    t->op = sd.op;
+                    t->t0 = tr0;
+                    t->t1 = tr1;
+                    t->t2 = tr2;
+                    t->t3 = globaltimer();
                 }
             }
         }

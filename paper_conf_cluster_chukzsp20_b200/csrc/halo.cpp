@@ -23,6 +23,7 @@
 //   and tells each sender where its messages land; iterations can be replayed
 //   from a CUDA graph captured on first use.
 #include <algorithm>
+#include <cstddef>
 #include <cstdlib>
 #include <cstring>
 #include <map>
@@ -697,7 +698,9 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             x.counter = npack++;
             x.parity_stride = d.parity_stride;
             // same vector width on both sides => identical chunking: per-chunk flags
-            x.per_item = lw == match[(size_t)i]->lw ? 1u : 0u;
+            // (DDT_CHUNK_FLAGS=0: experiments, release every flag at message end)
+            const char* cf = getenv("DDT_CHUNK_FLAGS");
+            x.per_item = (lw == match[(size_t)i]->lw && !(cf && cf[0] == '0')) ? 1u : 0u;
             x.fanout = (uint32_t)match[(size_t)i]->nflags;  // else: all of the receiver's flags at the end
             xb.xinfo.push_back(x);
         }
@@ -793,6 +796,20 @@ ddt_status_t ddt_halo_set_timeout(ddt_halo_t h, int64_t timeout_ns) {
         h->gexec = nullptr;
     }
     return DDT_OK;
+}
+
+ddt_status_t ddt_halo_set_trace(ddt_halo_t h, void* dev_records, int64_t capacity) {
+    if (!h || capacity < 0 || (capacity > 0 && !dev_records)) return DDT_ERR_ARG;
+    if (!h->ctrl) return DDT_ERR_STATE;  // tracing covers the fused exchange kernel (P2P plans)
+    DevGuard g(h->device);
+    unsigned long long v[2] = {(unsigned long long)(uintptr_t)dev_records, (unsigned long long)capacity};
+    unsigned int zero = 0;
+    cudaError_t e = cudaMemcpyAsync((char*)h->ctrl + offsetof(XCtrl, trace), v, sizeof(v), cudaMemcpyHostToDevice,
+                                    h->stream);
+    if (e == cudaSuccess)
+        e = cudaMemcpyAsync((char*)h->ctrl + offsetof(XCtrl, trace_n), &zero, 4, cudaMemcpyHostToDevice, h->stream);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
+    return e == cudaSuccess ? DDT_OK : cuda_fail("halo trace", e);
 }
 
 ddt_status_t ddt_halo_set_graph(ddt_halo_t h, int32_t use_graph) {

@@ -159,6 +159,23 @@ class Halo:
     def exchange(self):
         check(lib().ddt_exchange(self._h), "ddt_exchange")
 
+    def trace(self, capacity: int = 4096):
+        """Start tracing the fused exchange kernel into a device buffer; returns a
+        reader: reader() -> structured numpy array of per-item records."""
+        import numpy as np
+        import torch
+        buf = torch.zeros(capacity * 48, dtype=torch.uint8, device=f"cuda:{self.queue.device}")
+        check(lib().ddt_halo_set_trace(self._h, ctypes.c_void_p(buf.data_ptr()), int(capacity)), "ddt_halo_set_trace")
+        self._trace_buf = buf
+        dt = np.dtype([("cta", "<u4"), ("item", "<u4"), ("req", "<u4"), ("op", "<u4"),
+                       ("t0", "<u8"), ("t1", "<u8"), ("t2", "<u8"), ("t3", "<u8")])
+
+        def read():
+            torch.cuda.synchronize()
+            rec = buf.cpu().numpy().view(dt)
+            return rec[rec["t3"] > 0]
+        return read
+
     def set_timeout(self, seconds: float):
         """Bound of the device-side flag waits (DDT_ERR_TIMEOUT instead of a hang)."""
         check(lib().ddt_halo_set_timeout(self._h, int(seconds * 1e9)), "ddt_halo_set_timeout")

@@ -1,0 +1,39 @@
+"""Trace one fused P2P exchange (configs[1], self messages through the window
+path) and print the per-phase critical path (diagnostic)."""
+import os
+import sys
+os.environ.setdefault("DDT_SELF_VIA_WINDOW", "1")
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+import paper_conf_cluster_chukzsp20_b200 as ddt  # noqa: E402
+from ddt_inputs import halo_messages, FACE_DIRS  # noqa: E402
+
+torch.cuda.set_device(0)
+local = (128, 128, 128)
+a = torch.zeros((130, 130, 130), dtype=torch.int64, device="cuda")
+msgs = halo_messages(0, 1, local, dirs=FACE_DIRS)
+sends = [(m["peer"], m["tag"], ddt.Type.from_spec(m["send_spec"]), a, 1) for m in msgs]
+recvs = [(m["recv_peer"], m["recv_tag"], ddt.Type.from_spec(m["recv_spec"]), a, 1) for m in msgs]
+h = ddt.Halo(ddt.Queue(), ddt.Comm.single(0), sends, recvs, mode="p2p", graph=False)
+flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
+for _ in range(5):
+    h.exchange()
+torch.cuda.synchronize()
+for it in range(3):
+    read = h.trace(8192)
+    flush.fill_(it)
+    torch.cuda.synchronize()
+    h.exchange()
+    r = read()
+    t = r["t0"].min()
+    ph = {k: (r[k] - t) / 1e3 for k in ("t0", "t1", "t2", "t3")}
+    pack = r["op"] == 0
+    unp = r["op"] == 1
+    print(f"iter {it}: records {len(r)}  span {ph['t3'].max():.2f} us")
+    for name, m in (("pack", pack), ("unpack", unp)):
+        if m.any():
+            print(f"  {name:6s} start [{ph['t0'][m].min():.2f}, {ph['t0'][m].max():.2f}]  wait-done max {ph['t1'][m].max():.2f}"
+                  f"  data-done [{ph['t2'][m].min():.2f}, {ph['t2'][m].max():.2f}]  signal-done max {ph['t3'][m].max():.2f}"
+                  f"  | per-item wait {np.median((r['t1']-r['t0'])[m])/1e3:.2f}  data {np.median((r['t2']-r['t1'])[m])/1e3:.2f}"
+                  f"  signal {np.median((r['t3']-r['t2'])[m])/1e3:.2f} us (medians)")
