@@ -276,8 +276,11 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* comm, int32_t nsen
                              int32_t nrecv, const ddt_recv_t* recvs, int32_t mode, ddt_halo_t* out);
 /* One exchange iteration, asynchronous on the queue's stream: every send
  * packed, transferred, every receive unpacked.  NCCL mode: fused
- * pack launch -> grouped send/recv -> fused unpack launch.  P2P mode: a single
- * launch.  `use_graph` != 0 replays a CUDA graph captured on first use.      */
+ * pack launch -> grouped send/recv -> fused unpack launch.  P2P modes: a
+ * single launch.  ddt_halo_set_graph(h, 1) replays a CUDA graph captured on
+ * first use -- except for P2P plans with remote messages, whose per-exchange
+ * epoch travels as a kernel argument (always one direct launch).  All ranks
+ * must issue the same sequence of ddt_exchange calls.                        */
 ddt_status_t ddt_exchange(ddt_halo_t h);
 ddt_status_t ddt_halo_set_graph(ddt_halo_t h, int32_t use_graph);
 /* Bound of every device-side flag wait of a P2P plan (default 10 s).  A wait

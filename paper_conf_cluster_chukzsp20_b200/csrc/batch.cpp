@@ -135,10 +135,9 @@ int launch_fused(const Launchable& l, void* stream, int grid_cap) {
     return launch_fused_form(l.form, l.variant, src, l.total_items, stream, grid_cap);
 }
 
-int launch_exchange(const Launchable& l, void* ctrl, int* err_flag_dev, uint64_t timeout_ns, void* stream,
-                    int grid_cap) {
+int launch_exchange(const Launchable& l, const XArgs& xa, void* stream, int grid_cap) {
     const void* src = l.form == 3 ? l.dev : (const void*)l.blob.data();
-    return launch_exchange_form(l.form, l.variant, src, l.total_items, ctrl, err_flag_dev, timeout_ns, stream, grid_cap);
+    return launch_exchange_form(l.form, l.variant, src, l.total_items, xa, stream, grid_cap);
 }
 
 }  // namespace ddt

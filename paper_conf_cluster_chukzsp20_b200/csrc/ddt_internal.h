@@ -150,11 +150,10 @@ int choose_ub(const HostBatch& b, int sm_count);
 // force_ub > 0 fixes the item size (exchange plans: sender and receiver chunk alike).
 void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count = 148, int force_ub = 0);
 int launch_fused(const Launchable& l, void* stream, int grid_cap);
-int launch_exchange(const Launchable& l, void* ctrl, int* err_flag_dev, uint64_t timeout_ns, void* stream,
-                    int grid_cap);
+int launch_exchange(const Launchable& l, const XArgs& xa, void* stream, int grid_cap);
 int launch_fused_form(int form, int variant, const void* param_or_table, uint32_t total_items, void* stream, int grid_cap);
-int launch_exchange_form(int form, int variant, const void* param_or_table, uint32_t total_items, void* ctrl, int* err_flag_dev,
-                         uint64_t timeout_ns, void* stream, int grid_cap);
+int launch_exchange_form(int form, int variant, const void* param_or_table, uint32_t total_items, const XArgs& xa,
+                         void* stream, int grid_cap);
 int device_sm_count(int device);
 
 // queue accessors (queue.cpp)

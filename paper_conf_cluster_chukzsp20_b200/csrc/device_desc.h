@@ -86,7 +86,8 @@ struct alignas(16) XInfo {
     int64_t parity_stride;  // window half size: the window side moves by (epoch & 1) * stride
     uint32_t per_item;      // 1: item k signals / waits on flag k (sender and receiver chunk alike)
     uint32_t fanout;        // per-message signal: number of consecutive flags to release (>= 1)
-    uint64_t pad;
+    uint32_t gpu_scope;     // 1: the flag's reader runs on this GPU -> gpu-scope release suffices
+    uint32_t pad;
 };
 // Exchange plans chunk every message in items of kThreads * kXchgUb vectors on
 // both sides, so a receiver's unpack item k depends only on the sender's pack
@@ -121,11 +122,8 @@ static_assert(sizeof(ParamBatch<kParamLarge>) <= 32000, "kernel parameter limit"
 
 // Control block of the fused exchange kernel (device memory, zeroed at create).
 struct XCtrl {
-    unsigned int done;            // CTAs finished (reset by the last CTA to exit)
     unsigned int trace_n;         // trace records written (tracing on)
-    unsigned long long epoch;     // completed exchanges
-    unsigned long long trace;     // device pointer to TraceRec[trace_cap], 0 = tracing off
-    unsigned long long trace_cap;
+    unsigned int pad;
     unsigned long long counters[1];  // [nsend] monotonic per-message item counters
 };
 
@@ -135,6 +133,19 @@ struct XCtrl {
 struct TraceRec {
     unsigned int cta, item, req, op;
     unsigned long long t0, t1, t2, t3;
+};
+
+// Per-launch arguments of the fused exchange kernel.  The epoch (1, 2, ...) is
+// counted by the host -- every rank runs the same sequence of exchanges -- so
+// no CTA reads or advances device state before its first item.
+struct TraceRec;
+struct XArgs {
+    XCtrl* ctrl;
+    int* err_flag;               // host-mapped: a wait timed out
+    unsigned long long timeout_ns;
+    unsigned long long epoch;
+    TraceRec* trace;             // 0 = tracing off
+    unsigned long long trace_cap;
 };
 
 }  // namespace ddt

@@ -224,8 +224,16 @@ __device__ __forceinline__ uint64_t ld_acquire_sys(const uint64_t* p) {
     asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
     return v;
 }
+__device__ __forceinline__ uint64_t ld_acquire_gpu(const uint64_t* p) {
+    uint64_t v;
+    asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
 __device__ __forceinline__ void st_relaxed_sys(uint64_t* p, uint64_t v) {
     asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void st_release_gpu(uint64_t* p, uint64_t v) {
+    asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 __device__ __forceinline__ void st_release_sys(uint64_t* p, uint64_t v) {
     asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
@@ -245,17 +253,18 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // its own pack items; with grid <= resident CTAs nothing waits on work that
 // cannot run (deadlock freedom without a global ticket).
 template <bool XCHG, int LW, bool SONLY>
-__device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int* err_flag, uint64_t timeout_ns) {
+__device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa) {
     __shared__ ReqDesc sd;
     __shared__ ReqDesc sa;
     __shared__ XInfo sx;
-    __shared__ uint64_t s_epoch;
     __shared__ int s_ok;
     uint64_t epoch = 0;
+    XCtrl* ctrl = nullptr;
+    TraceRec* trace = nullptr;
     if constexpr (XCHG) {
-        if (threadIdx.x == 0) s_epoch = *reinterpret_cast<volatile unsigned long long*>(&ctrl->epoch) + 1ull;
-        __syncthreads();
-        epoch = s_epoch;
+        epoch = xa->epoch;
+        ctrl = xa->ctrl;
+        trace = xa->trace;
     }
     constexpr int kWords = (int)(sizeof(ReqDesc) / 16);
     constexpr int kXWords = (int)(sizeof(XInfo) / 16);
@@ -296,7 +305,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
         bool run = true;
         uint64_t tr0 = 0, tr1 = 0, tr2 = 0;
         if constexpr (XCHG) {
-            if (ctrl->trace && threadIdx.x == 0) tr0 = globaltimer();
+            if (trace && threadIdx.x == 0) tr0 = globaltimer();
         }
         if constexpr (XCHG) {
             if (sx.wait) {  // acquire: the peer's data / ready signal has arrived
@@ -304,12 +313,13 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
                     const uint64_t* flag = reinterpret_cast<const uint64_t*>(sx.wait) +
                                            (sx.per_item ? (item - cur_first) : 0u);
                     int ok = 1;
-                    if (ld_acquire_sys(flag) < epoch) {
+                    const bool g = sx.gpu_scope != 0;  // the writer runs on this GPU
+                    if ((g ? ld_acquire_gpu(flag) : ld_acquire_sys(flag)) < epoch) {
                         const uint64_t t0 = globaltimer();
-                        while (ld_acquire_sys(flag) < epoch) {
-                            if (globaltimer() - t0 > timeout_ns) {
+                        while ((g ? ld_acquire_gpu(flag) : ld_acquire_sys(flag)) < epoch) {
+                            if (globaltimer() - t0 > xa->timeout_ns) {
                                 ok = 0;
-                                *reinterpret_cast<volatile int*>(err_flag) = 1;
+                                *reinterpret_cast<volatile int*>(xa->err_flag) = 1;
                                 __threadfence_system();
                                 break;
                             }
@@ -321,7 +331,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
                 __syncthreads();
                 run = s_ok != 0;
             }
-            if (ctrl->trace && threadIdx.x == 0) tr1 = globaltimer();
+            if (trace && threadIdx.x == 0) tr1 = globaltimer();
         }
         if (run) run_desc<LW, SONLY>(sd, sa, v0, XCHG && sd.op == OP_UNPACK, (int)tv.ub);
         if constexpr (!XCHG) {
@@ -339,7 +349,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
             }
         }
         if constexpr (XCHG) {
-            if (ctrl->trace) {
+            if (trace) {
                 __syncthreads();
                 if (threadIdx.x == 0) tr2 = globaltimer();
             }
@@ -348,7 +358,8 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
                 if (threadIdx.x == 0) {
                     uint64_t* flag = reinterpret_cast<uint64_t*>(sx.signal);
                     if (sx.per_item) {
-                        st_release_sys(flag + (item - cur_first), epoch);
+                        if (sx.gpu_scope) st_release_gpu(flag + (item - cur_first), epoch);
+                        else st_release_sys(flag + (item - cur_first), epoch);
                     } else if (sx.nitems <= 1) {
                         __threadfence_system();
                         for (uint32_t k = 0; k < sx.fanout; k++) st_relaxed_sys(flag + k, epoch);
@@ -362,10 +373,10 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
                     }
                 }
             }
-            if (ctrl->trace && threadIdx.x == 0) {
+            if (trace && threadIdx.x == 0) {
                 unsigned int slot = atomicAdd(&ctrl->trace_n, 1u);
-                if (slot < ctrl->trace_cap) {
-                    TraceRec* t = reinterpret_cast<TraceRec*>(ctrl->trace) + slot;
+                if (slot < xa->trace_cap) {
+                    TraceRec* t = trace + slot;
                     t->cta = blockIdx.x;
                     t->item = item;
                     t->req = cur;
@@ -375,18 +386,6 @@ __device__ __forceinline__ void fused_body(const TableView& tv, XCtrl* ctrl, int
                     t->t2 = tr2;
                     t->t3 = globaltimer();
                 }
-            }
-        }
-    }
-    if constexpr (XCHG) {
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            __threadfence();
-            unsigned int n = atomicAdd(&ctrl->done, 1u);
-            if (n == gridDim.x - 1) {
-                ctrl->done = 0;
-                *reinterpret_cast<volatile unsigned long long*>(&ctrl->epoch) = epoch;
-                __threadfence();
             }
         }
     }
@@ -400,24 +399,24 @@ template <int V> struct VarT { static constexpr int LW = V == 0 ? -1 : V - 1; st
 
 template <int V>
 __global__ void __launch_bounds__(kThreads) ddt_fused_dev(const uint8_t* __restrict__ table) {
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY>(view_of(table), nullptr, nullptr, 0);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY>(view_of(table), nullptr);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY>(view_of(pb), nullptr, nullptr, 0);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY>(view_of(pb), nullptr);
 }
 
 template <int V>
 __global__ void __launch_bounds__(kThreads)
-    ddt_exchange_dev(const uint8_t* __restrict__ table, XCtrl* ctrl, int* err_flag, uint64_t timeout_ns) {
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY>(view_of(table), ctrl, err_flag, timeout_ns);
+    ddt_exchange_dev(const uint8_t* __restrict__ table, const XArgs xa) {
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY>(view_of(table), &xa);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads)
-    ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, XCtrl* ctrl, int* err_flag, uint64_t timeout_ns) {
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY>(view_of(pb), ctrl, err_flag, timeout_ns);
+    ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, const XArgs xa) {
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY>(view_of(pb), &xa);
 }
 
 // ------------------------------------------------------------------ host side
@@ -464,21 +463,21 @@ static void launch_fused_v(int form, const void* src, uint32_t total, cudaStream
 }
 
 template <int V>
-static void launch_exchange_v(int form, const void* src, uint32_t total, XCtrl* c, int* err, uint64_t timeout_ns,
-                              cudaStream_t s, int grid_cap) {
+static void launch_exchange_v(int form, const void* src, uint32_t total, const XArgs& xa, cudaStream_t s,
+                              int grid_cap) {
     static int res[4] = {0, 0, 0, 0};
     if (form == 1) {
         if (!res[1]) res[1] = resident_ctas(ddt_exchange_param<kParamSmall, V>);
         ddt_exchange_param<kParamSmall, V><<<grid_for(total, res[1], grid_cap), kThreads, 0, s>>>(
-            *reinterpret_cast<const ParamBatch<kParamSmall>*>(src), c, err, timeout_ns);
+            *reinterpret_cast<const ParamBatch<kParamSmall>*>(src), xa);
     } else if (form == 2) {
         if (!res[2]) res[2] = resident_ctas(ddt_exchange_param<kParamLarge, V>);
         ddt_exchange_param<kParamLarge, V><<<grid_for(total, res[2], grid_cap), kThreads, 0, s>>>(
-            *reinterpret_cast<const ParamBatch<kParamLarge>*>(src), c, err, timeout_ns);
+            *reinterpret_cast<const ParamBatch<kParamLarge>*>(src), xa);
     } else {
         if (!res[3]) res[3] = resident_ctas(ddt_exchange_dev<V>);
         ddt_exchange_dev<V><<<grid_for(total, res[3], grid_cap), kThreads, 0, s>>>(
-            reinterpret_cast<const uint8_t*>(src), c, err, timeout_ns);
+            reinterpret_cast<const uint8_t*>(src), xa);
     }
 }
 
@@ -497,18 +496,17 @@ int launch_fused_form(int form, int variant, const void* src, uint32_t total_ite
     return (int)cudaGetLastError();
 }
 
-int launch_exchange_form(int form, int variant, const void* src, uint32_t total_items, void* ctrl, int* err_flag_dev,
-                         uint64_t timeout_ns, void* stream, int grid_cap) {
+int launch_exchange_form(int form, int variant, const void* src, uint32_t total_items, const XArgs& xa, void* stream,
+                         int grid_cap) {
     if (total_items == 0) return 0;
     cudaStream_t s = (cudaStream_t)stream;
-    XCtrl* c = reinterpret_cast<XCtrl*>(ctrl);
     switch (variant) {
-    case 1: launch_exchange_v<1>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
-    case 2: launch_exchange_v<2>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
-    case 3: launch_exchange_v<3>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
-    case 4: launch_exchange_v<4>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
-    case 5: launch_exchange_v<5>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
-    default: launch_exchange_v<0>(form, src, total_items, c, err_flag_dev, timeout_ns, s, grid_cap); break;
+    case 1: launch_exchange_v<1>(form, src, total_items, xa, s, grid_cap); break;
+    case 2: launch_exchange_v<2>(form, src, total_items, xa, s, grid_cap); break;
+    case 3: launch_exchange_v<3>(form, src, total_items, xa, s, grid_cap); break;
+    case 4: launch_exchange_v<4>(form, src, total_items, xa, s, grid_cap); break;
+    case 5: launch_exchange_v<5>(form, src, total_items, xa, s, grid_cap); break;
+    default: launch_exchange_v<0>(form, src, total_items, xa, s, grid_cap); break;
     }
     return (int)cudaGetLastError();
 }

@@ -133,6 +133,9 @@ struct ddt_halo_s {
     uint64_t timeout_ns = 10ull * 1000 * 1000 * 1000;
     int grid_cap = 0;
     bool x_flags = false;         // P2P plan has remote messages (flags); else the plain fused kernel runs
+    uint64_t epoch = 0;           // exchanges issued (every rank issues the same sequence)
+    void* trace = nullptr;        // device TraceRec buffer (tracing on) and its capacity
+    int64_t trace_cap = 0;
     std::vector<void*> ipc_opened;  // peers' receive buffers mapped for pack-free writes
     // graph replay
     bool use_graph = false;
@@ -355,8 +358,19 @@ void free_halo(ddt_halo_s* h) {
 
 ddt_status_t record_exchange(ddt_halo_s* h) {
     if (h->mode != DDT_XCHG_NCCL) {
-        int e = h->x_flags ? launch_exchange(h->x_l, h->ctrl, h->err_dev, h->timeout_ns, h->stream, h->grid_cap)
-                           : launch_fused(h->x_l, h->stream, h->grid_cap);  // self messages only: no signalling
+        int e;
+        if (h->x_flags) {
+            XArgs xa{};
+            xa.ctrl = reinterpret_cast<XCtrl*>(h->ctrl);
+            xa.err_flag = h->err_dev;
+            xa.timeout_ns = h->timeout_ns;
+            xa.epoch = ++h->epoch;  // flags hold the epoch; windows alternate halves by its parity
+            xa.trace = reinterpret_cast<TraceRec*>(h->trace);
+            xa.trace_cap = (unsigned long long)h->trace_cap;
+            e = launch_exchange(h->x_l, xa, h->stream, h->grid_cap);
+        } else {
+            e = launch_fused(h->x_l, h->stream, h->grid_cap);  // self messages only: no signalling
+        }
         if (e) return cuda_fail("exchange kernel launch", e);
         return DDT_OK;
     }
@@ -701,6 +715,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             // (DDT_CHUNK_FLAGS=0: experiments, release every flag at message end)
             const char* cf = getenv("DDT_CHUNK_FLAGS");
             x.per_item = (lw == match[(size_t)i]->lw && !(cf && cf[0] == '0')) ? 1u : 0u;
+            // the reader of this flag runs on our own device (self window): gpu scope suffices
+            x.gpu_scope = s.peer == c->rank ? 1u : 0u;
             x.fanout = (uint32_t)match[(size_t)i]->nflags;  // else: all of the receiver's flags at the end
             xb.xinfo.push_back(x);
         }
@@ -754,6 +770,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                 x.parity_stride = RL.parity_stride;
                 x.per_item = 1;
             }
+            x.gpu_scope = r.peer == c->rank ? 1u : 0u;  // the writer runs on this GPU
             xb.xinfo.push_back(x);
         }
         for (const auto& x : xb.xinfo) h->x_flags |= x.signal != 0 || x.wait != 0;
@@ -802,12 +819,11 @@ ddt_status_t ddt_halo_set_trace(ddt_halo_t h, void* dev_records, int64_t capacit
     if (!h || capacity < 0 || (capacity > 0 && !dev_records)) return DDT_ERR_ARG;
     if (!h->ctrl) return DDT_ERR_STATE;  // tracing covers the fused exchange kernel (P2P plans)
     DevGuard g(h->device);
-    unsigned long long v[2] = {(unsigned long long)(uintptr_t)dev_records, (unsigned long long)capacity};
+    h->trace = capacity > 0 ? dev_records : nullptr;
+    h->trace_cap = capacity;
     unsigned int zero = 0;
-    cudaError_t e = cudaMemcpyAsync((char*)h->ctrl + offsetof(XCtrl, trace), v, sizeof(v), cudaMemcpyHostToDevice,
-                                    h->stream);
-    if (e == cudaSuccess)
-        e = cudaMemcpyAsync((char*)h->ctrl + offsetof(XCtrl, trace_n), &zero, 4, cudaMemcpyHostToDevice, h->stream);
+    cudaError_t e =
+        cudaMemcpyAsync((char*)h->ctrl + offsetof(XCtrl, trace_n), &zero, 4, cudaMemcpyHostToDevice, h->stream);
     if (e == cudaSuccess) e = cudaStreamSynchronize(h->stream);
     return e == cudaSuccess ? DDT_OK : cuda_fail("halo trace", e);
 }
@@ -828,7 +844,9 @@ ddt_status_t ddt_exchange(ddt_halo_t h) {
         return DDT_ERR_TIMEOUT;
     }
     DevGuard g(h->device);
-    if (h->use_graph && h->stream) {
+    // a flagged P2P plan passes the epoch as a kernel argument: launched directly
+    // (a captured graph would freeze it); every other plan may replay a graph
+    if (h->use_graph && h->stream && !(h->mode != DDT_XCHG_NCCL && h->x_flags)) {
         if (!h->gexec) {
             cudaError_t e = cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal);
             if (e != cudaSuccess) return cuda_fail("graph capture begin", e);
