@@ -104,7 +104,7 @@ static int batch_variant(const HostBatch& b) {
     if (lw < 0) return 0;
     for (const auto* v : {&b.descs, &b.aux})
         for (const ReqDesc& d : *v)
-            if (d.nvec && ((d.kind != K_STRIDED && d.kind != K_CONTIG) || d.lw != lw)) return 0;
+            if (d.nvec && ((d.kind != K_STRIDED && d.kind != K_CONTIG && d.kind != K_LL) || d.lw != lw)) return 0;
     return 1 + lw;
 }
 

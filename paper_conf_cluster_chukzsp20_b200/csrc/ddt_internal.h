@@ -107,6 +107,8 @@ ddt_status_t build_direct(ddt_type_s* ts, const DeviceLayout* dls, const void* s
                           const DeviceLayout* dld, void* dst, int64_t dcount, ReqDesc* s, ReqDesc* d);
 ddt_status_t build_typed(ddt_type_s* t, const DeviceLayout* dl, const void* p, int64_t count, ReqDesc* d);
 ddt_status_t rescale_desc(ReqDesc* d, int lw);
+ddt_status_t build_ll(int op, ddt_type_s* t, const DeviceLayout* dl, const void* typed, const void* window,
+                      int64_t count, ReqDesc* s, ReqDesc* d);
 // Largest legal log2 vector width of one typed side (type layout over pointer p).
 int side_lw(ddt_type_s* t, const void* p, int64_t count);
 // Base address of the device allocation containing p (CUDA driver, for IPC).

@@ -181,6 +181,26 @@ ddt_status_t build_typed(ddt_type_s* t, const DeviceLayout* dl, const void* p, i
     return layout_desc(t, dl, p, count, side_lw(t, p, count), d);
 }
 
+// LL exchange request: the typed side at 8-B vectors, the window side in LL
+// format (16 B per vector).  Needs a typed side whose width allows 8 B.
+ddt_status_t build_ll(int op, ddt_type_s* t, const DeviceLayout* dl, const void* typed, const void* window,
+                      int64_t count, ReqDesc* s, ReqDesc* d) {
+    ReqDesc ty, ll;
+    ddt_status_t st = build_typed(t, dl, typed, count, &ty);
+    if (st != DDT_OK) return st;
+    if (ty.lw < 3) return DDT_ERR_UNSUPPORTED;
+    if (ty.lw > 3 && (st = rescale_desc(&ty, 3)) != DDT_OK) return st;
+    std::memset(&ll, 0, sizeof(ll));
+    ll.ptr = (uint64_t)(uintptr_t)window;
+    ll.nvec = ty.nvec;
+    ll.lw = 3;
+    ll.kind = K_LL;
+    *s = op == OP_PACK ? ty : ll;
+    *d = op == OP_PACK ? ll : ty;
+    s->op = d->op = (uint8_t)op;
+    return DDT_OK;
+}
+
 // Re-express a closed-form descriptor at a smaller vector width.
 ddt_status_t rescale_desc(ReqDesc* d, int lw) {
     if (lw > d->lw) return DDT_ERR_ARG;

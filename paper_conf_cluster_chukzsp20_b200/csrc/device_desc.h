@@ -32,7 +32,12 @@ constexpr int kItemVecs = kThreads * kUnroll;  // max vectors per work item
 // DIRECT: typed -> typed (the paper's DirectIPC op; self
 // messages of a halo exchange).  K_CONTIG is the packed side (offset = v * w).
 enum DescOp : uint8_t { OP_PACK = 0, OP_UNPACK = 1, OP_DIRECT = 2, OP_SIGNAL = 3 };  // SIGNAL: ready / wait items, no data
-enum DescKind : uint8_t { K_STRIDED = 0, K_UNIFORM32 = 1, K_UNIFORM64 = 2, K_GENERAL = 3, K_CONTIG = 4 };
+enum DescKind : uint8_t { K_STRIDED = 0, K_UNIFORM32 = 1, K_UNIFORM64 = 2, K_GENERAL = 3, K_CONTIG = 4, K_LL = 5 };
+// K_LL: a window in "low-latency" format (exchange plans, small messages): 8-B
+// vector v lives at byte 16*v as {u32 lo, u32 epoch, u32 hi, u32 epoch}; every
+// 8-byte half carries the exchange epoch, so the receiver validates the data
+// itself -- no release fence, no flag (the LL idea of NCCL's protocols).
+constexpr int64_t kLLMaxBytes = 512 << 10;  // messages up to this size may use LL
 
 // Unsigned 32-bit division by a runtime constant d via a 64-bit reciprocal:
 // q = umulhi64(n, ceil(2^64 / d)) is exact for n, d < 2^32 (error < 1/d);

@@ -9,7 +9,7 @@
 //
 // B200 design: pure HBM-bound byte movement, no tensor
 // cores.  The host builds a work table (exclusive prefix sum of per-request
-// item counts); CTA b walks its contiguous range of items in
+// item counts); CTA b walks items b, b + grid, ... in
 // increasing order (grid <= resident CTAs on the 148 SMs), finds its request
 // with a binary search of the prefix, caches the descriptors in shared memory
 // and moves kItemVecs vectors of the request's packed stream.  Thread i of the
@@ -101,6 +101,7 @@ template <int LW, bool SONLY>
 __device__ __forceinline__ int64_t vec_offset(const ReqDesc& d, uint32_t v) {
     const int lw = LW >= 0 ? LW : d.lw;
     if (d.kind == K_CONTIG) return (int64_t)v << lw;  // the packed side
+    if (d.kind == K_LL) return (int64_t)v << 4;       // 16 B per 8-B vector
     if (SONLY || d.kind == K_STRIDED) {
         uint32_t s = divu(v, d.vps);
         uint32_t within = v - s * d.vps.d;
@@ -138,13 +139,46 @@ __device__ __forceinline__ int64_t vec_offset(const ReqDesc& d, uint32_t v) {
     }
 }
 
-// One work item: kItemVecs vectors starting at v0, loaded through the source
-// descriptor S and stored through the destination descriptor D (one code path
-// for pack, unpack and DirectIPC).  coh: the source is written by another GPU
-// during this kernel (P2P window) -> L2-coherent loads instead of the
-// non-coherent read-only path.
-template <int LW, bool SONLY>
-__device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uint32_t v0, bool coh, int ub) {
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+    uint64_t t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
+// LL receive: spin until both halves of the 16-B word carry this epoch.
+__device__ __forceinline__ uint4 ll_load(const uint8_t* p, uint32_t epoch, const XArgs* xa) {
+    uint4 r;
+    uint64_t t0 = 0;
+    for (uint32_t n = 0;; n++) {
+        asm volatile("ld.volatile.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+                     : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p) : "memory");
+        if (r.y == epoch && r.w == epoch) break;
+        if ((n & 63) == 0) {
+            const uint64_t t = globaltimer_ns();
+            if (n == 0) t0 = t;
+            else if (t - t0 > xa->timeout_ns) {
+                *reinterpret_cast<volatile int*>(xa->err_flag) = 1;
+                break;
+            }
+        }
+        __nanosleep(64);
+    }
+    return make_uint4(r.x, r.z, 0u, 0u);
+}
+
+__device__ __forceinline__ void ll_store(uint8_t* p, const uint4& d, uint32_t epoch) {
+    asm volatile("st.volatile.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(d.x), "r"(epoch), "r"(d.y),
+                 "r"(epoch) : "memory");
+}
+
+// One work item: up to kItemVecs vectors starting at v0, loaded through the
+// source descriptor S and stored through the destination descriptor D (one
+// code path for pack, unpack and DirectIPC).  coh: the source is written by
+// another GPU during this kernel (P2P window) -> L2-coherent loads instead of
+// the non-coherent read-only path.  XC: exchange kernel (LL windows possible).
+template <int LW, bool SONLY, bool XC>
+__device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uint32_t v0, bool coh, int ub,
+                                         const XArgs* xa = nullptr, uint32_t epoch = 0) {
     const uint32_t nvec = S.nvec;
     const int lw = LW >= 0 ? LW : S.lw;
     const uint8_t* src = reinterpret_cast<const uint8_t*>(S.ptr);
@@ -155,13 +189,18 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
         uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
         if (u < ub && v < nvec) {
             const uint8_t* p = src + vec_offset<LW, SONLY>(S, v);
-            buf[u] = coh ? ld_vec<false, LW>(p, lw) : ld_vec<true, LW>(p, lw);
+            if (XC && S.kind == K_LL) buf[u] = ll_load(p, epoch, xa);
+            else buf[u] = coh ? ld_vec<false, LW>(p, lw) : ld_vec<true, LW>(p, lw);
         }
     }
 #pragma unroll
     for (int u = 0; u < kUnroll; u++) {
         uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-        if (u < ub && v < nvec) st_vec<LW>(dst + vec_offset<LW, SONLY>(D, v), lw, buf[u]);
+        if (u < ub && v < nvec) {
+            uint8_t* p = dst + vec_offset<LW, SONLY>(D, v);
+            if (XC && D.kind == K_LL) ll_store(p, buf[u], epoch);
+            else st_vec<LW>(p, lw, buf[u]);
+        }
     }
 }
 
@@ -333,7 +372,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             }
             if (trace && threadIdx.x == 0) tr1 = globaltimer();
         }
-        if (run) run_desc<LW, SONLY>(sd, sa, v0, XCHG && sd.op == OP_UNPACK, (int)tv.ub);
+        if (run) run_desc<LW, SONLY, XCHG>(sd, sa, v0, XCHG && sd.op == OP_UNPACK, (int)tv.ub, xa, (uint32_t)epoch);
         if constexpr (!XCHG) {
             if (sd.resp) {  // scheduler (3): the CTA finishing the request's last item signals it
                 __syncthreads();

@@ -50,6 +50,7 @@ struct RecvLayout {
     std::vector<int> flag_idx;       // per recv index: first of its per-chunk flag slots
     std::vector<int> lw;             // per recv index: vector width of the unpack side
     std::vector<int> nflags;         // per recv index: chunks (items at kXchgUb) of the message
+    std::vector<int> ll_ok;          // per recv index: window space reserved for the LL format
     int64_t ready_off = 0;           // byte offset of the per-sender "ready" slots (pack-free mode)
     int64_t flags_bytes = 0, parity_stride = 0, window_bytes = 0;
 };
@@ -65,6 +66,7 @@ RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs) {
     L.flag_idx.assign((size_t)nrecv, 0);
     L.lw.assign((size_t)nrecv, 0);
     L.nflags.assign((size_t)nrecv, 1);
+    L.ll_ok.assign((size_t)nrecv, 0);
     int64_t off = 0, nflag = 0;
     const int64_t chunk = (int64_t)kThreads * kXchgUb;  // vectors per exchange item
     for (size_t k = 0; k < L.order.size(); k++) {
@@ -77,7 +79,9 @@ RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs) {
         L.nflags[(size_t)i] = (int)std::max<int64_t>(1, ((bytes >> lw) + chunk - 1) / chunk);
         L.flag_idx[(size_t)i] = (int)nflag;
         nflag += L.nflags[(size_t)i];
-        off += bytes;
+        // small messages of 8-B-capable layouts may travel in LL format (2x the bytes)
+        L.ll_ok[(size_t)i] = (lw >= 3 && bytes <= kLLMaxBytes && bytes % 8 == 0) ? 1 : 0;
+        off += L.ll_ok[(size_t)i] ? 2 * bytes : bytes;
     }
     int64_t nready = 0;  // one slot per possible sender rank
     for (int i = 0; i < nrecv; i++) nready = std::max<int64_t>(nready, (int64_t)recvs[i].peer + 1);
@@ -89,7 +93,7 @@ RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs) {
 }
 
 struct DirEntry {
-    int64_t tag, bytes, data_off, flag_idx, lw, nflags;
+    int64_t tag, bytes, data_off, flag_idx, lw, nflags, ll_ok;
     // pack-free mode: where the receive buffer lives and how it is laid out
     int64_t ipc[8];      // cudaIpcMemHandle_t of the buffer's allocation
     int64_t alloc_off;   // buffer address - allocation base
@@ -312,7 +316,7 @@ ddt_status_t agree(ddt_halo_s* h, ddt_status_t mine) {
 }
 
 // [n, parity_stride, data_base, ready_base, direct] then n entries of
-// [tag, bytes, data_off, flag_idx, lw, nflags] (+ [ipc x8, alloc_off, desc x kDescWords] if direct)
+// [tag, bytes, data_off, flag_idx, lw, nflags, ll_ok] (+ [ipc x8, alloc_off, desc x kDescWords] if direct)
 Directory parse_dir(const std::vector<int64_t>& v) {
     Directory d;
     if (v.size() < 5) return d;
@@ -322,7 +326,7 @@ Directory parse_dir(const std::vector<int64_t>& v) {
     d.ready_base = v[3];
     d.direct = v[4];
     size_t pos = 5;
-    const size_t stride = 6 + (d.direct ? 9 + kDescWords : 0);
+    const size_t stride = 7 + (d.direct ? 9 + kDescWords : 0);
     for (int64_t i = 0; i < n && pos + stride <= v.size(); i++, pos += stride) {
         DirEntry e{};
         e.tag = v[pos];
@@ -331,10 +335,11 @@ Directory parse_dir(const std::vector<int64_t>& v) {
         e.flag_idx = v[pos + 3];
         e.lw = v[pos + 4];
         e.nflags = v[pos + 5];
+        e.ll_ok = v[pos + 6];
         if (d.direct) {
-            std::memcpy(e.ipc, &v[pos + 6], 64);
-            e.alloc_off = v[pos + 14];
-            std::memcpy(&e.desc, &v[pos + 15], sizeof(ReqDesc));
+            std::memcpy(e.ipc, &v[pos + 7], 64);
+            e.alloc_off = v[pos + 15];
+            std::memcpy(&e.desc, &v[pos + 16], sizeof(ReqDesc));
         }
         d.e.push_back(e);
     }
@@ -495,6 +500,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             v.push_back(RL.flag_idx[(size_t)k]);
             v.push_back(RL.lw[(size_t)k]);
             v.push_back(RL.nflags[(size_t)k]);
+            v.push_back(RL.ll_ok[(size_t)k]);
             if (!dmsg) continue;
             // pack-free: publish the receive buffer (IPC handle + offset) and its layout
             int64_t words[9 + kDescWords] = {0};
@@ -567,6 +573,52 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     if (st != DDT_OK) {
         free_halo(h);
         return st;
+    }
+
+    // test hook (never set in production): route self messages through the
+    // window path instead of DirectIPC, so single-GPU tests and benchmarks
+    // exercise and time the multi-GPU protocols
+    const char* svw = getenv("DDT_SELF_VIA_WINDOW");
+    const bool self_window = p2p && !direct && svw && svw[0] == '1';
+    auto remote = [&](int peer) { return peer != c->rank || self_window; };
+
+    // ---- second metadata round (window mode): sender -> receiver, which
+    // messages travel in the LL format (receiver offered it, sender can do 8-B)
+    std::map<std::pair<int, int>, int> send_ll, recv_ll;
+    if (p2p && !direct) {
+        std::vector<std::vector<int64_t>> out2((size_t)P), in2;
+        std::vector<std::vector<std::pair<int64_t, int64_t>>> lists((size_t)P);
+        for (int i = 0; i < nsend; i++) {
+            const auto& s = sends[i];
+            if (s.count * s.type->size == 0 || !remote(s.peer)) continue;
+            const int lw_s = std::min(4, side_lw(s.type, s.buf, s.count));
+            const int ll = (match[(size_t)i]->ll_ok && lw_s >= 3) ? 1 : 0;
+            send_ll[{s.peer, s.tag}] = ll;
+            lists[(size_t)s.peer].push_back({s.tag, ll});
+        }
+        for (int p = 0; p < P; p++) {
+            std::sort(lists[(size_t)p].begin(), lists[(size_t)p].end());
+            out2[(size_t)p].push_back((int64_t)lists[(size_t)p].size());
+            for (auto& e : lists[(size_t)p]) {
+                out2[(size_t)p].push_back(e.first);
+                out2[(size_t)p].push_back(e.second);
+            }
+        }
+        if (P > 1) {
+            st = h->ag ? exchange_directories_host(h, out2, in2) : exchange_directories(h, out2, in2);
+            if (st != DDT_OK) {
+                free_halo(h);
+                return st;
+            }
+        } else {
+            in2.assign(1, {});
+        }
+        in2[(size_t)c->rank] = out2[(size_t)c->rank];
+        for (int p = 0; p < P; p++) {
+            const auto& v = in2[(size_t)p];
+            for (int64_t k = 0; v.size() >= 1 && k < v[0] && (size_t)(2 + 2 * k) < v.size() + 1; k++)
+                recv_ll[{p, (int)v[(size_t)(1 + 2 * k)]}] = (int)v[(size_t)(2 + 2 * k)];
+        }
     }
 
     // ---- build the device work tables
@@ -675,12 +727,6 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         HostBatch xb;
         char* mywin = (char*)c->peer_windows[c->rank];
         uint32_t npack = 0;
-        // test hook (never set in production): route self messages through the
-        // window + flag path instead of DirectIPC, so the single-GPU tests and
-        // benchmarks exercise and time the multi-GPU signalling protocol
-        const char* svw = getenv("DDT_SELF_VIA_WINDOW");
-        const bool self_window = !direct && svw && svw[0] == '1';
-        auto remote = [&](int peer) { return peer != c->rank || self_window; };
         ReqDesc none;
         std::memset(&none, 0, sizeof(none));
         none.kind = K_CONTIG;
@@ -705,6 +751,20 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             if (s.count * s.type->size == 0 || !remote(s.peer)) continue;
             const Directory& d = dirs[(size_t)s.peer];
             char* win = (char*)c->peer_windows[s.peer];
+            if (send_ll[{s.peer, s.tag}]) {  // LL: the data carries its own epoch, no signal
+                DeviceLayout* dl = nullptr;
+                ReqDesc sd, dd;
+                st = type_device_layout(s.type, h->device, &dl);
+                if (st == DDT_OK)
+                    st = build_ll(OP_PACK, s.type, dl, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count,
+                                  &sd, &dd);
+                if (st != DDT_OK) break;
+                xb.add(sd, dd);
+                XInfo x{};
+                x.parity_stride = d.parity_stride;
+                xb.xinfo.push_back(x);
+                continue;
+            }
             int lw = 0;
             st = add_req(xb, s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, &lw);
             XInfo x{};
@@ -764,6 +824,17 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             x.wait = (uint64_t)(uintptr_t)(mywin + 8 * RL.flag_idx[(size_t)i]);
             if (direct) {  // the data lands by itself; wait for its completion flag
                 xb.add(none, none);
+            } else if (recv_ll[{r.peer, r.tag}]) {  // LL: every 8 B validates itself
+                DeviceLayout* dl = nullptr;
+                ReqDesc sd, dd;
+                st = type_device_layout(r.type, h->device, &dl);
+                if (st == DDT_OK)
+                    st = build_ll(OP_UNPACK, r.type, dl, r.buf, mywin + RL.flags_bytes + RL.data_off[(size_t)i],
+                                  r.count, &sd, &dd);
+                if (st != DDT_OK) break;
+                xb.add(sd, dd);
+                x.wait = 0;
+                x.parity_stride = RL.parity_stride;
             } else {  // unpack chunk k as soon as the sender's chunk k has landed
                 st = add_req(xb, r.type, OP_UNPACK, mywin + RL.flags_bytes + RL.data_off[(size_t)i], r.buf, r.count,
                              nullptr);
@@ -774,6 +845,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             xb.xinfo.push_back(x);
         }
         for (const auto& x : xb.xinfo) h->x_flags |= x.signal != 0 || x.wait != 0;
+        for (size_t i = 0; i < xb.descs.size(); i++)  // LL windows need the exchange kernel (and its epoch)
+            h->x_flags |= xb.descs[i].kind == K_LL || xb.aux[xb.descs[i].aux].kind == K_LL;
         if (st == DDT_OK && !xb.descs.empty()) {
             // exchange plans chunk every message alike on both sides (kXchgUb)
             for (size_t i = 0; i < xb.descs.size(); i++)
