@@ -592,7 +592,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             const auto& s = sends[i];
             if (s.count * s.type->size == 0 || !remote(s.peer)) continue;
             const int lw_s = std::min(4, side_lw(s.type, s.buf, s.count));
-            const int ll = (match[(size_t)i]->ll_ok && lw_s >= 3) ? 1 : 0;
+            const char* nl = getenv("DDT_NO_LL");  // experiments: flag protocol only
+            const int ll = (match[(size_t)i]->ll_ok && lw_s >= 3 && !(nl && nl[0] == '1')) ? 1 : 0;
             send_ll[{s.peer, s.tag}] = ll;
             lists[(size_t)s.peer].push_back({s.tag, ll});
         }
@@ -776,7 +777,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             const char* cf = getenv("DDT_CHUNK_FLAGS");
             x.per_item = (lw == match[(size_t)i]->lw && !(cf && cf[0] == '0')) ? 1u : 0u;
             // the reader of this flag runs on our own device (self window): gpu scope suffices
-            x.gpu_scope = s.peer == c->rank ? 1u : 0u;
+            const char* fs = getenv("DDT_FORCE_SYS_SCOPE");  // experiments: emulate a peer GPU's flags
+            x.gpu_scope = (s.peer == c->rank && !(fs && fs[0] == '1')) ? 1u : 0u;
             x.fanout = (uint32_t)match[(size_t)i]->nflags;  // else: all of the receiver's flags at the end
             xb.xinfo.push_back(x);
         }
@@ -841,7 +843,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                 x.parity_stride = RL.parity_stride;
                 x.per_item = 1;
             }
-            x.gpu_scope = r.peer == c->rank ? 1u : 0u;  // the writer runs on this GPU
+            const char* fs2 = getenv("DDT_FORCE_SYS_SCOPE");
+            x.gpu_scope = (r.peer == c->rank && !(fs2 && fs2[0] == '1')) ? 1u : 0u;  // the writer runs on this GPU
             xb.xinfo.push_back(x);
         }
         for (const auto& x : xb.xinfo) h->x_flags |= x.signal != 0 || x.wait != 0;
