@@ -68,6 +68,17 @@ def config3_cm_spec(nblocks: int = 100_000, npoints: int = 1 << 20, s: int | Non
     return spec, 12 * npoints
 
 
+def milc_spec(L: int = 16):
+    """MILC-style nested vector ("nested vectors (MILC)"; SURVEY
+    D2/W4): the y = 0 face of an L^4 lattice of su3 vectors (3 complex doubles =
+    6 doubles per site, x fastest): an hvector over t of a vector over z of
+    x-rows.  Returns (spec, footprint_bytes)."""
+    row = L * 6                                   # doubles per x-row
+    inner = ("vector", L, row, L * row, ("basic", "double"))          # z rows at stride L*L sites
+    spec = ("hvector", L, 1, L ** 3 * 6 * 8, inner)                   # t planes at stride L^3 sites
+    return spec, L ** 4 * 48
+
+
 # ----------------------------------------------------------------- config 5
 def config5_spec(S: int):
     """BASELINE.json configs[4]: dense vector of doubles, block = min(S, 256 B),

@@ -386,3 +386,12 @@ def test_config3_cm_struct_on_indexed_full(ddt, q):
     eu = np.full(nb, SENTINEL, np.uint8)
     oracle.unpack(o, exp, eu)
     assert_bytes_equal(host(d_un), eu, "config3-cm unpack")
+
+
+@pytest.mark.parametrize("L", [6, 16])
+def test_milc_nested_vector(ddt, q, L):
+    """MILC-style hvector-of-vector face of an L^4 su3 lattice: pack + unpack bit-exact."""
+    from ddt_inputs import milc_spec
+    spec, fp = milc_spec(L)
+    _run_case(ddt, q, Case(ddt, spec, 1, misalign=0, seed=L))
+    _run_case(ddt, q, Case(ddt, spec, 2, misalign=8, seed=L + 1))

@@ -421,3 +421,13 @@ def test_config3_cm_struct_on_indexed_matches_fancy_indexing():
     f = src.view(np.float32).reshape(3, -1)
     idx = np.array(spec[3][0][2])
     np.testing.assert_array_equal(oracle.pack(t, src), np.concatenate([f[0][idx], f[1][idx], f[2][idx]]).view(np.uint8))
+
+
+def test_milc_nested_vector_matches_numpy():
+    from ddt_inputs import milc_spec
+    L = 4
+    spec, fp = milc_spec(L)
+    t = oracle.Type(spec)
+    src = random_bytes(fp, 31)
+    lat = src.view(np.float64).reshape(L, L, L, L, 6)          # [t][z][y][x][6]
+    np.testing.assert_array_equal(oracle.pack(t, src).view(np.float64), lat[:, :, 0, :, :].reshape(-1))
