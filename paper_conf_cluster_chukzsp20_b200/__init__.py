@@ -21,6 +21,6 @@ from ._abi import (DDTError, lib, check, LAYOUT_KINDS, BASE_CODES, STATE_NAMES, 
                    DDT_XCHG_NCCL, DDT_XCHG_P2P, DDT_XCHG_P2P_DIRECT, DDT_PENDING, DDT_BUSY, DDT_COMPLETED)
 from .types import Type  # noqa: F401
 from .queue import Queue, Plan  # noqa: F401
-from .halo import Halo, Comm  # noqa: F401
+from .halo import Halo, Comm, Windows  # noqa: F401
 
-__all__ = ["DDTError", "Type", "Queue", "Plan", "Halo", "Comm", "lib", "DDT_XCHG_NCCL", "DDT_XCHG_P2P"]
+__all__ = ["DDTError", "Type", "Queue", "Plan", "Halo", "Comm", "Windows", "lib", "DDT_XCHG_NCCL", "DDT_XCHG_P2P"]

@@ -854,7 +854,9 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             // exchange plans chunk every message alike on both sides (kXchgUb)
             for (size_t i = 0; i < xb.descs.size(); i++)
                 if (xb.xinfo[i].signal) xb.xinfo[i].nitems = desc_items(xb.descs[i], kXchgUb);
-            st = make_table(xb, h->x_l, queue_sm_count(q), kXchgUb);
+            // flag-free plans (self messages only) run the plain fused kernel:
+            // adaptive item size, like any other batch
+            st = make_table(xb, h->x_l, queue_sm_count(q), h->x_flags ? kXchgUb : 0);
         }
         size_t ctrl_bytes = sizeof(XCtrl) + sizeof(unsigned long long) * std::max<size_t>(npack, 1);
         if (st == DDT_OK) {

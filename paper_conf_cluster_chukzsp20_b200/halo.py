@@ -37,9 +37,47 @@ def _c_allgather(gather):
     return ALLGATHER_FN(cb)
 
 
+class Windows:
+    """One plan's symmetric receive windows: this rank's window (ddt_window_alloc)
+    and every peer's, opened through CUDA IPC (collective over comm.gather).
+    Each P2P / P2P_DIRECT plan owns its own set: flags hold the plan's epoch, so
+    two plans sharing a window would read each other's signals."""
+
+    def __init__(self, comm, nbytes: int):
+        self.comm, self.nbytes = comm, int(nbytes)
+        ptr = P()
+        handle = ctypes.create_string_buffer(64)
+        check(lib().ddt_window_alloc(comm.device, self.nbytes, ctypes.byref(ptr), handle), "ddt_window_alloc")
+        self.own = ptr.value
+        self._opened = []
+        ptrs = [0] * comm.nranks
+        ptrs[comm.rank] = ptr.value
+        if comm.nranks > 1:
+            import pickle
+            allh = [pickle.loads(b) for b in comm.gather(pickle.dumps((bytes(handle.raw), self.nbytes)))]
+            for p, (h, nb) in enumerate(allh):
+                if p == comm.rank:
+                    continue
+                q = P()
+                check(lib().ddt_window_open(comm.device, ctypes.create_string_buffer(h, 64), ctypes.byref(q)),
+                      "ddt_window_open")
+                ptrs[p] = q.value
+                self._opened.append(q.value)
+        self.peer_ptrs = (P * comm.nranks)(*ptrs)
+
+    def close(self):
+        """Every rank must have finished its last exchange on the plan first."""
+        for q in self._opened:
+            lib().ddt_window_close(ctypes.c_void_p(q))
+        self._opened = []
+        if self.own:
+            lib().ddt_window_free(ctypes.c_void_p(self.own))
+            self.own = None
+
+
 class Comm:
-    """rank / nranks, an NCCL communicator (nranks > 1) and, for the P2P mode,
-    the device pointers of every rank's receive window."""
+    """rank / nranks, the host all-gather used for plan metadata and window
+    handles, and an NCCL communicator (nranks > 1, NCCL mode)."""
 
     def __init__(self, rank: int = 0, nranks: int = 1, device: int = 0, nccl_comm=None, group=None, gather=None):
         self.rank, self.nranks, self.device = int(rank), int(nranks), int(device)
@@ -47,10 +85,6 @@ class Comm:
         self.group = group
         self.gather = gather        # python all-gather of bytes (metadata plumbing)
         self._cb = _c_allgather(gather) if gather is not None else None
-        self.window = None          # own window (device pointer)
-        self.window_bytes = 0
-        self.peer_windows = None    # ctypes array of device pointers (own included)
-        self._opened = []
 
     @staticmethod
     def single(device: int = 0) -> "Comm":
@@ -79,45 +113,18 @@ class Comm:
             c.nccl_comm = comm
         return c
 
-    def setup_windows(self, nbytes: int):
-        """Allocate this rank's receive window and map every peer's (CUDA IPC)."""
-        ptr = P()
-        handle = ctypes.create_string_buffer(64)
-        check(lib().ddt_window_alloc(self.device, int(nbytes), ctypes.byref(ptr), handle), "ddt_window_alloc")
-        self.window, self.window_bytes = ptr.value, int(nbytes)
-        ptrs = [0] * self.nranks
-        ptrs[self.rank] = ptr.value
-        if self.nranks > 1:
-            import pickle
-            allh = [pickle.loads(b) for b in self.gather(pickle.dumps((bytes(handle.raw), int(nbytes))))]
-            for p, (h, nb) in enumerate(allh):
-                if p == self.rank:
-                    continue
-                q = P()
-                check(lib().ddt_window_open(self.device, ctypes.create_string_buffer(h, 64), ctypes.byref(q)),
-                      "ddt_window_open")
-                ptrs[p] = q.value
-                self._opened.append(q.value)
-        self.peer_windows = (P * self.nranks)(*ptrs)
-        return self.window
-
-    def as_struct(self) -> ddt_comm_t:
+    def as_struct(self, windows=None) -> ddt_comm_t:
         c = ddt_comm_t()
         c.rank, c.nranks = self.rank, self.nranks
         c.nccl_comm = self.nccl_comm.value if isinstance(self.nccl_comm, P) else self.nccl_comm
-        c.peer_windows = ctypes.cast(self.peer_windows, ctypes.POINTER(P)) if self.peer_windows else None
-        c.window_bytes = self.window_bytes
+        if windows is not None:
+            c.peer_windows = ctypes.cast(windows.peer_ptrs, ctypes.POINTER(P))
+            c.window_bytes = windows.nbytes
         if self._cb is not None:
             c.host_allgather = self._cb
         return c
 
     def close(self):
-        for q in self._opened:
-            lib().ddt_window_close(ctypes.c_void_p(q))
-        self._opened = []
-        if self.window:
-            lib().ddt_window_free(ctypes.c_void_p(self.window))
-            self.window = None
         if self.nccl_comm is not None:
             lib().ddt_nccl_comm_destroy(self.nccl_comm)
             self.nccl_comm = None
@@ -145,14 +152,21 @@ class Halo:
         s_arr = _msgs(sends, ddt_send_t)
         r_arr = _msgs(recvs, ddt_recv_t)
         self.mode = {"nccl": DDT_XCHG_NCCL, "p2p": DDT_XCHG_P2P, "p2p_direct": DDT_XCHG_P2P_DIRECT}[mode]
-        if self.mode != DDT_XCHG_NCCL and comm.window is None:
+        self.windows = None
+        if self.mode != DDT_XCHG_NCCL:
             nb = ctypes.c_int64()
             check(lib().ddt_halo_window_bytes(len(recvs), r_arr, ctypes.byref(nb)), "ddt_halo_window_bytes")
-            comm.setup_windows(nb.value)
-        cs = comm.as_struct()
+            self.windows = Windows(comm, nb.value)
+        cs = comm.as_struct(self.windows)
         out = P()
-        check(lib().ddt_halo_create(queue.handle, ctypes.byref(cs), len(sends), s_arr, len(recvs), r_arr,
-                                    self.mode, ctypes.byref(out)), "ddt_halo_create")
+        try:
+            check(lib().ddt_halo_create(queue.handle, ctypes.byref(cs), len(sends), s_arr, len(recvs), r_arr,
+                                        self.mode, ctypes.byref(out)), "ddt_halo_create")
+        except Exception:
+            if self.windows is not None:
+                self.windows.close()
+                self.windows = None
+            raise
         self._h = out
         check(lib().ddt_halo_set_graph(self._h, 1 if graph else 0), "ddt_halo_set_graph")
 
@@ -187,9 +201,14 @@ class Halo:
         return v.value
 
     def destroy(self):
+        """Frees the plan and its windows: every rank must have finished its last
+        exchange on this plan (synchronize + barrier) before any rank destroys it."""
         if self._h and self._h.value:
             check(lib().ddt_halo_destroy(self._h), "ddt_halo_destroy")
         self._h = P()
+        if getattr(self, "windows", None) is not None:
+            self.windows.close()
+            self.windows = None
 
     def __del__(self):
         try:

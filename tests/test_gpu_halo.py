@@ -108,6 +108,37 @@ def test_config2_face_halo_full_size(ddt, mode):
     comm.close()
 
 
+def test_config2_bench_launch_configuration(ddt):
+    """bench.py's N = 1 launch configuration at full size: R independent 130^3
+    arrays with one plan each (graph=False) on a side stream, K steps round
+    robin captured into ONE CUDA graph, replayed; every replica's ghosts must
+    equal np.pad(wrap) after each replay (sentinels reset in between)."""
+    import torch
+    local = (128, 128, 128)
+    R, K = 3, 7
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        reps = [_setup(ddt, local, FACE_DIRS, 1, "p2p", False, 2) for _ in range(R)]
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for k in range(K):
+                reps[k % R][2].exchange()
+        for it in range(2):
+            befores = []
+            for r, (_, arrs, _, _) in enumerate(reps):
+                arrs[0].view(torch.uint8).fill_(0xA5)
+                _fill_interior(arrs, local, 10 * it + r, 2)
+                befores.append([arrs[0][1:-1, 1:-1, 1:-1].cpu().numpy()])
+            g.replay()
+            torch.cuda.synchronize()
+            for (_, arrs, _, _), before in zip(reps, befores):
+                _check(arrs, local, FACE_DIRS, before)
+        for q, _, h, comm in reps:
+            h.destroy()
+            comm.close()
+            q.destroy()
+
+
 def test_config4_comb_halo_full_size_p1(ddt):
     """BASELINE.json configs[3] at its 1-GPU point: 512^3 doubles, 4 variables,
     26 neighbours, 104 + 104 messages per iteration; variable 0 fully checked,

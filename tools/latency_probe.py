@@ -67,6 +67,63 @@ def main():
                   f"{per_iter(h.exchange, flush=flush)} b2b {back_to_back(h.exchange):.2f}")
             h.destroy()
             q.destroy()
+    rotating(sends, recvs, local)
+
+
+def rotating(sends0, recvs0, local, R=64, K=640):
+    """configs[1] exchanges over R independent 130^3 arrays (touched DRAM
+    footprint R x ~3 MB > L2), K back to back: (a) host-issued launches,
+    (b) captured K-exchange CUDA graph; plus a K-node graph of trivial kernels
+    as the launch floor.  Per-exchange device time = total / K."""
+    s = torch.cuda.Stream()
+    torch.cuda.set_stream(s)
+    msgs = halo_messages(0, 1, local, dirs=FACE_DIRS)
+    q = ddt.Queue(stream=s)
+    arrs, halos = [], []
+    for r in range(R):
+        a = torch.zeros((130, 130, 130), dtype=torch.int64, device="cuda")
+        sends = [(m["peer"], m["tag"], ddt.Type.from_spec(m["send_spec"]), a, 1) for m in msgs]
+        recvs = [(m["recv_peer"], m["recv_tag"], ddt.Type.from_spec(m["recv_spec"]), a, 1) for m in msgs]
+        arrs.append(a)
+        halos.append(ddt.Halo(q, ddt.Comm.single(0), sends, recvs, mode="p2p", graph=False))
+
+    def host_loop():
+        for k in range(K):
+            halos[k % R].exchange()
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(2)]
+    host_loop()
+    torch.cuda.synchronize()
+    ev[0].record(s)
+    host_loop()
+    ev[1].record(s)
+    torch.cuda.synchronize()
+    print(f"rotating R={R} host-issued b2b: {ev[0].elapsed_time(ev[1]) * 1e3 / K:.2f} us/exchange")
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        for k in range(K):
+            halos[k % R].exchange()
+    g.replay()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(5):
+        ev[0].record(s)
+        g.replay()
+        ev[1].record(s)
+        torch.cuda.synchronize()
+        ts.append(ev[0].elapsed_time(ev[1]) * 1e3 / K)
+    print(f"rotating R={R} K-exchange graph: {statistics.median(ts):.2f} us/exchange")
+    x = torch.zeros(1, device="cuda")
+    g2 = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g2, stream=s):
+        for k in range(K):
+            x.add_(1)
+    g2.replay()
+    torch.cuda.synchronize()
+    ev[0].record(s)
+    g2.replay()
+    ev[1].record(s)
+    torch.cuda.synchronize()
+    print(f"trivial K-node graph: {ev[0].elapsed_time(ev[1]) * 1e3 / K:.2f} us/node")
 
 
 if __name__ == "__main__":
