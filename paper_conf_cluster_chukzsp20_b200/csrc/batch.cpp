@@ -16,11 +16,16 @@
 
 namespace ddt {
 
-static uint32_t fill_prefix(uint32_t* prefix, const std::vector<ReqDesc>& d, int ub) {
+// Exclusive prefix of item counts; a group of m members occupies m * n items
+// and every member's entry holds the group's first item (device_desc.h).
+static uint32_t fill_prefix(uint32_t* prefix, const HostBatch& b, int ub) {
+    const std::vector<ReqDesc>& d = b.descs;
     uint64_t acc = 0;
-    for (size_t i = 0; i < d.size(); i++) {
-        prefix[i] = (uint32_t)acc;
-        acc += desc_items(d[i], ub);
+    for (size_t i = 0; i < d.size();) {
+        const size_t m = b.gm.empty() ? 1 : std::max<uint32_t>(1, b.gm[i]);
+        for (size_t j = 0; j < m; j++) prefix[i + j] = (uint32_t)acc;
+        acc += (uint64_t)m * desc_items(d[i], ub);
+        i += m;
     }
     prefix[d.size()] = (uint32_t)acc;
     return (uint32_t)acc;
@@ -29,14 +34,65 @@ static uint32_t fill_prefix(uint32_t* prefix, const std::vector<ReqDesc>& d, int
 static size_t pad16(size_t v) { return (v + 15) & ~(size_t)15; }
 
 // Item order (experiments: DDT_ITEM_ORDER=blocked); cyclic is the default.
-static uint32_t item_order_blocked() {
+static uint32_t batch_flags(const HostBatch& b) {
     const char* e = getenv("DDT_ITEM_ORDER");
-    return (e && e[0] == 'b') ? 1u : 0u;
+    uint32_t f = (e && e[0] == 'b') ? kBatchBlocked : 0u;
+    if (!b.gm.empty()) f |= kBatchGrouped;
+    return f;
+}
+
+// An LL unpack spins on its window data: it waits like a flagged unpack.
+static int exchange_class(const HostBatch& b, size_t i) {
+    if (b.xinfo.empty()) return 0;
+    const bool waits = b.xinfo[i].wait != 0 || b.descs[i].kind == K_LL;
+    return (waits ? 2 : 0) | (b.xinfo[i].signal ? 1 : 0);
+}
+
+void group_equal_requests(HostBatch& b, int ub, int max_m) {
+    const char* off = getenv("DDT_NO_GROUP");  // experiments: no interleaving
+    const size_t n = b.descs.size();
+    if ((off && off[0] == '1') || n < 2 || max_m < 2) return;
+    std::vector<size_t> order;
+    std::vector<uint32_t> gm;
+    order.reserve(n);
+    for (size_t lo = 0; lo < n;) {
+        size_t hi = lo + 1;
+        while (hi < n && exchange_class(b, hi) == exchange_class(b, lo)) hi++;
+        // within [lo, hi): requests with equal item counts, in first-seen order
+        std::vector<bool> taken(hi - lo, false);
+        for (size_t i = lo; i < hi; i++) {
+            if (taken[i - lo]) continue;
+            const uint32_t it = desc_items(b.descs[i], ub);
+            std::vector<size_t> g{i};
+            taken[i - lo] = true;
+            for (size_t j = i + 1; j < hi && it > 0 && g.size() < (size_t)max_m; j++)
+                if (!taken[j - lo] && desc_items(b.descs[j], ub) == it) {
+                    g.push_back(j);
+                    taken[j - lo] = true;
+                }
+            for (size_t k : g) {
+                order.push_back(k);
+                gm.push_back((uint32_t)g.size());
+            }
+        }
+        lo = hi;
+    }
+    bool any = false;
+    for (uint32_t m : gm) any |= m > 1;
+    if (!any) return;
+    HostBatch out;
+    for (size_t k : order) {
+        out.add(b.descs[k], b.aux[b.descs[k].aux]);
+        if (!b.xinfo.empty()) out.xinfo.push_back(b.xinfo[k]);
+    }
+    out.gm = std::move(gm);
+    b = std::move(out);
 }
 
 size_t device_table_bytes(const HostBatch& b) {
     size_t n = b.descs.size();
     size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
+    if (!b.gm.empty()) off += pad16(n * 4);
     off += n * sizeof(ReqDesc) + b.aux.size() * sizeof(ReqDesc);
     if (!b.xinfo.empty()) off += n * sizeof(XInfo);
     return off;
@@ -58,10 +114,14 @@ uint32_t write_device_table(void* dst, const HostBatch& b, int ub) {
     auto* h = reinterpret_cast<BatchHeader*>(dst);
     std::memset(h, 0, sizeof(*h));
     auto* prefix = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(dst) + sizeof(BatchHeader));
-    uint32_t items = fill_prefix(prefix, b.descs, ub);
+    uint32_t items = fill_prefix(prefix, b, ub);
     size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
+    if (!b.gm.empty()) {
+        std::memcpy(reinterpret_cast<char*>(dst) + off, b.gm.data(), n * 4);
+        off += pad16(n * 4);
+    }
     h->ub = (uint32_t)ub;
-    h->blocked = item_order_blocked();
+    h->flags = batch_flags(b);
     h->nreq = (uint32_t)n;
     h->total_items = items;
     h->desc_offset = (uint32_t)off;
@@ -84,8 +144,9 @@ static void to_param(const HostBatch& b, Launchable& out) {
     auto* p = reinterpret_cast<ParamBatch<CAP>*>(out.blob.data());
     p->h.nreq = (uint32_t)b.descs.size();
     p->h.ub = (uint32_t)out.ub;
-    p->h.blocked = item_order_blocked();
-    p->h.total_items = fill_prefix(p->prefix, b.descs, out.ub);
+    p->h.flags = batch_flags(b);
+    p->h.total_items = fill_prefix(p->prefix, b, out.ub);
+    std::copy(b.gm.begin(), b.gm.end(), p->gm);
     std::copy(b.descs.begin(), b.descs.end(), p->descs);
     std::copy(b.aux.begin(), b.aux.end(), p->aux);
     std::copy(b.xinfo.begin(), b.xinfo.end(), p->xinfo);
@@ -126,7 +187,7 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
     } else {
         out.form = 3;
         std::vector<uint32_t> prefix(b.descs.size() + 1);
-        out.total_items = fill_prefix(prefix.data(), b.descs, out.ub);
+        out.total_items = fill_prefix(prefix.data(), b, out.ub);
     }
 }
 

@@ -126,7 +126,8 @@ inline uint32_t desc_items(const ReqDesc& d, int ub = kUnroll) {
 struct HostBatch {
     std::vector<ReqDesc> descs, aux;
     std::vector<XInfo> xinfo;
-    void clear() { descs.clear(); aux.clear(); xinfo.clear(); }
+    std::vector<uint32_t> gm;  // group size per request (empty: no groups), see device_desc.h
+    void clear() { descs.clear(); aux.clear(); xinfo.clear(); gm.clear(); }
     void add(ReqDesc s, const ReqDesc& d) {
         s.aux = (uint32_t)aux.size();
         aux.push_back(d);
@@ -148,6 +149,11 @@ uint32_t write_device_table(void* dst, const HostBatch& b, int ub);
 // Items per thread for a batch: the largest of {4, 2, 1} that still gives
 // >= 2 items per SM, so latency-bound batches use every SM.
 int choose_ub(const HostBatch& b, int sm_count);
+// Reorder the requests of b so that requests with equal item counts (at item
+// size ub) sit together in groups of at most max_m, and fill b.gm.  Requests only
+// move within maximal runs of consecutive requests of the same exchange class
+// (wait? / signal?), so the exchange kernel's item order stays deadlock-free.
+void group_equal_requests(HostBatch& b, int ub, int max_m = 8);
 // Param form if it fits (and allowed), else form 3 with `dev` left to the caller.
 // force_ub > 0 fixes the item size (exchange plans: sender and receiver chunk alike).
 void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count = 148, int force_ub = 0);

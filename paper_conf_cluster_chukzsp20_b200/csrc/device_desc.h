@@ -100,7 +100,14 @@ struct alignas(16) XInfo {
 constexpr int kXchgUb = 2;
 
 // Header of a device batch table:
-//   BatchHeader | uint32 prefix[nreq + 1] (16 B padded) | ReqDesc src[nreq] | ReqDesc dst[naux] | XInfo[nreq]?
+//   BatchHeader | uint32 prefix[nreq + 1] (16 B padded) | uint32 gm[nreq] (16 B padded, grouped only)
+//   | ReqDesc src[nreq] | ReqDesc dst[naux] | XInfo[nreq]?
+// Grouped batches: m consecutive requests with equal item counts n form one
+// group whose m*n items interleave chunk by chunk (item j of the group = chunk
+// j / m of member j % m), so the members' same-position chunks run at the same
+// time -- the +x / -x faces of a halo then touch each DRAM row together.  In
+// the prefix, a group's members all hold the group's first item (the binary
+// search lands on the last member) and gm[r] = m for every member.
 struct alignas(16) BatchHeader {
     uint32_t nreq;
     uint32_t total_items;
@@ -109,14 +116,16 @@ struct alignas(16) BatchHeader {
     uint32_t xinfo_offset;  // 0 = no exchange info
     uint32_t naux;
     uint32_t ub;            // vectors per thread per item (1, 2 or 4)
-    uint32_t blocked;       // item order: 0 = cyclic over CTAs, 1 = contiguous block per CTA
+    uint32_t flags;         // bit 0: blocked item order (else cyclic over CTAs); bit 1: grouped (gm[] present)
 };
+constexpr uint32_t kBatchBlocked = 1u, kBatchGrouped = 2u;
 
 // A small batch carried in the kernel parameters.
 template <int CAP>
 struct alignas(16) ParamBatch {
     BatchHeader h;                 // offsets unused
     uint32_t prefix[CAP + 4];
+    uint32_t gm[CAP];
     ReqDesc descs[CAP];
     ReqDesc aux[CAP];
     XInfo xinfo[CAP];

@@ -216,8 +216,9 @@ __device__ __forceinline__ uint32_t find_request(const uint32_t* prefix, uint32_
 }
 
 struct TableView {
-    uint32_t nreq, total, ub, blocked;
+    uint32_t nreq, total, ub, flags;
     const uint32_t* prefix;
+    const uint32_t* gm;       // group size per request (kBatchGrouped)
     const ReqDesc* descs;
     const ReqDesc* aux;
     const XInfo* xinfo;
@@ -229,8 +230,9 @@ __device__ __forceinline__ TableView view_of(const uint8_t* t) {
     v.nreq = h->nreq;
     v.total = h->total_items;
     v.ub = h->ub;
-    v.blocked = h->blocked;
+    v.flags = h->flags;
     v.prefix = reinterpret_cast<const uint32_t*>(t + sizeof(BatchHeader));
+    v.gm = reinterpret_cast<const uint32_t*>(t + sizeof(BatchHeader) + ((((size_t)h->nreq + 1) * 4 + 15) & ~(size_t)15));
     v.descs = reinterpret_cast<const ReqDesc*>(t + h->desc_offset);
     v.aux = reinterpret_cast<const ReqDesc*>(t + h->aux_offset);
     v.xinfo = h->xinfo_offset ? reinterpret_cast<const XInfo*>(t + h->xinfo_offset) : nullptr;
@@ -243,8 +245,9 @@ __device__ __forceinline__ TableView view_of(const ParamBatch<CAP>& p) {
     v.nreq = p.h.nreq;
     v.total = p.h.total_items;
     v.ub = p.h.ub;
-    v.blocked = p.h.blocked;
+    v.flags = p.h.flags;
     v.prefix = p.prefix;
+    v.gm = p.gm;
     v.descs = p.descs;
     v.aux = p.aux;
     v.xinfo = p.xinfo;
@@ -307,20 +310,28 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
     }
     constexpr int kWords = (int)(sizeof(ReqDesc) / 16);
     constexpr int kXWords = (int)(sizeof(XInfo) / 16);
-    uint32_t cur = 0xffffffffu, cur_first = 0;
+    uint32_t cur = 0xffffffffu;
     // cyclic (default): CTA b takes items b, b + grid, ... -- at any moment the
     // grid streams one contiguous window of each request (DRAM page locality);
     // blocked: CTA b owns [b*per, (b+1)*per) -- fewer descriptor reloads.
     // Both visit each CTA's items in increasing order (exchange deadlock freedom).
     uint32_t first = blockIdx.x, last = tv.total, step = gridDim.x;
-    if (tv.blocked) {
+    if (tv.flags & kBatchBlocked) {
         const uint32_t per = (tv.total + gridDim.x - 1) / gridDim.x;
         first = blockIdx.x * per;
         last = min(tv.total, first + per);
         step = 1;
     }
     for (uint32_t item = first; item < last; item += step) {
-        const uint32_t r = find_request(tv.prefix, tv.nreq, item);
+        uint32_t r = find_request(tv.prefix, tv.nreq, item);
+        uint32_t local = item - tv.prefix[r];  // the item's chunk index within its request
+        if (tv.flags & kBatchGrouped) {        // interleaved group: chunk local / m of member local % m
+            const uint32_t m = tv.gm[r];
+            if (m > 1) {
+                r = r + 1u - m + local % m;
+                local /= m;
+            }
+        }
         if (r != cur) {
             __syncthreads();  // every warp is done with the previous descriptor
             copy_words(&sd, tv.descs + r, kWords, 0);
@@ -337,10 +348,9 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
                     __syncthreads();
                 }
             }
-            cur_first = tv.prefix[r];
             cur = r;
         }
-        const uint32_t v0 = (item - cur_first) * (uint32_t)(kThreads * tv.ub);
+        const uint32_t v0 = local * (uint32_t)(kThreads * tv.ub);
         bool run = true;
         uint64_t tr0 = 0, tr1 = 0, tr2 = 0;
         if constexpr (XCHG) {
@@ -350,7 +360,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             if (sx.wait) {  // acquire: the peer's data / ready signal has arrived
                 if (threadIdx.x == 0) {
                     const uint64_t* flag = reinterpret_cast<const uint64_t*>(sx.wait) +
-                                           (sx.per_item ? (item - cur_first) : 0u);
+                                           (sx.per_item ? local : 0u);
                     int ok = 1;
                     const bool g = sx.gpu_scope != 0;  // the writer runs on this GPU
                     if ((g ? ld_acquire_gpu(flag) : ld_acquire_sys(flag)) < epoch) {
@@ -397,8 +407,8 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
                 if (threadIdx.x == 0) {
                     uint64_t* flag = reinterpret_cast<uint64_t*>(sx.signal);
                     if (sx.per_item) {
-                        if (sx.gpu_scope) st_release_gpu(flag + (item - cur_first), epoch);
-                        else st_release_sys(flag + (item - cur_first), epoch);
+                        if (sx.gpu_scope) st_release_gpu(flag + local, epoch);
+                        else st_release_sys(flag + local, epoch);
                     } else if (sx.nitems <= 1) {
                         __threadfence_system();
                         for (uint32_t k = 0; k < sx.fanout; k++) st_relaxed_sys(flag + k, epoch);

@@ -75,8 +75,13 @@ def _check(arrs, local, dirs, before=None):
     ((5, 6, 7), ALL_DIRS, 2, 4),
     ((9, 4, 3), FACE_DIRS, 1, 2),
 ])
-def test_halo_small(ddt, mode, graph, local, dirs, nvars, cfg):
+@pytest.mark.parametrize("group", [False, True])
+def test_halo_small(ddt, mode, graph, local, dirs, nvars, cfg, group, monkeypatch):
+    """group=True: equal-size requests interleaved chunk by chunk even though the
+    plan is one wave (the default only groups multi-wave plans)."""
     import torch
+    if group:
+        monkeypatch.setenv("DDT_GROUP_ALWAYS", "1")
     q, arrs, h, comm = _setup(ddt, local, dirs, nvars, mode, graph, cfg)
     for it in range(4):
         _fill_interior(arrs, local, it, cfg)

@@ -17,8 +17,10 @@ from mp_util import free_port, init  # noqa: E402
 pytestmark = pytest.mark.gpu
 
 
-def _worker(rank, world, port, dirs_name, iters, mode, q):
+def _worker(rank, world, port, dirs_name, iters, mode, q, group=False):
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    if group:  # interleave equal-size requests even in one-wave plans (halo.cpp make_table)
+        os.environ["DDT_GROUP_ALWAYS"] = "1"
     ok = False
     try:
         init(rank, world, port)
@@ -80,15 +82,18 @@ def _worker(rank, world, port, dirs_name, iters, mode, q):
 
 
 @pytest.mark.timeout(600)
-@pytest.mark.parametrize("world,dirs_name,iters,mode", [(2, "faces", 3, "p2p"), (2, "all", 4, "p2p"), (4, "all", 3, "p2p"),
-                                                       (8, "faces", 2, "p2p"), (2, "all", 4, "p2p_direct"),
-                                                       (4, "all", 3, "p2p_direct"), (8, "faces", 2, "p2p_direct")])
-def test_p2p_exchange_multiprocess_one_gpu(world, dirs_name, iters, mode):
+@pytest.mark.parametrize("world,dirs_name,iters,mode,group", [
+    (2, "faces", 3, "p2p", False), (2, "all", 4, "p2p", False), (4, "all", 3, "p2p", False),
+    (8, "faces", 2, "p2p", False), (2, "all", 4, "p2p_direct", False), (4, "all", 3, "p2p_direct", False),
+    (8, "faces", 2, "p2p_direct", False), (2, "all", 4, "p2p", True), (4, "all", 3, "p2p", True),
+    (4, "all", 3, "p2p_direct", True)])
+def test_p2p_exchange_multiprocess_one_gpu(world, dirs_name, iters, mode, group):
     import torch.multiprocessing as mp
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, dirs_name, iters, mode, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, dirs_name, iters, mode, q, group))
+             for r in range(world)]
     for p in procs:
         p.start()
     res = {}
