@@ -154,8 +154,12 @@ static void to_param(const HostBatch& b, Launchable& out) {
 }
 
 // The compact kernel variant applies when every source and destination
-// descriptor is closed-form (strided or contiguous) with one vector width.
+// descriptor is closed-form (strided or contiguous) with one vector width;
+// batches holding a general list take variant 6 (shared-memory windows).
 static int batch_variant(const HostBatch& b) {
+    for (const auto* v : {&b.descs, &b.aux})
+        for (const ReqDesc& d : *v)
+            if (d.nvec && d.kind == K_GENERAL) return 6;
     int lw = -1;
     for (const ReqDesc& d : b.descs)
         if (d.nvec) {

@@ -45,6 +45,7 @@ struct DeviceLayout {
     void* offsets = nullptr;  // u32 or i64
     void* lens = nullptr;     // i64 (general)
     void* prefix = nullptr;   // i64 (general)
+    void* skip = nullptr;     // u32 (general): segment holding packed byte i << kSkipShift
 };
 
 struct Layout {

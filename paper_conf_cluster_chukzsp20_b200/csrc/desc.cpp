@@ -123,7 +123,7 @@ static ddt_status_t layout_desc(ddt_type_s* t, const DeviceLayout* dl, const voi
         d->kind = K_GENERAL;
         d->vps = make_div((uint32_t)(t->size >> lw));  // vectors per instance
         d->list = (uint64_t)(uintptr_t)dl->offsets;
-        d->lens = (uint64_t)(uintptr_t)dl->lens;
+        d->skip = (uint64_t)(uintptr_t)dl->skip;
         d->prefix = (uint64_t)(uintptr_t)dl->prefix;
         d->list_n = (uint32_t)L.nseg;
     } else {

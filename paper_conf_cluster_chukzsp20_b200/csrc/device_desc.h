@@ -63,7 +63,7 @@ struct alignas(16) ReqDesc {
     DivU32 radix[kMaxDims]; // strided: dim sizes, innermost first
     int64_t stride[kMaxDims];
     uint64_t list;          // device pointer: offsets (u32 / i64) for lists
-    uint64_t lens;          // general: int64 lengths
+    uint64_t skip;          // general: u32 skip[i] = segment holding packed byte i << kSkipShift of an instance
     uint64_t prefix;        // general: int64 exclusive packed prefix (nseg + 1 entries)
     uint32_t list_n;        // general: number of segments per instance
     uint32_t uid_lo;        // low bits of the request UID (debug / tracing)
@@ -98,6 +98,16 @@ struct alignas(16) XInfo {
 // both sides, so a receiver's unpack item k depends only on the sender's pack
 // item k (per-chunk flags: unpack of a message overlaps its packing).
 constexpr int kXchgUb = 2;
+
+// General lists: a CTA work item stages the prefix / offset entries of the
+// segments it touches in shared memory (found through the skip table, whose
+// entry i is the segment holding packed byte i << kSkipShift of an instance)
+// and every thread finds its segment by a short shared-memory search -- the
+// north star's "warp-level segment lookup", at CTA level.  Windows of more
+// than kGenWin segments (byte-granular types) fall back to the per-vector
+// global search.
+constexpr int kSkipShift = 8;
+constexpr int kGenWin = 1280;
 
 // Header of a device batch table:
 //   BatchHeader | uint32 prefix[nreq + 1] (16 B padded) | uint32 gm[nreq] (16 B padded, grouped only)

@@ -171,24 +171,94 @@ __device__ __forceinline__ void ll_store(uint8_t* p, const uint4& d, uint32_t ep
                  "r"(epoch) : "memory");
 }
 
+// A general-list window: the prefix (relative to the window's first segment)
+// and offsets of the segments one work item touches (device_desc.h kGenWin).
+struct GenWin {
+    uint32_t rel_pre[kGenWin + 1];
+    long long off[kGenWin];
+};
+
+// Offset of vector v of instance k through a staged window (pre0 = absolute
+// packed position of the window's first segment).
+__device__ __forceinline__ int64_t gen_offset_win(const ReqDesc& d, uint32_t v, const GenWin& w, int64_t pre0,
+                                                  uint32_t cnt, int lw) {
+    const uint32_t k = divu(v, d.vps);
+    const int64_t pos = (int64_t)(v - k * d.vps.d) << lw;
+    const uint32_t rel = (uint32_t)(pos - pre0);
+    uint32_t lo = 0, hi = cnt;  // rel_pre[lo] <= rel < rel_pre[hi]
+    while (hi - lo > 1) {
+        const uint32_t mid = (lo + hi) >> 1;
+        if (w.rel_pre[mid] <= rel) lo = mid;
+        else hi = mid;
+    }
+    return (int64_t)k * d.extent + w.off[lo] + (int64_t)(rel - w.rel_pre[lo]);
+}
+
+// CTA-uniform: stage the window of general descriptor G for vectors [v0, vend)
+// (all in one instance, <= kGenWin segments) -> true; else false (fallback).
+__device__ __forceinline__ bool stage_gen_window(const ReqDesc& G, uint32_t v0, uint32_t vend, int lw, GenWin& w,
+                                                 int64_t& pre0, uint32_t& cnt) {
+    if (!G.skip || vend <= v0) return false;
+    const uint32_t vl = vend - 1;
+    const uint32_t k0 = divu(v0, G.vps), k1 = divu(vl, G.vps);
+    if (k0 != k1) return false;
+    const int64_t p0 = (int64_t)(v0 - k0 * G.vps.d) << lw;
+    const int64_t p1 = ((int64_t)(vl - k1 * G.vps.d) << lw) + ((1 << lw) - 1);
+    const int64_t inst_bytes = (int64_t)G.vps.d << lw;
+    const uint32_t last_i = (uint32_t)((inst_bytes + (1 << kSkipShift) - 1) >> kSkipShift);
+    const uint32_t i0 = (uint32_t)(p0 >> kSkipShift);
+    const uint32_t i1 = min((uint32_t)(p1 >> kSkipShift) + 1u, last_i);
+    const uint32_t* sk = reinterpret_cast<const uint32_t*>(G.skip);
+    const uint32_t seg0 = __ldg(sk + i0), seg1 = __ldg(sk + i1);
+    cnt = seg1 - seg0 + 1;
+    if (cnt > (uint32_t)kGenWin) return false;
+    const long long* pre = reinterpret_cast<const long long*>(G.prefix);
+    const long long* off = reinterpret_cast<const long long*>(G.list);
+    pre0 = __ldg(pre + seg0);
+    for (uint32_t j = threadIdx.x; j < cnt; j += kThreads) {
+        w.rel_pre[j] = (uint32_t)(__ldg(pre + seg0 + j) - pre0);
+        w.off[j] = __ldg(off + seg0 + j);
+    }
+    __syncthreads();
+    return true;
+}
+
 // One work item: up to kItemVecs vectors starting at v0, loaded through the
 // source descriptor S and stored through the destination descriptor D (one
 // code path for pack, unpack and DirectIPC).  coh: the source is written by
 // another GPU during this kernel (P2P window) -> L2-coherent loads instead of
 // the non-coherent read-only path.  XC: exchange kernel (LL windows possible).
-template <int LW, bool SONLY, bool XC>
+// Called by every thread of the CTA (general-list windows synchronise it).
+template <int LW, bool SONLY, bool XC, bool GW>
 __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uint32_t v0, bool coh, int ub,
                                          const XArgs* xa = nullptr, uint32_t epoch = 0) {
     const uint32_t nvec = S.nvec;
     const int lw = LW >= 0 ? LW : S.lw;
     const uint8_t* src = reinterpret_cast<const uint8_t*>(S.ptr);
     uint8_t* dst = reinterpret_cast<uint8_t*>(D.ptr);
+    // general lists: one side (the source if both) looks its segments up in a
+    // shared-memory window staged once per item
+    bool win_s = false, win_d = false;
+    int64_t pre0 = 0;
+    uint32_t cnt = 0;
+    GenWin* win = nullptr;
+    if constexpr (GW) {
+        __shared__ GenWin s_win;
+        win = &s_win;
+        if (S.kind == K_GENERAL || D.kind == K_GENERAL) {
+            const bool gs = S.kind == K_GENERAL;
+            const uint32_t vend = min(v0 + (uint32_t)(ub * kThreads), nvec);
+            const bool ok = stage_gen_window(gs ? S : D, v0, vend, lw, s_win, pre0, cnt);
+            win_s = ok && gs;
+            win_d = ok && !gs;
+        }
+    }
     uint4 buf[kUnroll];
 #pragma unroll
     for (int u = 0; u < kUnroll; u++) {
         uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
         if (u < ub && v < nvec) {
-            const uint8_t* p = src + vec_offset<LW, SONLY>(S, v);
+            const uint8_t* p = src + (win_s ? gen_offset_win(S, v, *win, pre0, cnt, lw) : vec_offset<LW, SONLY>(S, v));
             if (XC && S.kind == K_LL) buf[u] = ll_load(p, epoch, xa);
             else buf[u] = coh ? ld_vec<false, LW>(p, lw) : ld_vec<true, LW>(p, lw);
         }
@@ -197,11 +267,12 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
     for (int u = 0; u < kUnroll; u++) {
         uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
         if (u < ub && v < nvec) {
-            uint8_t* p = dst + vec_offset<LW, SONLY>(D, v);
+            uint8_t* p = dst + (win_d ? gen_offset_win(D, v, *win, pre0, cnt, lw) : vec_offset<LW, SONLY>(D, v));
             if (XC && D.kind == K_LL) ll_store(p, buf[u], epoch);
             else st_vec<LW>(p, lw, buf[u]);
         }
     }
+    if (win_s || win_d) __syncthreads();  // the next item may restage the window
 }
 
 // Largest r with prefix[r] <= item (prefix strictly increasing, prefix[0] = 0).
@@ -294,7 +365,7 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // items in increasing order, so a CTA only ever waits after finishing all of
 // its own pack items; with grid <= resident CTAs nothing waits on work that
 // cannot run (deadlock freedom without a global ticket).
-template <bool XCHG, int LW, bool SONLY>
+template <bool XCHG, int LW, bool SONLY, bool GW>
 __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa) {
     __shared__ ReqDesc sd;
     __shared__ ReqDesc sa;
@@ -382,7 +453,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             }
             if (trace && threadIdx.x == 0) tr1 = globaltimer();
         }
-        if (run) run_desc<LW, SONLY, XCHG>(sd, sa, v0, XCHG && sd.op == OP_UNPACK, (int)tv.ub, xa, (uint32_t)epoch);
+        if (run) run_desc<LW, SONLY, XCHG, GW>(sd, sa, v0, XCHG && sd.op == OP_UNPACK, (int)tv.ub, xa, (uint32_t)epoch);
         if constexpr (!XCHG) {
             if (sd.resp) {  // scheduler (3): the CTA finishing the request's last item signals it
                 __syncthreads();
@@ -443,29 +514,35 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
 // Kernel instances.  Variant V: 0 = generic (any kind, runtime width);
 // 1 + lw = closed-form strided layouts only, vector width 2^lw fixed at
 // compile time -- a compact kernel for halo plans and dense batches (a cold
-// SM fetches a few KB of code instead of the generic ~80 KB).
-template <int V> struct VarT { static constexpr int LW = V == 0 ? -1 : V - 1; static constexpr bool SONLY = V != 0; };
+// SM fetches a few KB of code instead of the generic ~80 KB); 6 = generic plus
+// shared-memory general-list windows (only batches holding a general list pay
+// its registers and shared memory).
+template <int V> struct VarT {
+    static constexpr int LW = (V == 0 || V == 6) ? -1 : V - 1;
+    static constexpr bool SONLY = V >= 1 && V <= 5;
+    static constexpr bool GW = V == 6;
+};
 
 template <int V>
 __global__ void __launch_bounds__(kThreads) ddt_fused_dev(const uint8_t* __restrict__ table) {
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY>(view_of(table), nullptr);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW>(view_of(table), nullptr);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY>(view_of(pb), nullptr);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW>(view_of(pb), nullptr);
 }
 
 template <int V>
 __global__ void __launch_bounds__(kThreads)
     ddt_exchange_dev(const uint8_t* __restrict__ table, const XArgs xa) {
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY>(view_of(table), &xa);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW>(view_of(table), &xa);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads)
     ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, const XArgs xa) {
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY>(view_of(pb), &xa);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW>(view_of(pb), &xa);
 }
 
 // ------------------------------------------------------------------ host side
@@ -540,6 +617,7 @@ int launch_fused_form(int form, int variant, const void* src, uint32_t total_ite
     case 3: launch_fused_v<3>(form, src, total_items, s, grid_cap); break;
     case 4: launch_fused_v<4>(form, src, total_items, s, grid_cap); break;
     case 5: launch_fused_v<5>(form, src, total_items, s, grid_cap); break;
+    case 6: launch_fused_v<6>(form, src, total_items, s, grid_cap); break;
     default: launch_fused_v<0>(form, src, total_items, s, grid_cap); break;
     }
     return (int)cudaGetLastError();
@@ -555,6 +633,7 @@ int launch_exchange_form(int form, int variant, const void* src, uint32_t total_
     case 3: launch_exchange_v<3>(form, src, total_items, xa, s, grid_cap); break;
     case 4: launch_exchange_v<4>(form, src, total_items, xa, s, grid_cap); break;
     case 5: launch_exchange_v<5>(form, src, total_items, xa, s, grid_cap); break;
+    case 6: launch_exchange_v<6>(form, src, total_items, xa, s, grid_cap); break;
     default: launch_exchange_v<0>(form, src, total_items, xa, s, grid_cap); break;
     }
     return (int)cudaGetLastError();

@@ -95,6 +95,7 @@ static void free_device_layouts(ddt_type_s* t) {
         cudaFree(kv.second.offsets);
         cudaFree(kv.second.lens);
         cudaFree(kv.second.prefix);
+        cudaFree(kv.second.skip);
     }
     if (cur >= 0) cudaSetDevice(cur);
 }
@@ -769,11 +770,24 @@ ddt_status_t type_device_layout(ddt_type_s* t, int device, DeviceLayout** out) {
             if (e == cudaSuccess) e = cudaMalloc(&dl.prefix, (n + 1) * 8);
             if (e == cudaSuccess)
                 e = cudaMemcpy(dl.prefix, L.prefix.data(), (n + 1) * 8, cudaMemcpyHostToDevice);
+            // skip[i] = segment holding packed byte i << kSkipShift (last entry: nseg - 1)
+            const int64_t bytes = L.prefix[n];
+            const size_t nskip = (size_t)((bytes + (1 << kSkipShift) - 1) >> kSkipShift) + 1;
+            std::vector<uint32_t> skip(nskip);
+            size_t j = 0;
+            for (size_t i = 0; i < nskip; i++) {
+                const int64_t pos = std::min<int64_t>((int64_t)i << kSkipShift, bytes - 1);
+                while (j + 1 < n && L.prefix[j + 1] <= pos) j++;
+                skip[i] = (uint32_t)j;
+            }
+            if (e == cudaSuccess) e = cudaMalloc(&dl.skip, nskip * 4);
+            if (e == cudaSuccess) e = cudaMemcpy(dl.skip, skip.data(), nskip * 4, cudaMemcpyHostToDevice);
         }
         if (e != cudaSuccess) {
             cudaFree(dl.offsets);
             cudaFree(dl.lens);
             cudaFree(dl.prefix);
+            cudaFree(dl.skip);
             return cuda_fail("layout cache upload", e);
         }
     }

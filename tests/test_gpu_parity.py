@@ -395,3 +395,54 @@ def test_milc_nested_vector(ddt, q, L):
     spec, fp = milc_spec(L)
     _run_case(ddt, q, Case(ddt, spec, 1, misalign=0, seed=L))
     _run_case(ddt, q, Case(ddt, spec, 2, misalign=8, seed=L + 1))
+
+
+def _irregular_hindexed(nblocks, npoints, base, maxlen, seed_, ones=False):
+    """hindexed with irregular block lengths (a GENERAL_LIST layout); ones=True:
+    mostly 1-element blocks of bytes (windows overflow -> per-vector fallback)."""
+    rng = np.random.default_rng(seed_)
+    esz = {"float": 4, "double": 8, "byte": 1}[base]
+    if ones:  # every other element at most: few merges, ~1 segment per byte packed
+        idx = 2 * np.sort(rng.choice(npoints // 2 - maxlen, nblocks, replace=False))
+    else:
+        idx = np.sort(rng.choice(npoints - maxlen, nblocks, replace=False))
+    lens = np.where(rng.random(nblocks) < 0.9, 1, 2) if ones else rng.integers(1, maxlen + 1, nblocks)
+    gaps = np.diff(np.append(idx, npoints))
+    lens = np.minimum(lens, gaps)
+    return ("hindexed", [int(x) for x in lens], [int(x) * esz for x in idx], ("basic", base))
+
+
+@pytest.mark.parametrize("spec,count,mis", [
+    (_irregular_hindexed(5000, 1 << 16, "float", 5, 1), 1, 0),
+    (_irregular_hindexed(5000, 1 << 16, "float", 5, 2), 2, 4),
+    (("indexed", [1, 3, 2, 5], [0, 4, 9, 20], ("basic", "double")), 200, 8),
+    (_irregular_hindexed(400000, 1 << 21, "byte", 2, 3, ones=True), 1, 1),
+    (_irregular_hindexed(3000, 1 << 15, "double", 7, 4), 3, 0),
+])
+def test_general_list_windows(ddt, q, spec, count, mis):
+    """GENERAL_LIST layouts: items whose segments fit a shared-memory window
+    (staged through the skip table), items spanning instances and byte-granular
+    windows that overflow (per-vector fallback) -- pack and unpack bit-exact."""
+    t = ddt.Type.from_spec(spec)
+    assert t.layout_kind == "general_list"
+    _run_case(ddt, q, Case(ddt, spec, count, misalign=mis, seed=count + mis))
+
+
+def test_general_list_direct_both_sides(ddt, q):
+    """DirectIPC general -> general (the source side uses the window, the
+    destination the per-vector lookup) == oracle unpack(pack(x))."""
+    import torch
+    ss = _irregular_hindexed(4000, 1 << 15, "float", 4, 5)
+    ds = _irregular_hindexed(4000, 1 << 15, "float", 4, 5)
+    os_, od = oracle.Type(ss), oracle.Type(ds)
+    ts, td = ddt.Type.from_spec(ss), ddt.Type.from_spec(ds)
+    _, shi = os_.footprint()
+    _, dhi = od.footprint()
+    src = random_bytes(shi + 64, 19)
+    s = cuda_bytes(src)
+    d = torch.full((dhi + 64,), SENTINEL, dtype=torch.uint8, device="cuda")
+    q.direct(ts, s, 1, td, d, 1)
+    q.wait()
+    exp = np.full(dhi + 64, SENTINEL, np.uint8)
+    oracle.unpack(od, oracle.pack(os_, src, 1, 0), exp, 1, 0)
+    assert_bytes_equal(host(d), exp, "direct general->general")

@@ -7,8 +7,8 @@ set -x
 OUT=gpurun_out/prof_r
 mkdir -p $OUT
 for m in nccl p2p; do
-  ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv --log-file $OUT/launches_cfg2_$m.csv \
-      python bench.py --steps 40 --warmup 5 --no-extras --mode $m > /dev/null 2>&1
+  ncu --metrics gpu__time_duration.sum --clock-control none -c 600 --csv --log-file $OUT/launches_cfg2_$m.csv \
+      python bench.py --steps 100 --warmup 5 --no-extras --mode $m > /dev/null 2>&1
 done
 ncu --set full --clock-control none --import-source on -k regex:ddt_ -s 10 -c 1 -o $OUT/full_cfg2 \
     python bench.py --steps 12 --warmup 3 --no-extras --mode nccl > /dev/null 2>&1
@@ -16,4 +16,8 @@ ncu --set full --clock-control none --import-source on -k regex:ddt_ -s 2 -c 1 -
     python tools/run_halo.py cfg4 nccl 4 > /dev/null 2>&1
 ncu --set full --clock-control none --import-source on -k regex:ddt_ -s 2 -c 1 -o $OUT/full_cfg5 \
     python tools/run_pack.py 4194304 64 4 > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on -k regex:ddt_ -s 2 -c 1 -o $OUT/full_cfg3 \
+    python tools/run_pack.py cfg3 32 4 > /dev/null 2>&1
+ncu --set full --clock-control none --import-source on -k regex:ddt_ -s 2 -c 1 -o $OUT/full_cfg3cm \
+    python tools/run_pack.py cfg3cm 32 4 > /dev/null 2>&1
 ls -la $OUT
