@@ -279,7 +279,9 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* comm, int32_t nsen
  * pack launch -> grouped send/recv -> fused unpack launch.  P2P modes: a
  * single launch.  ddt_halo_set_graph(h, 1) replays a CUDA graph captured on
  * first use -- except for P2P plans with remote messages, whose per-exchange
- * epoch travels as a kernel argument (always one direct launch).  All ranks
+ * epoch travels as a kernel argument (always one direct launch); for the same
+ * reason such a plan returns DDT_ERR_STATE when called while the caller
+ * captures the queue's stream (every other plan may be captured).  All ranks
  * must issue the same sequence of ddt_exchange calls.                        */
 ddt_status_t ddt_exchange(ddt_halo_t h);
 ddt_status_t ddt_halo_set_graph(ddt_halo_t h, int32_t use_graph);

@@ -55,7 +55,9 @@ struct RecvLayout {
     int64_t flags_bytes = 0, parity_stride = 0, window_bytes = 0;
 };
 
-RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs) {
+// reserve_ll: window space for the LL format (P2P window mode only; the NCCL
+// staging must not carry the gaps -- they would be transferred).
+RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs, bool reserve_ll = true) {
     RecvLayout L;
     L.order.resize((size_t)nrecv);
     for (int i = 0; i < nrecv; i++) L.order[(size_t)i] = i;
@@ -80,7 +82,7 @@ RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs) {
         L.flag_idx[(size_t)i] = (int)nflag;
         nflag += L.nflags[(size_t)i];
         // small messages of 8-B-capable layouts may travel in LL format (2x the bytes)
-        L.ll_ok[(size_t)i] = (lw >= 3 && bytes <= kLLMaxBytes && bytes % 8 == 0) ? 1 : 0;
+        L.ll_ok[(size_t)i] = (reserve_ll && lw >= 3 && bytes <= kLLMaxBytes && bytes % 8 == 0) ? 1 : 0;
         off += L.ll_ok[(size_t)i] ? 2 * bytes : bytes;
     }
     int64_t nready = 0;  // one slot per possible sender rank
@@ -487,7 +489,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     DevGuard g(h->device);
 
     // ---- receive layout and directories (receiver -> each sender)
-    RecvLayout RL = layout_recvs(nrecv, recvs);
+    RecvLayout RL = layout_recvs(nrecv, recvs, mode == DDT_XCHG_P2P);
     if (p2p && c->window_bytes < RL.window_bytes) {
         free_halo(h);
         set_error("window smaller than ddt_halo_window_bytes()");
@@ -933,6 +935,14 @@ ddt_status_t ddt_exchange(ddt_halo_t h) {
     DevGuard g(h->device);
     // a flagged P2P plan passes the epoch as a kernel argument: launched directly
     // (a captured graph would freeze it); every other plan may replay a graph
+    if (h->mode != DDT_XCHG_NCCL && h->x_flags && h->stream) {
+        cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+        if (cudaStreamIsCapturing(h->stream, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone) {
+            set_error("a P2P plan with remote messages cannot be captured into a CUDA graph (its epoch is a "
+                      "per-launch kernel argument): launch it directly or use DDT_XCHG_NCCL");
+            return DDT_ERR_STATE;
+        }
+    }
     if (h->use_graph && h->stream && !(h->mode != DDT_XCHG_NCCL && h->x_flags)) {
         if (!h->gexec) {
             cudaError_t e = cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal);
