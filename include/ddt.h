@@ -222,9 +222,11 @@ ddt_status_t ddt_queue_set_flush_threshold(ddt_queue_t q, int64_t bytes);
 ddt_status_t ddt_queue_set_response_flags(ddt_queue_t q, int32_t enable);
 
 /* Counters since queue creation: requests enqueued, fused kernel launches,
- * flushes, packed bytes moved (pack + unpack).                              */
+ * flushes, packed bytes moved (pack + unpack), and requests that moved as
+ * phased 16-B units (closed-form rows at 8 mod 16 on both sides, DESIGN.md
+ * "phased units"; introspection only).                                      */
 typedef struct {
-    int64_t requests, launches, flushes, bytes;
+    int64_t requests, launches, flushes, bytes, phased;
 } ddt_queue_stats_t;
 ddt_status_t ddt_queue_get_stats(ddt_queue_t q, ddt_queue_stats_t* out);
 

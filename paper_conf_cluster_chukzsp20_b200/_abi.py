@@ -44,7 +44,7 @@ class ddt_comm_t(ctypes.Structure):
 
 
 class ddt_queue_stats_t(ctypes.Structure):
-    _fields_ = [("requests", I64), ("launches", I64), ("flushes", I64), ("bytes", I64)]
+    _fields_ = [("requests", I64), ("launches", I64), ("flushes", I64), ("bytes", I64), ("phased", I64)]
 
 
 # name -> (restype, argtypes); the complete list of exported entry points

@@ -89,6 +89,66 @@ void group_equal_requests(HostBatch& b, int ub, int max_m) {
     b = std::move(out);
 }
 
+// Segment length (bytes) and phase (start address mod 16) of one closed-form
+// side at 8-B vectors; false if its segments do not all share one phase.
+// L = 0: contiguous side, segment length free (the other side's).
+static bool side_phase(const ReqDesc& d, uint64_t total, uint64_t& L, int& phase) {
+    if (d.kind == K_CONTIG) {
+        L = 0;
+        phase = (int)(d.ptr & 15);
+        return true;
+    }
+    L = (uint64_t)d.vps.d << 3;
+    if (L == 0 || total % L) return false;
+    phase = (int)((d.ptr + (uint64_t)d.base) & 15);
+    if (total / L > 1) {
+        for (int k = 0; k < d.ndim; k++)
+            if (d.stride[k] & 15) return false;
+        if (d.extent & 15) return false;
+    }
+    return true;
+}
+
+static bool try_phase(ReqDesc& S, ReqDesc& D) {
+    if (S.ph || D.ph || S.lw != 3 || D.lw != 3 || S.nvec == 0 || S.nvec != D.nvec) return false;
+    for (const ReqDesc* d : {&S, &D})
+        if (d->kind != K_STRIDED && d->kind != K_CONTIG) return false;
+    const uint64_t total = (uint64_t)S.nvec << 3;
+    uint64_t Ls, Ld;
+    int ps, pd;
+    if (!side_phase(S, total, Ls, ps) || !side_phase(D, total, Ld, pd) || ps != pd || (ps & 7)) return false;
+    if (Ls && Ld && Ls != Ld) return false;
+    const uint64_t L = Ls ? Ls : (Ld ? Ld : total);
+    const uint64_t nseg = total / L;
+    if (nseg > 1 && (L & 15) && (S.kind == K_CONTIG || D.kind == K_CONTIG)) return false;  // phase would flip
+    const uint64_t hd = ps == 8, tl = ((ps + L) & 15) == 8;
+    const uint64_t m = (L - 8 * hd - 8 * tl) / 16;
+    if (m < 2) return false;
+    const uint64_t U = hd + m + tl;
+    if (nseg * U >= (1ull << 32)) return false;
+    for (ReqDesc* d : {&S, &D}) {
+        d->ph = (uint8_t)(kPhOn | (hd ? kPhHead : 0) | (tl ? kPhTail : 0));
+        d->lw = 4;
+        d->vps = make_div((uint32_t)U);
+        d->nvec = (uint32_t)(nseg * U);
+    }
+    return true;
+}
+
+void phase_batch(HostBatch& b) {
+    const char* off = getenv("DDT_NO_PHASE");  // experiments: plain 8-B vectors
+    if (off && off[0] == '1') return;
+    for (const auto* v : {&b.descs, &b.aux})
+        for (const ReqDesc& d : *v)
+            if (d.nvec && d.kind != K_STRIDED && d.kind != K_CONTIG && d.kind != K_LL) return;
+    for (size_t i = 0; i < b.descs.size(); i++) {
+        if (!b.xinfo.empty() && (b.xinfo[i].signal || b.xinfo[i].wait)) continue;
+        ReqDesc& S = b.descs[i];
+        if (S.op == OP_SIGNAL) continue;
+        try_phase(S, b.aux[S.aux]);
+    }
+}
+
 size_t device_table_bytes(const HostBatch& b) {
     size_t n = b.descs.size();
     size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
@@ -160,6 +220,8 @@ static int batch_variant(const HostBatch& b) {
     for (const auto* v : {&b.descs, &b.aux})
         for (const ReqDesc& d : *v)
             if (d.nvec && d.kind == K_GENERAL) return 6;
+    for (const ReqDesc& d : b.descs)
+        if (d.ph) return 7;  // phase_batch only phases strided-only batches
     int lw = -1;
     for (const ReqDesc& d : b.descs)
         if (d.nvec) {

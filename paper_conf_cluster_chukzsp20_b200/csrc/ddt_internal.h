@@ -142,7 +142,7 @@ struct Launchable {
     std::vector<uint8_t> blob;  // ParamBatch<CAP> bytes (form 1 / 2)
     void* dev = nullptr;        // device table (form 3)
     uint32_t total_items = 0;
-    int variant = 0;            // 0 generic; 1 + lw: strided-only, one vector width
+    int variant = 0;            // 0 generic; 1 + lw: strided-only, one vector width; 6 general lists; 7 strided-only, phased units
     int ub = kUnroll;           // vectors per thread per item
 };
 size_t device_table_bytes(const HostBatch& b);
@@ -155,6 +155,12 @@ int choose_ub(const HostBatch& b, int sm_count);
 // move within maximal runs of consecutive requests of the same exchange class
 // (wait? / signal?), so the exchange kernel's item order stays deadlock-free.
 void group_equal_requests(HostBatch& b, int ub, int max_m = 8);
+// Re-cut eligible 8-B-wide closed-form requests into phased 16-B units
+// (device_desc.h kPh*).  Only batches whose every descriptor is closed-form
+// are touched (they launch the strided-only kernel variants); requests that
+// signal or wait (exchange flags, LL windows) keep their chunking.  Call before
+// choose_ub / group_equal_requests / make_launchable (item counts change).
+void phase_batch(HostBatch& b);
 // Param form if it fits (and allowed), else form 3 with `dev` left to the caller.
 // force_ub > 0 fixes the item size (exchange plans: sender and receiver chunk alike).
 void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count = 148, int force_ub = 0);

@@ -71,8 +71,17 @@ struct alignas(16) ReqDesc {
     uint32_t resp_val;      // value written to *resp when the request's last item is done
     uint64_t done_ctr;      // device u32 counter of finished items (reset by the finishing CTA)
     uint32_t nitems;        // items of this request in its batch (set at flush)
-    uint32_t pad3;
+    uint8_t ph;             // phased 16-B units (kPh*), 0 = plain vectors; see below
+    uint8_t pad3[3];
 };
+
+// Phased units (batch.cpp phase_batch).  A closed-form request whose common
+// width is 8 B only because its segments start at 8 mod 16 (halo rows begin at
+// x = 1) is re-cut per segment into [8-B head] [16-B body units] [8-B tail]
+// when both sides put every segment at the same phase mod 16: vector index v
+// -> segment s = v / vps, unit j = v % vps (vps = units per segment); the
+// body moves as 16-B accesses.  lw is 4, nvec counts units.
+constexpr uint8_t kPhOn = 1, kPhHead = 2, kPhTail = 4;
 
 // Exchange-only side info of a descriptor (fused P2P halo kernel).
 // Per item of request r:  [wait] -> move the data -> [signal].

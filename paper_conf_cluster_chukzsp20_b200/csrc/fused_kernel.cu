@@ -29,6 +29,10 @@
 
 #include "device_desc.h"
 
+#ifndef DDT_V7_MINB
+#define DDT_V7_MINB 4
+#endif
+
 namespace ddt {
 
 __device__ __forceinline__ uint32_t divu(uint32_t n, const DivU32& d) {
@@ -223,19 +227,89 @@ __device__ __forceinline__ bool stage_gen_window(const ReqDesc& G, uint32_t v0, 
     return true;
 }
 
+// Byte offset of segment s of a closed-form side (phased units, device_desc.h
+// kPh*): the strided dims of s, or s * L on the contiguous side.
+__device__ __forceinline__ int64_t seg_offset(const ReqDesc& d, uint32_t s) {
+    if (d.kind == K_CONTIG) {
+        const uint32_t hd = (d.ph >> 1) & 1u, tl = (d.ph >> 2) & 1u;
+        const int64_t L = 8 * (int64_t)(hd + tl) + 16 * (int64_t)(d.vps.d - hd - tl);
+        return (int64_t)s * L;
+    }
+    int64_t off = d.base;
+    const int nd = d.ndim;
+    for (int k = 0; k < nd; k++) {
+        uint32_t q = divu(s, d.radix[k]);
+        off += (int64_t)(s - q * d.radix[k].d) * d.stride[k];
+        s = q;
+    }
+    return off + (int64_t)s * d.extent;
+}
+
+// Phased request: unit v -> (segment, byte offset within it, 16-B or 8-B).
+__device__ __forceinline__ void phased_unit(const ReqDesc& S, uint32_t v, uint32_t& s, uint32_t& within,
+                                            bool& wide) {
+    s = divu(v, S.vps);
+    const uint32_t j = v - s * S.vps.d;
+    const uint32_t hd = (S.ph >> 1) & 1u, tl = (S.ph >> 2) & 1u;
+    const uint32_t m = S.vps.d - hd - tl;
+    if (hd && j == 0) {
+        within = 0;
+        wide = false;
+    } else if (j - hd < m) {
+        within = 8 * hd + 16 * (j - hd);
+        wide = true;
+    } else {
+        within = 8 * hd + 16 * m;  // the tail
+        wide = false;
+    }
+}
+
 // One work item: up to kItemVecs vectors starting at v0, loaded through the
 // source descriptor S and stored through the destination descriptor D (one
 // code path for pack, unpack and DirectIPC).  coh: the source is written by
 // another GPU during this kernel (P2P window) -> L2-coherent loads instead of
 // the non-coherent read-only path.  XC: exchange kernel (LL windows possible).
+// PH: phased 16-B units possible (variant 7).
 // Called by every thread of the CTA (general-list windows synchronise it).
-template <int LW, bool SONLY, bool XC, bool GW>
+template <int LW, bool SONLY, bool XC, bool GW, bool PH>
 __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uint32_t v0, bool coh, int ub,
                                          const XArgs* xa = nullptr, uint32_t epoch = 0) {
     const uint32_t nvec = S.nvec;
-    const int lw = LW >= 0 ? LW : S.lw;
     const uint8_t* src = reinterpret_cast<const uint8_t*>(S.ptr);
     uint8_t* dst = reinterpret_cast<uint8_t*>(D.ptr);
+    if constexpr (PH) {
+        if (S.ph) {  // both sides cut alike: one (segment, unit) split serves both
+            // the destination side's split is recomputed after the loads are
+            // issued (ALU work under the loads' latency, no live offsets)
+            uint4 buf[kUnroll];
+#pragma unroll
+            for (int u = 0; u < kUnroll; u++) {
+                const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+                if (u < ub && v < nvec) {
+                    uint32_t s, within;
+                    bool wide;
+                    phased_unit(S, v, s, within, wide);
+                    const uint8_t* p = src + seg_offset(S, s) + within;
+                    if (wide) buf[u] = coh ? ld_vec<false, 4>(p, 4) : ld_vec<true, 4>(p, 4);
+                    else buf[u] = coh ? ld_vec<false, 3>(p, 3) : ld_vec<true, 3>(p, 3);
+                }
+            }
+#pragma unroll
+            for (int u = 0; u < kUnroll; u++) {
+                const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+                if (u < ub && v < nvec) {
+                    uint32_t s, within;
+                    bool wide;
+                    phased_unit(S, v, s, within, wide);
+                    uint8_t* p = dst + seg_offset(D, s) + within;
+                    if (wide) st_vec<4>(p, 4, buf[u]);
+                    else st_vec<3>(p, 3, buf[u]);
+                }
+            }
+            return;
+        }
+    }
+    const int lw = LW >= 0 ? LW : S.lw;
     // general lists: one side (the source if both) looks its segments up in a
     // shared-memory window staged once per item
     bool win_s = false, win_d = false;
@@ -365,7 +439,7 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // items in increasing order, so a CTA only ever waits after finishing all of
 // its own pack items; with grid <= resident CTAs nothing waits on work that
 // cannot run (deadlock freedom without a global ticket).
-template <bool XCHG, int LW, bool SONLY, bool GW>
+template <bool XCHG, int LW, bool SONLY, bool GW, bool PH>
 __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa) {
     __shared__ ReqDesc sd;
     __shared__ ReqDesc sa;
@@ -453,7 +527,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             }
             if (trace && threadIdx.x == 0) tr1 = globaltimer();
         }
-        if (run) run_desc<LW, SONLY, XCHG, GW>(sd, sa, v0, XCHG && sd.op == OP_UNPACK, (int)tv.ub, xa, (uint32_t)epoch);
+        if (run) run_desc<LW, SONLY, XCHG, GW, PH>(sd, sa, v0, XCHG && sd.op == OP_UNPACK, (int)tv.ub, xa, (uint32_t)epoch);
         if constexpr (!XCHG) {
             if (sd.resp) {  // scheduler (3): the CTA finishing the request's last item signals it
                 __syncthreads();
@@ -516,33 +590,36 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
 // compile time -- a compact kernel for halo plans and dense batches (a cold
 // SM fetches a few KB of code instead of the generic ~80 KB); 6 = generic plus
 // shared-memory general-list windows (only batches holding a general list pay
-// its registers and shared memory).
+// its registers and shared memory); 7 = closed-form layouts, runtime width,
+// phased 16-B units (batch.cpp phase_batch).
 template <int V> struct VarT {
-    static constexpr int LW = (V == 0 || V == 6) ? -1 : V - 1;
-    static constexpr bool SONLY = V >= 1 && V <= 5;
+    static constexpr int LW = (V == 0 || V >= 6) ? -1 : V - 1;
+    static constexpr bool SONLY = (V >= 1 && V <= 5) || V == 7;
     static constexpr bool GW = V == 6;
+    static constexpr bool PH = V == 7;
+    static constexpr int MINB = V == 7 ? DDT_V7_MINB : 1;  // resident CTAs per SM the register budget must allow
 };
 
 template <int V>
-__global__ void __launch_bounds__(kThreads) ddt_fused_dev(const uint8_t* __restrict__ table) {
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW>(view_of(table), nullptr);
+__global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_dev(const uint8_t* __restrict__ table) {
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH>(view_of(table), nullptr);
 }
 
 template <int CAP, int V>
-__global__ void __launch_bounds__(kThreads) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW>(view_of(pb), nullptr);
+__global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH>(view_of(pb), nullptr);
 }
 
 template <int V>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads, VarT<V>::MINB)
     ddt_exchange_dev(const uint8_t* __restrict__ table, const XArgs xa) {
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW>(view_of(table), &xa);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH>(view_of(table), &xa);
 }
 
 template <int CAP, int V>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads, VarT<V>::MINB)
     ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, const XArgs xa) {
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW>(view_of(pb), &xa);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH>(view_of(pb), &xa);
 }
 
 // ------------------------------------------------------------------ host side
@@ -618,6 +695,7 @@ int launch_fused_form(int form, int variant, const void* src, uint32_t total_ite
     case 4: launch_fused_v<4>(form, src, total_items, s, grid_cap); break;
     case 5: launch_fused_v<5>(form, src, total_items, s, grid_cap); break;
     case 6: launch_fused_v<6>(form, src, total_items, s, grid_cap); break;
+    case 7: launch_fused_v<7>(form, src, total_items, s, grid_cap); break;
     default: launch_fused_v<0>(form, src, total_items, s, grid_cap); break;
     }
     return (int)cudaGetLastError();
@@ -634,6 +712,7 @@ int launch_exchange_form(int form, int variant, const void* src, uint32_t total_
     case 4: launch_exchange_v<4>(form, src, total_items, xa, s, grid_cap); break;
     case 5: launch_exchange_v<5>(form, src, total_items, xa, s, grid_cap); break;
     case 6: launch_exchange_v<6>(form, src, total_items, xa, s, grid_cap); break;
+    case 7: launch_exchange_v<7>(form, src, total_items, xa, s, grid_cap); break;
     default: launch_exchange_v<0>(form, src, total_items, xa, s, grid_cap); break;
     }
     return (int)cudaGetLastError();

@@ -180,6 +180,7 @@ ddt_status_t upload(const std::vector<uint8_t>& host, void** dev) {
 // otherwise run at different times (measured: COMB 139 -> 124 us; a one-wave
 // batch such as configs[1] only pays the extra lookup, 3.5 -> 3.75 us).
 ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub = 0) {
+    phase_batch(b);
     const int ub = force_ub > 0 ? force_ub : choose_ub(b, sm_count);
     uint64_t items = 0;
     for (const auto& d : b.descs) items += desc_items(d, ub);

@@ -213,6 +213,7 @@ int64_t gather_pending(ddt_queue_s* q) {
         b.add(r.desc, r.aux);
         moved += r.bytes;
     }
+    phase_batch(b);
     if (q->resp_on) {  // the finishing CTA compares its count with the request's item count
         int ub = choose_ub(b, q->sm_count);
         for (auto& d : b.descs) d.nitems = desc_items(d, ub);
@@ -369,6 +370,7 @@ int32_t ddt_flush(ddt_queue_t q) {
         if (le != 0) return q->sticky = cuda_fail("fused kernel launch", le);
         q->stats.launches++;
         q->stats.bytes += moved;
+        for (const ReqDesc& d : q->scratch.descs) q->stats.phased += d.ph ? 1 : 0;
     }
     ddt_queue_s::Batch b{q->flushed, q->tail, get_event(q)};
     cudaEventRecord(b.ev, q->stream);
@@ -454,6 +456,7 @@ ddt_status_t ddt_plan_create(ddt_queue_t q, ddt_plan_t* out) {
     }
     if (!q->scratch.descs.empty()) {
         make_launchable(q->scratch, true, p->launch, q->sm_count);
+        for (const ReqDesc& d : q->scratch.descs) q->stats.phased += d.ph ? 1 : 0;
         if (p->launch.form == 3) {
             std::vector<uint8_t> host(device_table_bytes(q->scratch));
             write_device_table(host.data(), q->scratch, p->launch.ub);

@@ -94,7 +94,8 @@ class Queue:
     def stats(self) -> dict:
         s = ddt_queue_stats_t()
         check(lib().ddt_queue_get_stats(self._h, ctypes.byref(s)), "ddt_queue_get_stats")
-        return {"requests": s.requests, "launches": s.launches, "flushes": s.flushes, "bytes": s.bytes}
+        return {"requests": s.requests, "launches": s.launches, "flushes": s.flushes, "bytes": s.bytes,
+                "phased": s.phased}
 
     def destroy(self):
         if self._h and self._h.value:
