@@ -29,6 +29,9 @@
 
 #include "device_desc.h"
 
+#ifndef DDT_INPLACE_PARAM
+#define DDT_INPLACE_PARAM true
+#endif
 #ifndef DDT_V7_MINB
 #define DDT_V7_MINB 4
 #endif
@@ -439,7 +442,11 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // items in increasing order, so a CTA only ever waits after finishing all of
 // its own pack items; with grid <= resident CTAs nothing waits on work that
 // cannot run (deadlock freedom without a global ticket).
-template <bool XCHG, int LW, bool SONLY, bool GW, bool PH>
+// INPLACE: the batch rides in the kernel parameters (constant bank): every
+// thread reads its request's descriptors in place (uniform constant loads),
+// with no shared-memory staging and no barrier before the first data load --
+// the latency-bound small-batch case (configs[1]: one item per CTA).
+template <bool XCHG, int LW, bool SONLY, bool GW, bool PH, bool INPLACE = false>
 __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa) {
     __shared__ ReqDesc sd;
     __shared__ ReqDesc sa;
@@ -477,7 +484,12 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
                 local /= m;
             }
         }
-        if (r != cur) {
+        const ReqDesc* S = &sd;  // this item's source / destination descriptors
+        const ReqDesc* D = &sa;
+        if constexpr (INPLACE && !XCHG) {
+            S = tv.descs + r;
+            D = tv.aux + r;  // aux[r], see HostBatch::add
+        } else if (r != cur) {
             __syncthreads();  // every warp is done with the previous descriptor
             copy_words(&sd, tv.descs + r, kWords, 0);
             if constexpr (XCHG) copy_words(&sx, tv.xinfo + r, kXWords, 32);
@@ -527,17 +539,17 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             }
             if (trace && threadIdx.x == 0) tr1 = globaltimer();
         }
-        if (run) run_desc<LW, SONLY, XCHG, GW, PH>(sd, sa, v0, XCHG && sd.op == OP_UNPACK, (int)tv.ub, xa, (uint32_t)epoch);
+        if (run) run_desc<LW, SONLY, XCHG, GW, PH>(*S, *D, v0, XCHG && S->op == OP_UNPACK, (int)tv.ub, xa, (uint32_t)epoch);
         if constexpr (!XCHG) {
-            if (sd.resp) {  // scheduler (3): the CTA finishing the request's last item signals it
+            if (S->resp) {  // scheduler (3): the CTA finishing the request's last item signals it
                 __syncthreads();
                 if (threadIdx.x == 0) {
                     __threadfence();
-                    unsigned int* ctr = reinterpret_cast<unsigned int*>(sd.done_ctr);
-                    if (atomicAdd(ctr, 1u) + 1u == sd.nitems) {
+                    unsigned int* ctr = reinterpret_cast<unsigned int*>(S->done_ctr);
+                    if (atomicAdd(ctr, 1u) + 1u == S->nitems) {
                         *ctr = 0u;
                         __threadfence_system();
-                        *reinterpret_cast<volatile unsigned int*>(sd.resp) = sd.resp_val;
+                        *reinterpret_cast<volatile unsigned int*>(S->resp) = S->resp_val;
                     }
                 }
             }
@@ -607,7 +619,7 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_dev(const u
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH>(view_of(pb), nullptr);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_PARAM>(view_of(pb), nullptr);
 }
 
 template <int V>
