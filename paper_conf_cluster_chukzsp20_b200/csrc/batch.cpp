@@ -149,12 +149,43 @@ void phase_batch(HostBatch& b) {
     }
 }
 
+bool spread_items(HostBatch& b, int ub) {
+    const size_t n = b.descs.size();
+    if (n < 2 || n > (1u << (32 - kSpreadShift))) return false;
+    for (const XInfo& x : b.xinfo)
+        if (x.signal || x.wait) return false;
+    for (const ReqDesc& d : b.descs)
+        if (d.kind == K_LL || d.op == OP_SIGNAL) return false;
+    std::vector<uint32_t> items(n);
+    uint64_t total = 0;
+    for (size_t r = 0; r < n; r++) {
+        items[r] = desc_items(b.descs[r], ub);
+        if (items[r] > (1u << kSpreadShift)) return false;
+        total += items[r];
+    }
+    // chunk c of request r at relative position (2c + 1) / (2 n_r); ties by r
+    struct E { uint32_t r, c; };
+    std::vector<E> e;
+    e.reserve(total);
+    for (size_t r = 0; r < n; r++)
+        for (uint32_t c = 0; c < items[r]; c++) e.push_back(E{(uint32_t)r, c});
+    std::stable_sort(e.begin(), e.end(), [&](const E& x, const E& y) {
+        const uint64_t a = (2ull * x.c + 1) * items[y.r], c = (2ull * y.c + 1) * items[x.r];
+        return a != c ? a < c : x.r < y.r;
+    });
+    b.gm.clear();
+    b.order.resize(total);
+    for (size_t i = 0; i < e.size(); i++) b.order[i] = (e[i].r << kSpreadShift) | e[i].c;
+    return true;
+}
+
 size_t device_table_bytes(const HostBatch& b) {
     size_t n = b.descs.size();
     size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
     if (!b.gm.empty()) off += pad16(n * 4);
     off += n * sizeof(ReqDesc) + b.aux.size() * sizeof(ReqDesc);
     if (!b.xinfo.empty()) off += n * sizeof(XInfo);
+    off += b.order.size() * 4;
     return off;
 }
 
@@ -194,6 +225,11 @@ uint32_t write_device_table(void* dst, const HostBatch& b, int ub) {
     if (!b.xinfo.empty()) {
         h->xinfo_offset = (uint32_t)off;
         std::memcpy(reinterpret_cast<char*>(dst) + off, b.xinfo.data(), n * sizeof(XInfo));
+        off += n * sizeof(XInfo);
+    }
+    if (!b.order.empty()) {
+        h->order_offset = (uint32_t)off;
+        std::memcpy(reinterpret_cast<char*>(dst) + off, b.order.data(), b.order.size() * 4);
     }
     return items;
 }

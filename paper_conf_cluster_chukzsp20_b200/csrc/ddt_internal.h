@@ -128,7 +128,8 @@ struct HostBatch {
     std::vector<ReqDesc> descs, aux;
     std::vector<XInfo> xinfo;
     std::vector<uint32_t> gm;  // group size per request (empty: no groups), see device_desc.h
-    void clear() { descs.clear(); aux.clear(); xinfo.clear(); gm.clear(); }
+    std::vector<uint32_t> order;  // explicit item table (empty: prefix search), see device_desc.h kSpreadShift
+    void clear() { descs.clear(); aux.clear(); xinfo.clear(); gm.clear(); order.clear(); }
     void add(ReqDesc s, const ReqDesc& d) {
         s.aux = (uint32_t)aux.size();
         aux.push_back(d);
@@ -161,6 +162,10 @@ void group_equal_requests(HostBatch& b, int ub, int max_m = 8);
 // signal or wait (exchange flags, LL windows) keep their chunking.  Call before
 // choose_ub / group_equal_requests / make_launchable (item counts change).
 void phase_batch(HostBatch& b);
+// Build b.order (device_desc.h kSpreadShift) for a non-exchange batch at item
+// size ub; false (b unchanged) if the batch has exchange flags or exceeds the
+// encoding (4096 requests, 2^20 items per request).
+bool spread_items(HostBatch& b, int ub);
 // Param form if it fits (and allowed), else form 3 with `dev` left to the caller.
 // force_ub > 0 fixes the item size (exchange plans: sender and receiver chunk alike).
 void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count = 148, int force_ub = 0);

@@ -136,8 +136,17 @@ struct alignas(16) BatchHeader {
     uint32_t naux;
     uint32_t ub;            // vectors per thread per item (1, 2 or 4)
     uint32_t flags;         // bit 0: blocked item order (else cyclic over CTAs); bit 1: grouped (gm[] present)
+    uint32_t order_offset;  // 0, or byte offset of the explicit item table (kBatchSpread)
+    uint32_t pad[3];
 };
 constexpr uint32_t kBatchBlocked = 1u, kBatchGrouped = 2u;
+// Spread batches (batch.cpp spread_items): an explicit item table order[item] =
+// (request << kSpreadShift) | chunk, ordered so that every request's chunks are
+// spread evenly over the whole launch (chunk c of a request of n items sits at
+// relative position (c + 1/2) / n): all requests progress together, so the
+// DRAM-activation-bound 8-B x-face cells overlap the bandwidth-bound dense
+// rows instead of following them.  Non-exchange batches only.
+constexpr int kSpreadShift = 20;
 
 // A small batch carried in the kernel parameters.
 template <int CAP>

@@ -370,6 +370,7 @@ struct TableView {
     const ReqDesc* descs;
     const ReqDesc* aux;
     const XInfo* xinfo;
+    const uint32_t* order;    // explicit item table (kBatchSpread), or null
 };
 
 __device__ __forceinline__ TableView view_of(const uint8_t* t) {
@@ -384,6 +385,7 @@ __device__ __forceinline__ TableView view_of(const uint8_t* t) {
     v.descs = reinterpret_cast<const ReqDesc*>(t + h->desc_offset);
     v.aux = reinterpret_cast<const ReqDesc*>(t + h->aux_offset);
     v.xinfo = h->xinfo_offset ? reinterpret_cast<const XInfo*>(t + h->xinfo_offset) : nullptr;
+    v.order = h->order_offset ? reinterpret_cast<const uint32_t*>(t + h->order_offset) : nullptr;
     return v;
 }
 
@@ -399,6 +401,7 @@ __device__ __forceinline__ TableView view_of(const ParamBatch<CAP>& p) {
     v.descs = p.descs;
     v.aux = p.aux;
     v.xinfo = p.xinfo;
+    v.order = nullptr;
     return v;
 }
 
@@ -475,9 +478,16 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         step = 1;
     }
     for (uint32_t item = first; item < last; item += step) {
-        uint32_t r = find_request(tv.prefix, tv.nreq, item);
-        uint32_t local = item - tv.prefix[r];  // the item's chunk index within its request
-        if (tv.flags & kBatchGrouped) {        // interleaved group: chunk local / m of member local % m
+        uint32_t r, local;  // the item's request and chunk index within it
+        if (tv.order) {     // spread batch: explicit item table
+            const uint32_t e = __ldg(tv.order + item);
+            r = e >> kSpreadShift;
+            local = e & ((1u << kSpreadShift) - 1u);
+        } else {
+            r = find_request(tv.prefix, tv.nreq, item);
+            local = item - tv.prefix[r];
+        }
+        if (!tv.order && (tv.flags & kBatchGrouped)) {  // interleaved group: chunk local / m of member local % m
             const uint32_t m = tv.gm[r];
             if (m > 1) {
                 r = r + 1u - m + local % m;

@@ -185,8 +185,12 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
     uint64_t items = 0;
     for (const auto& d : b.descs) items += desc_items(d, ub);
     const char* ga = getenv("DDT_GROUP_ALWAYS");  // tests: exercise grouping on small plans
-    if (items > 8ull * (uint64_t)sm_count || (ga && ga[0] == '1')) group_equal_requests(b, ub);
-    make_launchable(b, true, l, sm_count, ub);
+    const char* sp = getenv("DDT_SPREAD");  // 0: group equal requests instead of spreading every request
+    const bool many = items > 8ull * (uint64_t)sm_count;
+    bool spread = false;
+    if (many && !(sp && sp[0] == '0')) spread = spread_items(b, ub);
+    if (!spread && (many || (ga && ga[0] == '1'))) group_equal_requests(b, ub);
+    make_launchable(b, !spread, l, sm_count, ub);
     if (l.form != 3) return DDT_OK;
     std::vector<uint8_t> host(device_table_bytes(b));
     write_device_table(host.data(), b, l.ub);

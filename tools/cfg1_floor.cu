@@ -20,6 +20,10 @@ constexpr long long PLANE = (long long)N * N;
 __device__ __forceinline__ long long idx(int z, int y, int x) { return ((long long)z * N + y) * N + x; }
 
 __global__ void empty_k(double*) {}
+struct Big { unsigned char b[4000]; };
+__global__ void empty_big(double*, const __grid_constant__ Big p) { if (p.b[threadIdx.x & 7] == 255 && threadIdx.x == 1000) asm volatile("trap;"); }
+// faces8 with a 4-KB parameter block (the size of the library's ParamBatch<8>)
+__global__ void faces8_big(double* __restrict__ a, const __grid_constant__ Big p);
 
 // face f: 0: z=1 -> z=129, 1: z=128 -> z=0, 2: y=1 -> y=129, 3: y=128 -> y=0 (r = the other coordinate - 1)
 __device__ __forceinline__ void face_rows(int f, int r, long long& s, long long& d) {
@@ -58,6 +62,21 @@ __global__ void phased(double* __restrict__ a) {
         else *reinterpret_cast<uint4*>(pd + 16 * j) = __ldg(reinterpret_cast<const uint4*>(ps + 16 * j));
     } else if (t < 4 * 128 * U + 2 * 16384) {
         const int u = t - 4 * 128 * U, f = u / 16384, c = u % 16384, z = 1 + c / 128, y = 1 + c % 128;
+        if (f == 0) a[idx(z, y, 129)] = __ldg(a + idx(z, y, 1));
+        else a[idx(z, y, 0)] = __ldg(a + idx(z, y, 128));
+    }
+}
+
+__global__ void faces8_big(double* __restrict__ a, const __grid_constant__ Big p) {
+    if (p.b[0] == 255 && threadIdx.x == 1000) asm volatile("trap;");
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    if (t < 4 * 16384) {
+        const int f = t / 16384, i = t % 16384, r = i / 128, x = 1 + i % 128;
+        long long s, d;
+        face_rows(f, r, s, d);
+        a[d + x] = __ldg(a + s + x);
+    } else if (t < 6 * 16384) {
+        const int u = t - 4 * 16384, f = u / 16384, c = u % 16384, z = 1 + c / 128, y = 1 + c % 128;
         if (f == 0) a[idx(z, y, 129)] = __ldg(a + idx(z, y, 1));
         else a[idx(z, y, 0)] = __ldg(a + idx(z, y, 128));
     }
@@ -107,7 +126,12 @@ int main() {
     double te = graph_us([&](cudaStream_t s, int r) { empty_k<<<gp, 256, 0, s>>>(arr[r]); }, R, K);
     double t8 = graph_us([&](cudaStream_t s, int r) { faces8<<<g8, 256, 0, s>>>(arr[r]); }, R, K);
     double tp = graph_us([&](cudaStream_t s, int r) { phased<<<gp, 256, 0, s>>>(arr[r]); }, R, K);
+    Big big{};
+    double teb = graph_us([&](cudaStream_t s, int r) { empty_big<<<gp, 256, 0, s>>>(arr[r], big); }, R, K);
+    double t8b = graph_us([&](cudaStream_t s, int r) { faces8_big<<<g8, 256, 0, s>>>(arr[r], big); }, R, K);
     printf("{\"kernel\": \"empty\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gp, te);
+    printf("{\"kernel\": \"empty_4KB_params\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gp, teb);
+    printf("{\"kernel\": \"faces8_4KB_params\", \"ctas\": %d, \"us_per_step\": %.3f}\n", g8, t8b);
     printf("{\"kernel\": \"faces8\", \"ctas\": %d, \"us_per_step\": %.3f}\n", g8, t8);
     printf("{\"kernel\": \"phased\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gp, tp);
     cudaError_t e = cudaGetLastError();
