@@ -189,10 +189,32 @@ size_t device_table_bytes(const HostBatch& b) {
     return off;
 }
 
+// Variant 8: every descriptor moves 4-B vectors through a closed-form or
+// uniform-list layout, at least one side is a list (the sparse configs[2]
+// shape); items may then hold kUnrollNarrow vectors per thread.
+static bool narrow_list_batch(const HostBatch& b) {
+    const char* off = getenv("DDT_NO_NARROW");  // experiments
+    if (off && off[0] == '1') return false;
+    bool list = false;
+    for (const auto* v : {&b.descs, &b.aux})
+        for (const ReqDesc& d : *v) {
+            if (!d.nvec) continue;
+            if (d.lw != 2 || d.ph) return false;
+            if (d.kind == K_UNIFORM32 || d.kind == K_UNIFORM64) list = true;
+            else if (d.kind != K_STRIDED && d.kind != K_CONTIG) return false;
+        }
+    return list && b.xinfo.empty();
+}
+
 int choose_ub(const HostBatch& b, int sm_count) {
     const char* env = getenv("DDT_UB");
-    if (env && (atoi(env) == 1 || atoi(env) == 2 || atoi(env) == 4)) return atoi(env);
-    for (int ub : {4, 2}) {
+    if (env && (atoi(env) == 1 || atoi(env) == 2 || atoi(env) == 4 || atoi(env) == 8)) {
+        const int u = atoi(env);
+        return u == 8 && !narrow_list_batch(b) ? 4 : u;
+    }
+    const bool narrow = narrow_list_batch(b);
+    for (int ub : {8, 4, 2}) {
+        if (ub == 8 && !narrow) continue;
         uint64_t items = 0;
         for (const auto& d : b.descs) items += desc_items(d, ub);
         if (items >= 2ull * (uint64_t)sm_count) return ub;
@@ -258,6 +280,7 @@ static int batch_variant(const HostBatch& b) {
             if (d.nvec && d.kind == K_GENERAL) return 6;
     for (const ReqDesc& d : b.descs)
         if (d.ph) return 7;  // phase_batch only phases strided-only batches
+    if (narrow_list_batch(b)) return 8;
     int lw = -1;
     for (const ReqDesc& d : b.descs)
         if (d.nvec) {

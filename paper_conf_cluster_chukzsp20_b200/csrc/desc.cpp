@@ -14,6 +14,7 @@
 // pointers and (count > 1) the extent, so every device access is naturally
 // aligned and the two sides of a pair always share one width.
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 
 #include "ddt_internal.h"
@@ -47,6 +48,15 @@ int side_lw(ddt_type_s* t, const void* p, int64_t count) {
     int w = std::min(t->layout.align, lowbit16((uint64_t)(uintptr_t)p));
     if (count > 1) w = std::min(w, lowbit16(uabs64(type_extent(t))));
     return log2i(w);
+}
+
+// experiments: DDT_NO_L2HINT=1 disables the sparse-side prefetch-size hint
+static bool l2_hint_on() {
+    static const bool on = [] {
+        const char* e = getenv("DDT_NO_L2HINT");
+        return !(e && e[0] == '1');
+    }();
+    return on;
 }
 
 // Fill the layout fields of `d` for `count` instances of t at `base_ptr`.
@@ -96,6 +106,7 @@ static ddt_status_t layout_desc(ddt_type_s* t, const DeviceLayout* dl, const voi
         d->kind = K_STRIDED;
         d->base = L.form.base;
         d->vps = make_div((uint32_t)(seg >> lw));
+        d->l2_64 = (D > 0 && seg < kSparseSeg && l2_hint_on()) ? 1 : 0;
         if (D == 0) {
             if (d->base == 0) d->kind = K_CONTIG;  // one contiguous run at the pointer itself
             d->ndim = 0;
@@ -116,11 +127,13 @@ static ddt_status_t layout_desc(ddt_type_s* t, const DeviceLayout* dl, const voi
         }
     } else if (L.kind == DDT_LAYOUT_UNIFORM_LIST) {
         d->kind = L.off32 ? K_UNIFORM32 : K_UNIFORM64;
+        d->l2_64 = (L.seg_len < kSparseSeg && l2_hint_on()) ? 1 : 0;
         d->vps = make_div((uint32_t)(L.seg_len >> lw));
         d->nseg = make_div((uint32_t)L.nseg);
         d->list = (uint64_t)(uintptr_t)dl->offsets;
     } else if (L.kind == DDT_LAYOUT_GENERAL_LIST) {
         d->kind = K_GENERAL;
+        d->l2_64 = (L.nseg > 0 && t->size < kSparseSeg * L.nseg && l2_hint_on()) ? 1 : 0;  // mean segment shorter than kSparseSeg
         d->vps = make_div((uint32_t)(t->size >> lw));  // vectors per instance
         d->list = (uint64_t)(uintptr_t)dl->offsets;
         d->skip = (uint64_t)(uintptr_t)dl->skip;

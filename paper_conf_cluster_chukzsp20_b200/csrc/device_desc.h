@@ -22,6 +22,7 @@ constexpr int kMaxDims = 4;          // closed-form strided dims per layout (R7)
 constexpr int kThreads = 256;        // threads per CTA of the fused kernel
 constexpr int kUnroll = 4;           // max vectors per thread per item (loads in flight)
 constexpr int kItemVecs = kThreads * kUnroll;  // max vectors per work item
+constexpr int kUnrollNarrow = 8;     // 4-B-vector batches (variant 8): twice the loads in flight
 // A batch picks ub in {1, 2, 4} vectors per thread per item: small batches use
 // smaller items so that their work spreads over all 148 SMs (latency-bound
 // regime), large batches use kUnroll for memory-level parallelism.
@@ -72,7 +73,8 @@ struct alignas(16) ReqDesc {
     uint64_t done_ctr;      // device u32 counter of finished items (reset by the finishing CTA)
     uint32_t nitems;        // items of this request in its batch (set at flush)
     uint8_t ph;             // phased 16-B units (kPh*), 0 = plain vectors; see below
-    uint8_t pad3[3];
+    uint8_t l2_64;          // 1: short segments (< kSparseSeg B) -> loads carry the .L2::64B prefetch-size hint
+    uint8_t pad3[2];
 };
 
 // Phased units (batch.cpp phase_batch).  A closed-form request whose common
@@ -82,6 +84,12 @@ struct alignas(16) ReqDesc {
 // -> segment s = v / vps, unit j = v % vps (vps = units per segment); the
 // body moves as 16-B accesses.  lw is 4, nvec counts units.
 constexpr uint8_t kPhOn = 1, kPhHead = 2, kPhTail = 4;
+
+// Sparse sides: the L2 fetches 128 B per missed line by default; a side whose
+// contiguous segments are shorter than kSparseSeg bytes loads with the PTX
+// prefetch-size hint .L2::64B, which halves the DRAM over-fetch of scattered
+// cells (configs[2] 12-B blocks: tools/hint_probe.cu, 137 -> 100 us).
+constexpr int64_t kSparseSeg = 128;
 
 // Exchange-only side info of a descriptor (fused P2P halo kernel).
 // Per item of request r:  [wait] -> move the data -> [signal].

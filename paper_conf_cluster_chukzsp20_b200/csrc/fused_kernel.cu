@@ -32,6 +32,12 @@
 #ifndef DDT_INPLACE_PARAM
 #define DDT_INPLACE_PARAM true
 #endif
+#ifndef DDT_MINB
+#define DDT_MINB 1
+#endif
+#ifndef DDT_V8_MINB
+#define DDT_V8_MINB 6
+#endif
 #ifndef DDT_V7_MINB
 #define DDT_V7_MINB 4
 #endif
@@ -49,46 +55,50 @@ __device__ __forceinline__ uint32_t divu(uint32_t n, const DivU32& d) {
 // NC: read-only data for the kernel's lifetime -> non-coherent path, no L1
 // allocation.  !NC: data another agent writes during the kernel (P2P window)
 // -> ld.global.cg (L2, coherent).
+// L2_64: the .L2::64B prefetch-size hint (sparse sides, device_desc.h kSparseSeg).
+#define DDT_LD(NCQ, H, V, ...)                                                                    \
+    do {                                                                                          \
+        if (H) asm volatile("ld.global." NCQ ".L2::64B" V : __VA_ARGS__);                        \
+        else asm volatile("ld.global." NCQ V : __VA_ARGS__);                                      \
+    } while (0)
 template <bool NC, int LW>
-__device__ __forceinline__ uint4 ld_vec(const uint8_t* p, int lw_rt) {
+__device__ __forceinline__ uint4 ld_vec(const uint8_t* p, int lw_rt, bool h64 = false) {
     const int lw = LW >= 0 ? LW : lw_rt;  // compile-time width folds the switch
     uint4 r = make_uint4(0, 0, 0, 0);
     switch (lw) {
     case 4:
         if constexpr (NC)
-            asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
-                         : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+            DDT_LD("nc.L1::no_allocate", h64, ".v4.u32 {%0,%1,%2,%3}, [%4];", "=r"(r.x), "=r"(r.y), "=r"(r.z),
+                   "=r"(r.w) : "l"(p));
         else
-            asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];"
-                         : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+            DDT_LD("cg", h64, ".v4.u32 {%0,%1,%2,%3}, [%4];", "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
         break;
     case 3:
-        if constexpr (NC)
-            asm volatile("ld.global.nc.L1::no_allocate.v2.u32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
-        else
-            asm volatile("ld.global.cg.v2.u32 {%0,%1}, [%2];" : "=r"(r.x), "=r"(r.y) : "l"(p));
+        if constexpr (NC) DDT_LD("nc.L1::no_allocate", h64, ".v2.u32 {%0,%1}, [%2];", "=r"(r.x), "=r"(r.y) : "l"(p));
+        else DDT_LD("cg", h64, ".v2.u32 {%0,%1}, [%2];", "=r"(r.x), "=r"(r.y) : "l"(p));
         break;
     case 2:
-        if constexpr (NC) asm volatile("ld.global.nc.u32 %0, [%1];" : "=r"(r.x) : "l"(p));
-        else asm volatile("ld.global.cg.u32 %0, [%1];" : "=r"(r.x) : "l"(p));
+        if constexpr (NC) DDT_LD("nc", h64, ".u32 %0, [%1];", "=r"(r.x) : "l"(p));
+        else DDT_LD("cg", h64, ".u32 %0, [%1];", "=r"(r.x) : "l"(p));
         break;
     case 1: {
         unsigned short h;
-        if constexpr (NC) asm volatile("ld.global.nc.u16 %0, [%1];" : "=h"(h) : "l"(p));
-        else asm volatile("ld.global.cg.u16 %0, [%1];" : "=h"(h) : "l"(p));
+        if constexpr (NC) DDT_LD("nc", h64, ".u16 %0, [%1];", "=h"(h) : "l"(p));
+        else DDT_LD("cg", h64, ".u16 %0, [%1];", "=h"(h) : "l"(p));
         r.x = h;
         break;
     }
     default: {
         unsigned short h;
-        if constexpr (NC) asm volatile("ld.global.nc.u8 %0, [%1];" : "=h"(h) : "l"(p));
-        else asm volatile("ld.global.cg.u8 %0, [%1];" : "=h"(h) : "l"(p));
+        if constexpr (NC) DDT_LD("nc", h64, ".u8 %0, [%1];", "=h"(h) : "l"(p));
+        else DDT_LD("cg", h64, ".u8 %0, [%1];", "=h"(h) : "l"(p));
         r.x = h;
         break;
     }
     }
     return r;
 }
+#undef DDT_LD
 
 template <int LW>
 __device__ __forceinline__ void st_vec(uint8_t* p, int lw_rt, const uint4& r) {
@@ -274,7 +284,7 @@ __device__ __forceinline__ void phased_unit(const ReqDesc& S, uint32_t v, uint32
 // the non-coherent read-only path.  XC: exchange kernel (LL windows possible).
 // PH: phased 16-B units possible (variant 7).
 // Called by every thread of the CTA (general-list windows synchronise it).
-template <int LW, bool SONLY, bool XC, bool GW, bool PH>
+template <int LW, bool SONLY, bool XC, bool GW, bool PH, int UNR = kUnroll>
 __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uint32_t v0, bool coh, int ub,
                                          const XArgs* xa = nullptr, uint32_t epoch = 0) {
     const uint32_t nvec = S.nvec;
@@ -284,9 +294,9 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
         if (S.ph) {  // both sides cut alike: one (segment, unit) split serves both
             // the destination side's split is recomputed after the loads are
             // issued (ALU work under the loads' latency, no live offsets)
-            uint4 buf[kUnroll];
+            uint4 buf[UNR];
 #pragma unroll
-            for (int u = 0; u < kUnroll; u++) {
+            for (int u = 0; u < UNR; u++) {
                 const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
                 if (u < ub && v < nvec) {
                     uint32_t s, within;
@@ -298,7 +308,7 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
                 }
             }
 #pragma unroll
-            for (int u = 0; u < kUnroll; u++) {
+            for (int u = 0; u < UNR; u++) {
                 const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
                 if (u < ub && v < nvec) {
                     uint32_t s, within;
@@ -330,18 +340,19 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
             win_d = ok && !gs;
         }
     }
-    uint4 buf[kUnroll];
+    const bool h64 = S.l2_64 != 0;
+    uint4 buf[UNR];
 #pragma unroll
-    for (int u = 0; u < kUnroll; u++) {
+    for (int u = 0; u < UNR; u++) {
         uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
         if (u < ub && v < nvec) {
             const uint8_t* p = src + (win_s ? gen_offset_win(S, v, *win, pre0, cnt, lw) : vec_offset<LW, SONLY>(S, v));
             if (XC && S.kind == K_LL) buf[u] = ll_load(p, epoch, xa);
-            else buf[u] = coh ? ld_vec<false, LW>(p, lw) : ld_vec<true, LW>(p, lw);
+            else buf[u] = coh ? ld_vec<false, LW>(p, lw, h64) : ld_vec<true, LW>(p, lw, h64);
         }
     }
 #pragma unroll
-    for (int u = 0; u < kUnroll; u++) {
+    for (int u = 0; u < UNR; u++) {
         uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
         if (u < ub && v < nvec) {
             uint8_t* p = dst + (win_d ? gen_offset_win(D, v, *win, pre0, cnt, lw) : vec_offset<LW, SONLY>(D, v));
@@ -449,7 +460,7 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // thread reads its request's descriptors in place (uniform constant loads),
 // with no shared-memory staging and no barrier before the first data load --
 // the latency-bound small-batch case (configs[1]: one item per CTA).
-template <bool XCHG, int LW, bool SONLY, bool GW, bool PH, bool INPLACE = false>
+template <bool XCHG, int LW, bool SONLY, bool GW, bool PH, bool INPLACE = false, int UNR = kUnroll>
 __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa) {
     __shared__ ReqDesc sd;
     __shared__ ReqDesc sa;
@@ -549,7 +560,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             }
             if (trace && threadIdx.x == 0) tr1 = globaltimer();
         }
-        if (run) run_desc<LW, SONLY, XCHG, GW, PH>(*S, *D, v0, XCHG && S->op == OP_UNPACK, (int)tv.ub, xa, (uint32_t)epoch);
+        if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, (int)tv.ub, xa, (uint32_t)epoch);
         if constexpr (!XCHG) {
             if (S->resp) {  // scheduler (3): the CTA finishing the request's last item signals it
                 __syncthreads();
@@ -613,35 +624,41 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
 // SM fetches a few KB of code instead of the generic ~80 KB); 6 = generic plus
 // shared-memory general-list windows (only batches holding a general list pay
 // its registers and shared memory); 7 = closed-form layouts, runtime width,
-// phased 16-B units (batch.cpp phase_batch).
+// phased 16-B units (batch.cpp phase_batch); 8 = 4-B vectors, closed-form or
+// uniform-list layouts, kUnrollNarrow loads in flight per thread (sparse lists
+// such as configs[2] are latency x concurrency bound, not bandwidth bound).
 template <int V> struct VarT {
-    static constexpr int LW = (V == 0 || V >= 6) ? -1 : V - 1;
+    static constexpr int LW = (V == 0 || V == 6 || V == 7) ? -1 : (V == 8 ? 2 : V - 1);
+    static constexpr int UNR = V == 8 ? kUnrollNarrow : kUnroll;
     static constexpr bool SONLY = (V >= 1 && V <= 5) || V == 7;
     static constexpr bool GW = V == 6;
     static constexpr bool PH = V == 7;
-    static constexpr int MINB = V == 7 ? DDT_V7_MINB : 1;  // resident CTAs per SM the register budget must allow
+    // resident CTAs per SM the register budget must allow
+    static constexpr int MINB = V == 7 ? DDT_V7_MINB : (V == 8 ? DDT_V8_MINB : DDT_MINB);
 };
 
 template <int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_dev(const uint8_t* __restrict__ table) {
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH>(view_of(table), nullptr);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(table),
+                                                                                                  nullptr);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_PARAM>(view_of(pb), nullptr);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_PARAM, VarT<V>::UNR>(
+        view_of(pb), nullptr);
 }
 
 template <int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB)
     ddt_exchange_dev(const uint8_t* __restrict__ table, const XArgs xa) {
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH>(view_of(table), &xa);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(table), &xa);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB)
     ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, const XArgs xa) {
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH>(view_of(pb), &xa);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(pb), &xa);
 }
 
 // ------------------------------------------------------------------ host side
@@ -718,6 +735,7 @@ int launch_fused_form(int form, int variant, const void* src, uint32_t total_ite
     case 5: launch_fused_v<5>(form, src, total_items, s, grid_cap); break;
     case 6: launch_fused_v<6>(form, src, total_items, s, grid_cap); break;
     case 7: launch_fused_v<7>(form, src, total_items, s, grid_cap); break;
+    case 8: launch_fused_v<8>(form, src, total_items, s, grid_cap); break;
     default: launch_fused_v<0>(form, src, total_items, s, grid_cap); break;
     }
     return (int)cudaGetLastError();
@@ -735,6 +753,7 @@ int launch_exchange_form(int form, int variant, const void* src, uint32_t total_
     case 5: launch_exchange_v<5>(form, src, total_items, xa, s, grid_cap); break;
     case 6: launch_exchange_v<6>(form, src, total_items, xa, s, grid_cap); break;
     case 7: launch_exchange_v<7>(form, src, total_items, xa, s, grid_cap); break;
+    case 8: launch_exchange_v<8>(form, src, total_items, xa, s, grid_cap); break;
     default: launch_exchange_v<0>(form, src, total_items, xa, s, grid_cap); break;
     }
     return (int)cudaGetLastError();

@@ -182,3 +182,24 @@ def test_direct_head_or_tail_only(ddt, q, L, sstride, dstride, mis, phased):
     exp = np.full(dn, SENTINEL, np.uint8)
     oracle.unpack(do, oracle.pack(so, sbuf, 1, soff), exp, 1, doff)
     assert_bytes_equal(host(gd), exp, "direct head/tail")
+
+
+def test_narrow_list_batch_device_table(ddt):
+    """40 sparse 4-B-vector list requests in one flush: the device-table form of
+    the narrow-list variant (8 loads in flight per thread), pack then unpack."""
+    import torch
+    from ddt_inputs import config3_spec
+    q2 = ddt.Queue()
+    cases = [Case(ddt, config3_spec(nblocks=700, npoints=1 << 12, s=100 + i, shuffled=(i % 3 == 0))[0], 1 + i % 2,
+                  misalign=4 * (i % 4), seed=i, pk_misalign=4 * (i % 2)) for i in range(40)]
+    outs = [c.gpu_pack(q2) for c in cases]
+    assert q2.flush() == 40
+    ins = [c.gpu_unpack(q2) for c in cases]
+    assert q2.flush() == 40
+    q2.wait()
+    torch.cuda.synchronize()
+    for c, (_, _, dp), (_, _, du) in zip(cases, outs, ins):
+        assert_bytes_equal(host(dp), c.expect_pack(), "narrow pack")
+        assert_bytes_equal(host(du), c.expect_unpack(), "narrow unpack")
+    assert q2.stats()["launches"] == 2
+    q2.destroy()
