@@ -33,7 +33,10 @@
 #define DDT_INPLACE_PARAM true
 #endif
 #ifndef DDT_MINB
-#define DDT_MINB 1
+#define DDT_MINB 5
+#endif
+#ifndef DDT_XMINB
+#define DDT_XMINB 1
 #endif
 #ifndef DDT_V8_MINB
 #define DDT_V8_MINB 6
@@ -633,8 +636,13 @@ template <int V> struct VarT {
     static constexpr bool SONLY = (V >= 1 && V <= 5) || V == 7;
     static constexpr bool GW = V == 6;
     static constexpr bool PH = V == 7;
-    // resident CTAs per SM the register budget must allow
+    // resident CTAs per SM the register budget must allow.  Plain batches: 5
+    // (48 registers) -- a dense multi-request pack reloads its descriptor at
+    // almost every item and needs the extra CTAs to keep loads in flight
+    // (tools/pack_probe.py: 1 MiB x 1024 packs 4.74 -> 6.08 TB/s from 3 to 5
+    // CTAs/SM); exchange kernels (flags, tracing) keep their registers.
     static constexpr int MINB = V == 7 ? DDT_V7_MINB : (V == 8 ? DDT_V8_MINB : DDT_MINB);
+    static constexpr int XMINB = V == 7 ? DDT_V7_MINB : (V == 8 ? DDT_V8_MINB : DDT_XMINB);
 };
 
 template <int V>
@@ -650,13 +658,13 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const
 }
 
 template <int V>
-__global__ void __launch_bounds__(kThreads, VarT<V>::MINB)
+__global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_dev(const uint8_t* __restrict__ table, const XArgs xa) {
     fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(table), &xa);
 }
 
 template <int CAP, int V>
-__global__ void __launch_bounds__(kThreads, VarT<V>::MINB)
+__global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, const XArgs xa) {
     fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(pb), &xa);
 }
