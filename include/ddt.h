@@ -23,9 +23,15 @@
  *     ddt_last_error_message() describe them.
  *   - Ownership: the library owns type objects, device layout caches, request
  *     rings, descriptor tables, staging buffers, windows it allocates and halo
- *     plans.  The CALLER owns every data buffer (device pointers on the queue's
- *     device) and must keep it alive and unmodified until the request is
- *     COMPLETED (MPI non-blocking semantics).
+ *     plans.  The CALLER owns every data buffer and must keep it alive and
+ *     unmodified until the request is COMPLETED (MPI non-blocking semantics,
+ *     P:241).  A data buffer is device memory of the queue's device, a
+ *     peer-mapped device pointer, or PAGE-LOCKED HOST memory (cudaHostAlloc /
+ *     cudaHostRegister; unified addressing): the fused kernel then reads /
+ *     writes exactly the typemap's bytes over PCIe with no staging copy (the
+ *     zero-copy path; tests/test_gpu_hostmem.py).  Pageable host memory is not
+ *     accepted (the kernel would fault).  P2P / P2P_DIRECT halo plans need
+ *     device memory for the buffers they open through CUDA IPC.
  *   - Byte displacements are signed 64-bit and relative to the user pointer;
  *     the caller guarantees the whole footprint is inside its allocation
  *     (reading R4).
