@@ -159,6 +159,16 @@ __device__ __forceinline__ int64_t vec_offset(const ReqDesc& d, uint32_t v) {
     }
 }
 
+// Programmatic dependent launch (sm_90+): a plain fused kernel lets the next
+// PDL-launched kernel on its stream start as soon as all of its own CTAs are
+// resident (trigger at entry); that kernel's CTAs then do their prologue
+// (parameter-space descriptors, item -> request search, address arithmetic)
+// and block in griddepcontrol.wait until this grid has completed and its
+// memory is visible -- every dependency still holds, the launch latency and
+// prologue of step k+1 hide under step k.
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 __device__ __forceinline__ uint64_t globaltimer_ns() {
     uint64_t t;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -289,7 +299,7 @@ __device__ __forceinline__ void phased_unit(const ReqDesc& S, uint32_t v, uint32
 // Called by every thread of the CTA (general-list windows synchronise it).
 template <int LW, bool SONLY, bool XC, bool GW, bool PH, int UNR = kUnroll>
 __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uint32_t v0, bool coh, int ub,
-                                         const XArgs* xa = nullptr, uint32_t epoch = 0) {
+                                         const XArgs* xa = nullptr, uint32_t epoch = 0, bool pdlw = false) {
     const uint32_t nvec = S.nvec;
     const uint8_t* src = reinterpret_cast<const uint8_t*>(S.ptr);
     uint8_t* dst = reinterpret_cast<uint8_t*>(D.ptr);
@@ -298,16 +308,38 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
             // the destination side's split is recomputed after the loads are
             // issued (ALU work under the loads' latency, no live offsets)
             uint4 buf[UNR];
+            if (pdlw) {  // first item after a programmatic launch: addresses first, then wait, then load
+                const uint8_t* ps[UNR];
+                bool wd[UNR];
 #pragma unroll
-            for (int u = 0; u < UNR; u++) {
-                const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-                if (u < ub && v < nvec) {
-                    uint32_t s, within;
-                    bool wide;
-                    phased_unit(S, v, s, within, wide);
-                    const uint8_t* p = src + seg_offset(S, s) + within;
-                    if (wide) buf[u] = coh ? ld_vec<false, 4>(p, 4) : ld_vec<true, 4>(p, 4);
-                    else buf[u] = coh ? ld_vec<false, 3>(p, 3) : ld_vec<true, 3>(p, 3);
+                for (int u = 0; u < UNR; u++) {
+                    const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+                    uint32_t s = 0, within = 0;
+                    wd[u] = false;
+                    if (u < ub && v < nvec) phased_unit(S, v, s, within, wd[u]);
+                    ps[u] = src + seg_offset(S, s) + within;
+                }
+                pdl_wait();
+#pragma unroll
+                for (int u = 0; u < UNR; u++) {
+                    const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+                    if (u < ub && v < nvec) {
+                        if (wd[u]) buf[u] = coh ? ld_vec<false, 4>(ps[u], 4) : ld_vec<true, 4>(ps[u], 4);
+                        else buf[u] = coh ? ld_vec<false, 3>(ps[u], 3) : ld_vec<true, 3>(ps[u], 3);
+                    }
+                }
+            } else {
+#pragma unroll
+                for (int u = 0; u < UNR; u++) {
+                    const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+                    if (u < ub && v < nvec) {
+                        uint32_t s, within;
+                        bool wide;
+                        phased_unit(S, v, s, within, wide);
+                        const uint8_t* p = src + seg_offset(S, s) + within;
+                        if (wide) buf[u] = coh ? ld_vec<false, 4>(p, 4) : ld_vec<true, 4>(p, 4);
+                        else buf[u] = coh ? ld_vec<false, 3>(p, 3) : ld_vec<true, 3>(p, 3);
+                    }
                 }
             }
 #pragma unroll
@@ -335,6 +367,10 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
     if constexpr (GW) {
         __shared__ GenWin s_win;
         win = &s_win;
+        if (pdlw && (S.kind == K_GENERAL || D.kind == K_GENERAL)) {  // the window reads global memory
+            pdl_wait();
+            pdlw = false;
+        }
         if (S.kind == K_GENERAL || D.kind == K_GENERAL) {
             const bool gs = S.kind == K_GENERAL;
             const uint32_t vend = min(v0 + (uint32_t)(ub * kThreads), nvec);
@@ -345,13 +381,32 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
     }
     const bool h64 = S.l2_64 != 0;
     uint4 buf[UNR];
+    if (!XC && pdlw) {  // first item after a programmatic launch: addresses first, then wait, then load
+        // (list layouts read their offset tables: those are written at commit, never by a kernel)
+        const uint8_t* ps[UNR];
 #pragma unroll
-    for (int u = 0; u < UNR; u++) {
-        uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-        if (u < ub && v < nvec) {
-            const uint8_t* p = src + (win_s ? gen_offset_win(S, v, *win, pre0, cnt, lw) : vec_offset<LW, SONLY>(S, v));
-            if (XC && S.kind == K_LL) buf[u] = ll_load(p, epoch, xa);
-            else buf[u] = coh ? ld_vec<false, LW>(p, lw, h64) : ld_vec<true, LW>(p, lw, h64);
+        for (int u = 0; u < UNR; u++) {
+            const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+            ps[u] = src + ((u < ub && v < nvec) ? (win_s ? gen_offset_win(S, v, *win, pre0, cnt, lw)
+                                                         : vec_offset<LW, SONLY>(S, v))
+                                                : 0);
+        }
+        pdl_wait();
+#pragma unroll
+        for (int u = 0; u < UNR; u++) {
+            const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+            if (u < ub && v < nvec) buf[u] = coh ? ld_vec<false, LW>(ps[u], lw, h64) : ld_vec<true, LW>(ps[u], lw, h64);
+        }
+    } else {
+#pragma unroll
+        for (int u = 0; u < UNR; u++) {
+            uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+            if (u < ub && v < nvec) {
+                const uint8_t* p =
+                    src + (win_s ? gen_offset_win(S, v, *win, pre0, cnt, lw) : vec_offset<LW, SONLY>(S, v));
+                if (XC && S.kind == K_LL) buf[u] = ll_load(p, epoch, xa);
+                else buf[u] = coh ? ld_vec<false, LW>(p, lw, h64) : ld_vec<true, LW>(p, lw, h64);
+            }
         }
     }
 #pragma unroll
@@ -463,7 +518,11 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // thread reads its request's descriptors in place (uniform constant loads),
 // with no shared-memory staging and no barrier before the first data load --
 // the latency-bound small-batch case (configs[1]: one item per CTA).
-template <bool XCHG, int LW, bool SONLY, bool GW, bool PH, bool INPLACE = false, int UNR = kUnroll>
+// LAZYW: the kernel was launched with programmatic serialization and its
+// batch is in the parameters: wait for the preceding grid just before the
+// first global-memory access (the first item's data loads).
+template <bool XCHG, int LW, bool SONLY, bool GW, bool PH, bool INPLACE = false, int UNR = kUnroll,
+          bool LAZYW = false>
 __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa) {
     __shared__ ReqDesc sd;
     __shared__ ReqDesc sa;
@@ -480,6 +539,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
     constexpr int kWords = (int)(sizeof(ReqDesc) / 16);
     constexpr int kXWords = (int)(sizeof(XInfo) / 16);
     uint32_t cur = 0xffffffffu;
+    bool waited = !LAZYW;
     // cyclic (default): CTA b takes items b, b + grid, ... -- at any moment the
     // grid streams one contiguous window of each request (DRAM page locality);
     // blocked: CTA b owns [b*per, (b+1)*per) -- fewer descriptor reloads.
@@ -563,7 +623,9 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             }
             if (trace && threadIdx.x == 0) tr1 = globaltimer();
         }
-        if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, (int)tv.ub, xa, (uint32_t)epoch);
+        if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, (int)tv.ub, xa,
+                                                          (uint32_t)epoch, !waited);
+        waited = true;
         if constexpr (!XCHG) {
             if (S->resp) {  // scheduler (3): the CTA finishing the request's last item signals it
                 __syncthreads();
@@ -647,13 +709,16 @@ template <int V> struct VarT {
 
 template <int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_dev(const uint8_t* __restrict__ table) {
+    pdl_trigger();
+    pdl_wait();  // the table may come from a copy just before this launch
     fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(table),
                                                                                                   nullptr);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_PARAM, VarT<V>::UNR>(
+    pdl_trigger();
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_PARAM, VarT<V>::UNR, true>(
         view_of(pb), nullptr);
 }
 
@@ -695,20 +760,44 @@ static uint32_t grid_for(uint32_t total, int resident, int grid_cap) {
     return total < cap ? total : cap;
 }
 
+static bool pdl_enabled() {
+    static const bool on = [] {
+        const char* e = getenv("DDT_NO_PDL");  // experiments: plain stream serialisation
+        return !(e && e[0] == '1');
+    }();
+    return on;
+}
+
+// Plain fused kernels launch with programmatic stream serialisation (see
+// pdl_trigger / pdl_wait above).
+template <class Arg>
+static void launch_pdl(void (*k)(Arg), uint32_t grid, cudaStream_t s, const Arg& arg) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(kThreads);
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = pdl_enabled() ? 1 : 0;
+    cudaLaunchKernelEx(&cfg, k, arg);
+}
+
 template <int V>
 static void launch_fused_v(int form, const void* src, uint32_t total, cudaStream_t s, int grid_cap) {
     static int res[4] = {0, 0, 0, 0};
     if (form == 1) {
         if (!res[1]) res[1] = resident_ctas(ddt_fused_param<kParamSmall, V>);
-        ddt_fused_param<kParamSmall, V><<<grid_for(total, res[1], grid_cap), kThreads, 0, s>>>(
-            *reinterpret_cast<const ParamBatch<kParamSmall>*>(src));
+        launch_pdl(ddt_fused_param<kParamSmall, V>, grid_for(total, res[1], grid_cap), s,
+                   *reinterpret_cast<const ParamBatch<kParamSmall>*>(src));
     } else if (form == 2) {
         if (!res[2]) res[2] = resident_ctas(ddt_fused_param<kParamLarge, V>);
-        ddt_fused_param<kParamLarge, V><<<grid_for(total, res[2], grid_cap), kThreads, 0, s>>>(
-            *reinterpret_cast<const ParamBatch<kParamLarge>*>(src));
+        launch_pdl(ddt_fused_param<kParamLarge, V>, grid_for(total, res[2], grid_cap), s,
+                   *reinterpret_cast<const ParamBatch<kParamLarge>*>(src));
     } else {
         if (!res[3]) res[3] = resident_ctas(ddt_fused_dev<V>);
-        ddt_fused_dev<V><<<grid_for(total, res[3], grid_cap), kThreads, 0, s>>>(reinterpret_cast<const uint8_t*>(src));
+        launch_pdl(ddt_fused_dev<V>, grid_for(total, res[3], grid_cap), s, reinterpret_cast<const uint8_t*>(src));
     }
 }
 
