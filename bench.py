@@ -577,8 +577,9 @@ def main():
             # the single-exchange view: events around each step, L2 flushed before it
             per, _ = timed_steps(torch, wl, max(50, args.steps // 5), 3, flush_buf, dist_on, None)
             iso_ms = max_over_ranks(torch, sum(per) / len(per), dist_on)
-            results[mode] = dict(wl=wl, mean_ms=ms, iso_ms=iso_ms, iso_p50_ms=statistics.median(per), comm=c,
-                                 wall=wall)
+            qs = np.percentile(np.asarray(per), [10, 50, 90])
+            results[mode] = dict(wl=wl, mean_ms=ms, iso_ms=iso_ms, iso_p50_ms=float(qs[1]), iso_p10_ms=float(qs[0]),
+                                 iso_p90_ms=float(qs[2]), comm=c, wall=wall)
         except Exception as e:  # report, keep the other mode
             results[mode] = dict(error=f"{type(e).__name__}: {e}")
     ok = {m: r for m, r in results.items() if "error" not in r}
@@ -674,7 +675,9 @@ def main():
             "cpu_baseline": cpu,
             "modes": {m: ({"us_per_iter": round(r["mean_ms"] * 1e3, 3),
                            "isolated_flushed_us": round(r["iso_ms"] * 1e3, 3),
-                           "isolated_flushed_p50_us": round(r["iso_p50_ms"] * 1e3, 3)} if "error" not in r else r)
+                           "isolated_flushed_p10_us": round(r["iso_p10_ms"] * 1e3, 3),
+                           "isolated_flushed_p50_us": round(r["iso_p50_ms"] * 1e3, 3),
+                           "isolated_flushed_p90_us": round(r["iso_p90_ms"] * 1e3, 3)} if "error" not in r else r)
                       for m, r in results.items()},
             "bytes_per_rank_per_iter": wl.S,
         }

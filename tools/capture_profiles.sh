@@ -21,3 +21,13 @@ ncu --set full --clock-control none --import-source on -k regex:ddt_ -s 2 -c 1 -
 ncu --set full --clock-control none --import-source on -k regex:ddt_ -s 2 -c 1 -o $OUT/full_cfg3cm \
     python tools/run_pack.py cfg3cm 32 4 > /dev/null 2>&1
 ls -la $OUT
+# summarise on the box (the five full reports exceed gpurun's 64 MiB return
+# limit): raw pages + summaries come back, only the headline report is kept
+python tools/summarize_profiles.py $OUT r01 gpurun_out/prof_sum > gpurun_out/prof_sum.log 2>&1
+for r in $OUT/full_*.ncu-rep; do
+  ncu -i $r --page raw --csv > ${r%.ncu-rep}_raw.csv 2>/dev/null
+  ncu -i $r --page details --csv > ${r%.ncu-rep}_details.csv 2>/dev/null
+done
+ncu -i $OUT/full_cfg2.ncu-rep --page source --csv > $OUT/full_cfg2_source.csv 2>/dev/null
+rm -f $OUT/full_cfg3.ncu-rep $OUT/full_cfg3cm.ncu-rep $OUT/full_cfg4.ncu-rep $OUT/full_cfg5.ncu-rep
+du -sh $OUT gpurun_out

@@ -11,7 +11,8 @@ import sys
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 src = sys.argv[1] if len(sys.argv) > 1 else os.path.join(ROOT, "gpurun_out", "prof_r")
 rnd = sys.argv[2] if len(sys.argv) > 2 else "r01"
-dst = os.path.join(ROOT, "profiles", rnd)
+out_root = sys.argv[3] if len(sys.argv) > 3 else os.path.join(ROOT, "profiles")  # run on the box: gpurun_out/...
+dst = os.path.join(out_root, rnd)
 os.makedirs(dst, exist_ok=True)
 KEYS = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
         "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed", "sm__throughput.avg.pct_of_peak_sustained_elapsed",
@@ -67,6 +68,6 @@ for f in sorted(os.listdir(src)):
                  for k, v in agg.items()}
 json.dump({"full_captures": summary, "launch_lists": launch}, open(os.path.join(dst, "ncu_summary.json"), "w"),
           indent=1)
-json.dump(traffic, open(os.path.join(ROOT, "profiles", "ncu_traffic.json"), "w"), indent=1)
+json.dump(traffic, open(os.path.join(out_root, "ncu_traffic.json"), "w"), indent=1)
 print(json.dumps({"full_captures": {k: {kk: v[kk] for kk in ("kernel", "gpu__time_duration.sum", "dram_bytes_per_launch")}
                                     for k, v in summary.items()}, "launch_lists": launch}, indent=1))
