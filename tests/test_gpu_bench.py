@@ -1,0 +1,47 @@
+"""bench.py end to end on one GPU: the N = 1 line and the N = 2 code path
+(torchrun, 2 ranks time-sliced on cuda:0 through the test hooks
+DDT_BENCH_BACKEND=gloo / DDT_BENCH_SHARE_GPU=1 -- timings meaningless, the
+point is that every arm of the multi-rank path runs and rank 0 prints one
+contract line)."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _line(out: str) -> dict:
+    lines = [ln for ln in out.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, out[-3000:]
+    return json.loads(lines[0])
+
+
+def _check(d, n):
+    assert d["n_gpus"] == n and d["unit"] == "us/iter" and d["higher_is_better"] is False
+    assert d["value"] > 0 and d["gpu_launches"] >= d["steps"]
+    assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
+    assert "failed" not in d["e2e"]["flow"], d["e2e"]["flow"]
+    assert d["roofline"]["bound"] == "hbm" and 0 < d["roofline"]["frac"]
+
+
+def test_bench_n1():
+    r = subprocess.run([sys.executable, "bench.py", "--steps", "30", "--warmup", "3", "--no-extras"], cwd=ROOT,
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-3000:]
+    _check(_line(r.stdout), 1)
+
+
+def test_bench_n2_shared_gpu():
+    env = dict(os.environ, DDT_BENCH_BACKEND="gloo", DDT_BENCH_SHARE_GPU="1", DDT_BENCH_REPLICAS="4")
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+                        "--master-addr", "127.0.0.1", "--master-port", "29533", "bench.py", "--gpus", "2",
+                        "--steps", "10", "--warmup", "3", "--no-extras", "--mode", "p2p"],
+                       cwd=ROOT, capture_output=True, text=True, timeout=900, env=env)
+    assert r.returncode == 0, (r.stdout[-2000:], r.stderr[-3000:])
+    d = _line(r.stdout)
+    _check(d, 2)
+    assert d["config"]["mode"] == "p2p"
