@@ -179,6 +179,22 @@ ddt_status_t ddt_queue_destroy(ddt_queue_t q);
 int64_t ddt_pack_enqueue(ddt_queue_t q, ddt_type_t t, const void* src, int64_t count, void* dst_packed);
 int64_t ddt_unpack_enqueue(ddt_queue_t q, ddt_type_t t, const void* src_packed, int64_t count, void* dst);
 
+/* Bulk enqueue: n requests of one operation in one call (the loop of
+ * Alg 3 lines 3-6, without a per-request trip across the ABI --
+ * the per-call cost of a binding such as ctypes dwarfs the ~0.1 us enqueue).
+ *   op      DDT_OP_PACK (0) or DDT_OP_UNPACK (1);
+ *   types   [n] committed types;  srcs / dsts [n] buffers as for
+ *           ddt_pack_enqueue / ddt_unpack_enqueue;  counts [n];
+ *   uids_out [n] (may be NULL) receives each request's uid.
+ * Requests are appended in array order.  Returns k = the number enqueued
+ * (n on success); if k < n, request k failed with the negative status
+ * returned in uids_out[k] (if given) and requests k..n-1 were not enqueued
+ * -- on DDT_ERR_QUEUE_FULL the caller flushes and resubmits from k.
+ * A negative return (DDT_ERR_ARG) means nothing was enqueued.               */
+enum { DDT_OP_PACK = 0, DDT_OP_UNPACK = 1 };
+int64_t ddt_enqueue_many(ddt_queue_t q, int32_t op, int64_t n, const ddt_type_t* types, const void* const* srcs,
+                         const int64_t* counts, void* const* dsts, int64_t* uids_out);
+
 /* DirectIPC request ("a direct non-contiguous data transfer", fused with
  * packing / unpacking in one kernel): gather `src_count` instances of
  * `src_type` at `src` and scatter them as `dst_count` instances of `dst_type`

@@ -74,6 +74,7 @@ PROTOTYPES = {
     "ddt_pack_enqueue": (I64, [P, P, P, I64, P]),
     "ddt_unpack_enqueue": (I64, [P, P, P, I64, P]),
     "ddt_direct_enqueue": (I64, [P, P, P, I64, P, P, I64]),
+    "ddt_enqueue_many": (I64, [P, I32, I64, P, P, P, P, P]),
     "ddt_flush": (I32, [P]),
     "ddt_query": (I32, [P, I64, I32P]),
     "ddt_wait": (I32, [P]),

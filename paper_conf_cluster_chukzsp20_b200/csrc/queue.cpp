@@ -309,6 +309,19 @@ int64_t ddt_unpack_enqueue(ddt_queue_t q, ddt_type_t t, const void* src_packed, 
     return enqueue(q, OP_UNPACK, t, src_packed, count, dst);
 }
 
+int64_t ddt_enqueue_many(ddt_queue_t q, int32_t op, int64_t n, const ddt_type_t* types, const void* const* srcs,
+                         const int64_t* counts, void* const* dsts, int64_t* uids_out) {
+    if (!q || n < 0 || (op != DDT_OP_PACK && op != DDT_OP_UNPACK)) return DDT_ERR_ARG;
+    if (n > 0 && (!types || !srcs || !counts || !dsts)) return DDT_ERR_ARG;
+    const int dop = op == DDT_OP_PACK ? OP_PACK : OP_UNPACK;
+    for (int64_t i = 0; i < n; i++) {
+        const int64_t uid = enqueue(q, dop, types[i], srcs[i], counts[i], dsts[i]);
+        if (uids_out) uids_out[i] = uid;
+        if (uid < 0) return i;
+    }
+    return n;
+}
+
 int64_t ddt_direct_enqueue(ddt_queue_t q, ddt_type_t src_type, const void* src, int64_t src_count,
                            ddt_type_t dst_type, void* dst, int64_t dst_count) {
     if (!q || !src_type || !dst_type || src_count < 0 || dst_count < 0) return DDT_ERR_ARG;

@@ -64,6 +64,42 @@ class Queue:
                                               dst_type.handle, ctypes.c_void_p(ptr_of(dst)), int(dst_count)),
                      "ddt_direct_enqueue")
 
+    def enqueue_many(self, op: str, types, srcs, counts, dsts):
+        """Bulk enqueue (ddt_enqueue_many): op 'pack' | 'unpack'; types a Type or
+        a sequence of n Types; srcs / dsts sequences of n buffers; counts an int
+        or n ints.  Returns the uids (numpy int64).  Raises on the first failed
+        request (requests before it stay enqueued); try_enqueue_many reports it."""
+        k, uids = self.try_enqueue_many(op, types, srcs, counts, dsts)
+        if k < len(uids):
+            check(int(uids[k]), f"ddt_enqueue_many (request {k})")
+        return uids
+
+    def try_enqueue_many(self, op: str, types, srcs, counts, dsts):
+        """Like enqueue_many but returns (k, uids): k requests were enqueued; if
+        k < n, uids[k] is request k's negative status (e.g. -3 = queue full:
+        flush and resubmit from k, P:215)."""
+        import numpy as np
+        n = len(srcs)
+        tys = np.asarray([t.handle.value for t in types] if isinstance(types, (list, tuple))
+                         else [types.handle.value] * n, dtype=np.uint64)
+        s = np.asarray([ptr_of(b) for b in srcs], dtype=np.uint64)
+        d = np.asarray([ptr_of(b) for b in dsts], dtype=np.uint64)
+        c = np.asarray(counts if isinstance(counts, (list, tuple, np.ndarray)) else [counts] * n, dtype=np.int64)
+        return self.enqueue_many_raw(0 if op == "pack" else 1, tys, s, c, d)
+
+    def enqueue_many_raw(self, op: int, tys, srcs, counts, dsts):
+        """ddt_enqueue_many over prepared numpy arrays (uint64 handles / pointers,
+        int64 counts): one call across the ABI for the whole batch.  Returns
+        (k, uids) as try_enqueue_many."""
+        import numpy as np
+        n = len(srcs)
+        uids = np.empty(n, dtype=np.int64)
+        k = self._lib.ddt_enqueue_many(self._h, int(op), n, tys.ctypes.data, srcs.ctypes.data, counts.ctypes.data,
+                                       dsts.ctypes.data, uids.ctypes.data)
+        if k < 0:
+            check(k, "ddt_enqueue_many")
+        return int(k), uids
+
     def try_pack(self, t, src, count, dst_packed) -> int:
         """Like pack() but returns the negative status instead of raising."""
         return lib().ddt_pack_enqueue(self._h, t.handle, ctypes.c_void_p(ptr_of(src)), int(count),

@@ -197,6 +197,43 @@ def test_queue_full_gives_negative_uid_then_recovers(ddt):
     q4.destroy()
 
 
+def test_enqueue_many_equals_oracle_and_stops_at_full_ring(ddt):
+    """ddt_enqueue_many: 40 mixed-type packs in one call, then 40 unpacks, two
+    launches, bit-exact vs the oracle; on a ring of 24 the bulk call stops at
+    the first DDT_ERR_QUEUE_FULL (returned for that request), the caller
+    flushes and resubmits the rest."""
+    import torch
+    specs = [config1_spec(), ("subarray", [9, 10, 11], [3, 4, 5], [1, 2, 3], "C", ("basic", "double")),
+             ("hindexed", [3, 1, 2], [100, 4, 37], ("basic", "byte")), ("vector", 5, 3, -4, ("basic", "int64"))]
+    cases = [Case(ddt, specs[i % len(specs)], count=1 + i % 3, misalign=i % 16, seed=500 + i) for i in range(40)]
+    srcs = [cuda_bytes(c.src) for c in cases]
+    pks = [torch.full((c.psize + 32,), SENTINEL, dtype=torch.uint8, device="cuda") for c in cases]
+    psrcs = [cuda_bytes(c.packed_src) for c in cases]
+    uns = [torch.full((c.nbytes,), SENTINEL, dtype=torch.uint8, device="cuda") for c in cases]
+    for cap in (0, 24):
+        qq = ddt.Queue(capacity=cap)
+        for p in pks:
+            p.fill_(SENTINEL)
+        for u in uns:
+            u.fill_(SENTINEL)
+        for op, ins, outs in (("pack", [(s, c.off) for s, c in zip(srcs, cases)], [(p, c.pk_off) for p, c in zip(pks, cases)]),
+                              ("unpack", [(s, c.pk_off) for s, c in zip(psrcs, cases)], [(u, c.off) for u, c in zip(uns, cases)])):
+            k0, partial = 0, 0
+            while k0 < len(cases):
+                k, uids = qq.try_enqueue_many(op, [c.t for c in cases[k0:]], ins[k0:],
+                                              [c.count for c in cases[k0:]], outs[k0:])
+                if k0 + k < len(cases):
+                    assert cap and uids[k] == -3, (k, uids[k])  # DDT_ERR_QUEUE_FULL for request k
+                    partial += 1
+                k0 += k
+                qq.wait()  # flush + completion frees the ring
+            assert partial == (0 if not cap else (len(cases) - 1) // cap)
+        for i, c in enumerate(cases):
+            assert_bytes_equal(host(pks[i]), c.expect_pack(), f"enqueue_many pack {i} cap={cap}")
+            assert_bytes_equal(host(uns[i]), c.expect_unpack(), f"enqueue_many unpack {i} cap={cap}")
+        qq.destroy()
+
+
 def test_zero_size_and_empty_requests(ddt, q):
     import torch
     t = ddt.Type.from_spec(("vector", 0, 3, 2, ("basic", "double")))
