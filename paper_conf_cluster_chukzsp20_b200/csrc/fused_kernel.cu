@@ -725,12 +725,16 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const
 template <int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_dev(const uint8_t* __restrict__ table, const XArgs xa) {
+    pdl_trigger();
+    pdl_wait();  // before any table read, flag or data access
     fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(table), &xa);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, const XArgs xa) {
+    pdl_trigger();
+    pdl_wait();
     fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(pb), &xa);
 }
 
@@ -770,8 +774,8 @@ static bool pdl_enabled() {
 
 // Plain fused kernels launch with programmatic stream serialisation (see
 // pdl_trigger / pdl_wait above).
-template <class Arg>
-static void launch_pdl(void (*k)(Arg), uint32_t grid, cudaStream_t s, const Arg& arg) {
+template <class... Args>
+static void launch_pdl(void (*k)(Args...), uint32_t grid, cudaStream_t s, const Args&... args) {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
     cfg.blockDim = dim3(kThreads);
@@ -781,7 +785,7 @@ static void launch_pdl(void (*k)(Arg), uint32_t grid, cudaStream_t s, const Arg&
     at[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     cfg.numAttrs = pdl_enabled() ? 1 : 0;
-    cudaLaunchKernelEx(&cfg, k, arg);
+    cudaLaunchKernelEx(&cfg, k, args...);
 }
 
 template <int V>
@@ -805,18 +809,23 @@ template <int V>
 static void launch_exchange_v(int form, const void* src, uint32_t total, const XArgs& xa, cudaStream_t s,
                               int grid_cap) {
     static int res[4] = {0, 0, 0, 0};
+    // programmatic serialisation: the launch overlaps the previous kernel's
+    // tail; every CTA waits (griddepcontrol.wait) before its first table, flag
+    // or data access, and all of this grid's CTAs are resident before the next
+    // PDL grid can be scheduled, so the co-residency argument for the flag
+    // waits (grid <= resident CTAs) is unchanged
     if (form == 1) {
         if (!res[1]) res[1] = resident_ctas(ddt_exchange_param<kParamSmall, V>);
-        ddt_exchange_param<kParamSmall, V><<<grid_for(total, res[1], grid_cap), kThreads, 0, s>>>(
-            *reinterpret_cast<const ParamBatch<kParamSmall>*>(src), xa);
+        launch_pdl(ddt_exchange_param<kParamSmall, V>, grid_for(total, res[1], grid_cap), s,
+                   *reinterpret_cast<const ParamBatch<kParamSmall>*>(src), xa);
     } else if (form == 2) {
         if (!res[2]) res[2] = resident_ctas(ddt_exchange_param<kParamLarge, V>);
-        ddt_exchange_param<kParamLarge, V><<<grid_for(total, res[2], grid_cap), kThreads, 0, s>>>(
-            *reinterpret_cast<const ParamBatch<kParamLarge>*>(src), xa);
+        launch_pdl(ddt_exchange_param<kParamLarge, V>, grid_for(total, res[2], grid_cap), s,
+                   *reinterpret_cast<const ParamBatch<kParamLarge>*>(src), xa);
     } else {
         if (!res[3]) res[3] = resident_ctas(ddt_exchange_dev<V>);
-        ddt_exchange_dev<V><<<grid_for(total, res[3], grid_cap), kThreads, 0, s>>>(
-            reinterpret_cast<const uint8_t*>(src), xa);
+        launch_pdl(ddt_exchange_dev<V>, grid_for(total, res[3], grid_cap), s, reinterpret_cast<const uint8_t*>(src),
+                   xa);
     }
 }
 
