@@ -321,6 +321,37 @@ def e2e_zero_copy(torch, ddt, rank, P, local, dirs, nvars, comm, mode, K, dist_o
     return ms, h2d, d2h
 
 
+def latency_floor(ddt, torch, K, R=96):
+    """The launch + dependent-DRAM-round-trip floor of ONE fused launch, timed
+    exactly like the configs[1] step: a K-step CUDA graph over R rotating
+    buffers, each step one fused pack of the configs[0] vector (512 B, one
+    request, 16 segments) from a buffer no recent step touched.  The configs[1]
+    step moves 1.57 MB in the same single launch; value / floor says how much
+    of the step is more than the floor."""
+    from ddt_inputs import config1_spec
+    t = ddt.Type.from_spec(config1_spec())
+    srcs = torch.empty((R, 2 << 20), dtype=torch.uint8, device="cuda")  # 2 MiB apart: distinct DRAM pages
+    srcs.random_(0, 256)
+    dsts = torch.empty((R, 2 << 20), dtype=torch.uint8, device="cuda")
+    q = ddt.Queue()
+    plans = []
+    for r in range(R):
+        q.pack(t, srcs[r], 1, dsts[r])
+        plans.append(ddt.Plan(q))
+
+    class _W:
+        k = 0
+
+        def step(self):
+            plans[self.k % R].launch()
+            self.k += 1
+    ms, _ = run_steps(torch, _W(), K, 10, False, None, capture=True)
+    for p in plans:
+        p.destroy()
+    q.destroy()
+    return ms * 1e3
+
+
 # ------------------------------------------------------------------ config 5 pack
 def pack_roofline(ddt, torch, hbm_peak, reps=20):
     """Dense vector pack (configs[4] layout: 256 B blocks, 50% density), fused
@@ -617,6 +648,15 @@ def main():
             "note": (f"latency-bound: {alg_bytes / 1e6:.2f} MB of algorithmic bytes per step (self messages: "
                      "DirectIPC 2S, remote: 4S); time = device time per step in the back-to-back K-step run "
                      "(kernel + inter-kernel gap)")}
+
+    if rank == 0 and not dist_on:
+        try:
+            fl = latency_floor(ddt, torch, K)
+            roof["latency_floor"] = {"us": round(fl, 3), "value_over_floor": round(best["mean_ms"] * 1e3 / fl, 2),
+                                     "what": "same K-step graph harness, one fused launch moving 512 B (configs[0] "
+                                             "vector pack) from cold buffers: launch + one dependent DRAM round trip"}
+        except Exception as e:
+            roof["latency_floor"] = {"error": f"{type(e).__name__}: {e}"}
 
     extras = {}
     if not args.no_extras:
