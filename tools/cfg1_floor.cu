@@ -82,6 +82,74 @@ __global__ void faces8_big(double* __restrict__ a, const __grid_constant__ Big p
     }
 }
 
+// ---- PDL variants (what the library does since §7g): trigger on entry,
+// address arithmetic, griddepcontrol.wait, then the loads
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__global__ void empty_pdl(double*) { pdl_trigger(); pdl_wait(); }
+__global__ void phased_pdl(double* __restrict__ a) {
+    pdl_trigger();
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    constexpr int U = 65;
+    if (t < 4 * 128 * U) {
+        const int f = t / (128 * U), r = (t / U) % 128, j = t % U;
+        long long s, d;
+        face_rows(f, r, s, d);
+        const char* ps = reinterpret_cast<const char*>(a + s);
+        char* pd = reinterpret_cast<char*>(a + d);
+        pdl_wait();
+        if (j == 0) *reinterpret_cast<uint2*>(pd + 8) = __ldg(reinterpret_cast<const uint2*>(ps + 8));
+        else if (j == U - 1) *reinterpret_cast<uint2*>(pd + 1024) = __ldg(reinterpret_cast<const uint2*>(ps + 1024));
+        else *reinterpret_cast<uint4*>(pd + 16 * j) = __ldg(reinterpret_cast<const uint4*>(ps + 16 * j));
+    } else if (t < 4 * 128 * U + 2 * 16384) {
+        const int u = t - 4 * 128 * U, f = u / 16384, c = u % 16384, z = 1 + c / 128, y = 1 + c % 128;
+        pdl_wait();
+        if (f == 0) a[idx(z, y, 129)] = __ldg(a + idx(z, y, 1));
+        else a[idx(z, y, 0)] = __ldg(a + idx(z, y, 128));
+    } else {
+        pdl_wait();
+    }
+}
+// x faces paired: one thread per row moves both of the row's x-face cells
+// (x=1 -> x=129 and x=128 -> x=0): the row's two ends are touched together
+__global__ void xpair_pdl(double* __restrict__ a) {
+    pdl_trigger();
+    const int t = blockIdx.x * blockDim.x + threadIdx.x;
+    constexpr int U = 65;
+    if (t < 4 * 128 * U) {
+        const int f = t / (128 * U), r = (t / U) % 128, j = t % U;
+        long long s, d;
+        face_rows(f, r, s, d);
+        const char* ps = reinterpret_cast<const char*>(a + s);
+        char* pd = reinterpret_cast<char*>(a + d);
+        pdl_wait();
+        if (j == 0) *reinterpret_cast<uint2*>(pd + 8) = __ldg(reinterpret_cast<const uint2*>(ps + 8));
+        else if (j == U - 1) *reinterpret_cast<uint2*>(pd + 1024) = __ldg(reinterpret_cast<const uint2*>(ps + 1024));
+        else *reinterpret_cast<uint4*>(pd + 16 * j) = __ldg(reinterpret_cast<const uint4*>(ps + 16 * j));
+    } else if (t < 4 * 128 * U + 16384) {
+        const int c = t - 4 * 128 * U, z = 1 + c / 128, y = 1 + c % 128;
+        pdl_wait();
+        const double v1 = __ldg(a + idx(z, y, 1)), v2 = __ldg(a + idx(z, y, 128));
+        a[idx(z, y, 129)] = v1;
+        a[idx(z, y, 0)] = v2;
+    } else {
+        pdl_wait();
+    }
+}
+template <class... A>
+static void launch_pdl(void (*k)(A...), int grid, cudaStream_t s, A... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(256);
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    cudaLaunchKernelEx(&cfg, k, args...);
+}
+
 template <class F>
 static double graph_us(F launch, int R, int K) {
     cudaStream_t st;
@@ -129,6 +197,13 @@ int main() {
     Big big{};
     double teb = graph_us([&](cudaStream_t s, int r) { empty_big<<<gp, 256, 0, s>>>(arr[r], big); }, R, K);
     double t8b = graph_us([&](cudaStream_t s, int r) { faces8_big<<<g8, 256, 0, s>>>(arr[r], big); }, R, K);
+    const int gx = (4 * 128 * 65 + 16384 + 255) / 256;
+    double tep = graph_us([&](cudaStream_t s, int r) { launch_pdl(empty_pdl, gp, s, arr[r]); }, R, K);
+    double tpp = graph_us([&](cudaStream_t s, int r) { launch_pdl(phased_pdl, gp, s, arr[r]); }, R, K);
+    double txp = graph_us([&](cudaStream_t s, int r) { launch_pdl(xpair_pdl, gx, s, arr[r]); }, R, K);
+    printf("{\"kernel\": \"empty_pdl\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gp, tep);
+    printf("{\"kernel\": \"phased_pdl\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gp, tpp);
+    printf("{\"kernel\": \"xpair_pdl\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gx, txp);
     printf("{\"kernel\": \"empty\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gp, te);
     printf("{\"kernel\": \"empty_4KB_params\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gp, teb);
     printf("{\"kernel\": \"faces8_4KB_params\", \"ctas\": %d, \"us_per_step\": %.3f}\n", g8, t8b);
