@@ -759,6 +759,7 @@ static int resident_ctas(K kernel) {
 }
 
 static uint32_t grid_for(uint32_t total, int resident, int grid_cap) {
+    if (grid_cap < 0) return total;  // DDT_GRID_ALL (plain batches only)
     uint32_t cap = (uint32_t)resident;
     if (grid_cap > 0 && (uint32_t)grid_cap < cap) cap = (uint32_t)grid_cap;
     return total < cap ? total : cap;
@@ -788,9 +789,20 @@ static void launch_pdl(void (*k)(Args...), uint32_t grid, cudaStream_t s, const 
     cudaLaunchKernelEx(&cfg, k, args...);
 }
 
+// experiments: DDT_GRID_ALL=1 launches one CTA per item (hardware CTA
+// scheduling) instead of a resident-sized grid walking the items
+static bool grid_all() {
+    static const bool on = [] {
+        const char* e = getenv("DDT_GRID_ALL");
+        return e && e[0] == '1';
+    }();
+    return on;
+}
+
 template <int V>
 static void launch_fused_v(int form, const void* src, uint32_t total, cudaStream_t s, int grid_cap) {
     static int res[4] = {0, 0, 0, 0};
+    if (grid_all() && grid_cap <= 0) grid_cap = -1;
     if (form == 1) {
         if (!res[1]) res[1] = resident_ctas(ddt_fused_param<kParamSmall, V>);
         launch_pdl(ddt_fused_param<kParamSmall, V>, grid_for(total, res[1], grid_cap), s,
