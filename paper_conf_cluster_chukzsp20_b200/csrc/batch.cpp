@@ -222,10 +222,11 @@ int choose_ub(const HostBatch& b, int sm_count) {
     return 1;
 }
 
-uint32_t write_device_table(void* dst, const HostBatch& b, int ub) {
+uint32_t write_device_table(void* dst, const HostBatch& b, int ub, uint64_t ticket) {
     size_t n = b.descs.size();
     auto* h = reinterpret_cast<BatchHeader*>(dst);
     std::memset(h, 0, sizeof(*h));
+    h->ticket = ticket;
     auto* prefix = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(dst) + sizeof(BatchHeader));
     uint32_t items = fill_prefix(prefix, b, ub);
     size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
@@ -264,6 +265,7 @@ static void to_param(const HostBatch& b, Launchable& out) {
     p->h.ub = (uint32_t)out.ub;
     p->h.flags = batch_flags(b);
     p->h.total_items = fill_prefix(p->prefix, b, out.ub);
+    p->h.ticket = out.ticket;
     std::copy(b.gm.begin(), b.gm.end(), p->gm);
     std::copy(b.descs.begin(), b.descs.end(), p->descs);
     std::copy(b.aux.begin(), b.aux.end(), p->aux);
@@ -294,10 +296,33 @@ static int batch_variant(const HostBatch& b) {
     return 1 + lw;
 }
 
+// Work distribution of a multi-wave plain batch (>= kTicketMinItemsPerSM
+// items per SM, no exchange flags; exchange batches keep the static order their
+// flag protocol is proven for).  Measured on one B200:
+//   * spread halo plans (COMB): one CTA per item (grid_mode 2) -- 128 -> 116 us;
+//   * <= kTicketMaxReqs large requests: dynamic tickets (grid_mode 1) --
+//     16 x 64 MiB packs 5.5 -> 6.4 TB/s;
+//   * many requests (1024 x 1 MiB): the static cyclic order stays best.
+static int grid_mode_for(const HostBatch& b, int ub, int sm_count) {
+    const char* e = getenv("DDT_GRID_MODE");  // experiments: force 0 / 1 / 2
+    for (const XInfo& x : b.xinfo)
+        if (x.signal || x.wait) return 0;
+    for (const ReqDesc& d : b.descs)
+        if (d.kind == K_LL || d.op == OP_SIGNAL) return 0;
+    uint64_t items = 0;
+    for (const ReqDesc& d : b.descs) items += desc_items(d, ub);
+    if (items < (uint64_t)kTicketMinItemsPerSM * (uint64_t)sm_count) return 0;
+    int m = !b.order.empty() ? 2 : (b.descs.size() <= (size_t)kTicketMaxReqs ? 1 : 0);
+    if (e && e[0] >= '0' && e[0] <= '2') m = e[0] - '0';
+    return (m == 1 && !b.ticket) ? 0 : m;
+}
+
 void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count, int force_ub) {
     size_t n = std::max(b.descs.size(), b.aux.size());
     out.variant = batch_variant(b);
     out.ub = force_ub > 0 ? force_ub : choose_ub(b, sm_count);
+    out.grid_mode = grid_mode_for(b, out.ub, sm_count);
+    out.ticket = out.grid_mode == 1 ? b.ticket : 0;
     out.blob.clear();
     const char* force = getenv("DDT_FORCE_TABLE");  // experiments: always use the device-table form
     if (force && force[0] == '1') allow_param = false;
@@ -318,6 +343,7 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
 
 int launch_fused(const Launchable& l, void* stream, int grid_cap) {
     const void* src = l.form == 3 ? l.dev : (const void*)l.blob.data();
+    if (l.grid_mode == 2 && grid_cap <= 0) grid_cap = -1;  // one CTA per item
     return launch_fused_form(l.form, l.variant, src, l.total_items, stream, grid_cap);
 }
 

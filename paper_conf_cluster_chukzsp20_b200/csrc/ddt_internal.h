@@ -129,7 +129,8 @@ struct HostBatch {
     std::vector<XInfo> xinfo;
     std::vector<uint32_t> gm;  // group size per request (empty: no groups), see device_desc.h
     std::vector<uint32_t> order;  // explicit item table (empty: prefix search), see device_desc.h kSpreadShift
-    void clear() { descs.clear(); aux.clear(); xinfo.clear(); gm.clear(); order.clear(); }
+    uint64_t ticket = 0;  // device u32[2] ticket counter offered by the caller (0: static order only)
+    void clear() { descs.clear(); aux.clear(); xinfo.clear(); gm.clear(); order.clear(); ticket = 0; }
     void add(ReqDesc s, const ReqDesc& d) {
         s.aux = (uint32_t)aux.size();
         aux.push_back(d);
@@ -145,9 +146,11 @@ struct Launchable {
     uint32_t total_items = 0;
     int variant = 0;            // 0 generic; 1 + lw: strided-only, one vector width; 6 general lists; 7 strided-only, phased units
     int ub = kUnroll;           // vectors per thread per item
+    uint64_t ticket = 0;        // dynamic item tickets in use (device counter), 0 = static order
+    int grid_mode = 0;          // 0: resident grid, static item order; 1: resident grid, tickets; 2: one CTA per item
 };
 size_t device_table_bytes(const HostBatch& b);
-uint32_t write_device_table(void* dst, const HostBatch& b, int ub);
+uint32_t write_device_table(void* dst, const HostBatch& b, int ub, uint64_t ticket = 0);
 // Items per thread for a batch: the largest of {4, 2, 1} that still gives
 // >= 2 items per SM, so latency-bound batches use every SM.
 int choose_ub(const HostBatch& b, int sm_count);
@@ -179,6 +182,7 @@ int device_sm_count(int device);
 // queue accessors (queue.cpp)
 int queue_device(ddt_queue_s* q);
 void* queue_stream(ddt_queue_s* q);
+uint64_t queue_ticket(ddt_queue_s* q);  // the queue's device ticket counter (see device_desc.h)
 int queue_sm_count(ddt_queue_s* q);
 ddt_status_t queue_sticky(ddt_queue_s* q);
 void queue_set_sticky(ddt_queue_s* q, ddt_status_t s);

@@ -145,8 +145,18 @@ struct alignas(16) BatchHeader {
     uint32_t ub;            // vectors per thread per item (1, 2 or 4)
     uint32_t flags;         // bit 0: blocked item order (else cyclic over CTAs); bit 1: grouped (gm[] present)
     uint32_t order_offset;  // 0, or byte offset of the explicit item table (kBatchSpread)
-    uint32_t pad[3];
+    uint32_t pad0;
+    uint64_t ticket;        // 0: static item order; else device u32[2] {next, exited}: dynamic item tickets
 };
+// Dynamic item tickets (multi-wave plain batches): a resident-sized grid takes
+// items in increasing order from an atomic counter instead of the static
+// cyclic assignment, so the items in flight stay a compact window (DRAM page
+// locality) however unevenly CTAs progress; the last CTA to exit resets the
+// counter for the next launch (launches sharing a counter are stream-ordered:
+// one counter per queue).  Used by multi-wave batches (>= kTicketMinItemsPerSM
+// items per SM) of at most kTicketMaxReqs requests (batch.cpp grid_mode_for).
+constexpr uint32_t kTicketMinItemsPerSM = 16;
+constexpr uint32_t kTicketMaxReqs = 64;
 constexpr uint32_t kBatchBlocked = 1u, kBatchGrouped = 2u;
 // Spread batches (batch.cpp spread_items): an explicit item table order[item] =
 // (request << kSpreadShift) | chunk, ordered so that every request's chunks are

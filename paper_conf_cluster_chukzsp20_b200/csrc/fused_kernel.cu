@@ -440,6 +440,7 @@ struct TableView {
     const ReqDesc* aux;
     const XInfo* xinfo;
     const uint32_t* order;    // explicit item table (kBatchSpread), or null
+    unsigned int* ticket;     // dynamic item tickets {next, exited}, or null (static order)
 };
 
 __device__ __forceinline__ TableView view_of(const uint8_t* t) {
@@ -455,6 +456,7 @@ __device__ __forceinline__ TableView view_of(const uint8_t* t) {
     v.aux = reinterpret_cast<const ReqDesc*>(t + h->aux_offset);
     v.xinfo = h->xinfo_offset ? reinterpret_cast<const XInfo*>(t + h->xinfo_offset) : nullptr;
     v.order = h->order_offset ? reinterpret_cast<const uint32_t*>(t + h->order_offset) : nullptr;
+    v.ticket = reinterpret_cast<unsigned int*>(h->ticket);
     return v;
 }
 
@@ -471,6 +473,7 @@ __device__ __forceinline__ TableView view_of(const ParamBatch<CAP>& p) {
     v.aux = p.aux;
     v.xinfo = p.xinfo;
     v.order = nullptr;
+    v.ticket = reinterpret_cast<unsigned int*>(p.h.ticket);
     return v;
 }
 
@@ -551,7 +554,22 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         last = min(tv.total, first + per);
         step = 1;
     }
-    for (uint32_t item = first; item < last; item += step) {
+    // dynamic tickets (device_desc.h): thread 0 fetches the next item's ticket
+    // while the CTA moves the current one (two shared slots, one barrier per item)
+    __shared__ uint32_t s_tk[2];
+    const bool dyn = !XCHG && tv.ticket != nullptr;
+    int par = 0;
+    if (dyn) {
+        if (!waited) {  // the counter is reset by the previous grid: wait for it first
+            pdl_wait();
+            waited = true;
+        }
+        if (threadIdx.x == 0) s_tk[0] = atomicAdd(tv.ticket, 1u);
+        __syncthreads();
+        first = s_tk[0];
+    }
+    for (uint32_t item = first; item < last;) {
+        if (dyn && threadIdx.x == 0) s_tk[par ^ 1] = atomicAdd(tv.ticket, 1u);
         uint32_t r, local;  // the item's request and chunk index within it
         if (tv.order) {     // spread batch: explicit item table
             const uint32_t e = __ldg(tv.order + item);
@@ -680,6 +698,21 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
                 }
             }
         }
+        if (dyn) {
+            __syncthreads();  // the prefetched ticket is visible; every thread is past this item
+            par ^= 1;
+            item = s_tk[par];
+        } else {
+            item += step;
+        }
+    }
+    if (dyn && threadIdx.x == 0) {  // the last CTA out resets the counter for the next launch
+        __threadfence();
+        if (atomicAdd(tv.ticket + 1, 1u) == gridDim.x - 1) {
+            tv.ticket[0] = 0u;
+            tv.ticket[1] = 0u;
+            __threadfence();
+        }
     }
 }
 
@@ -759,7 +792,7 @@ static int resident_ctas(K kernel) {
 }
 
 static uint32_t grid_for(uint32_t total, int resident, int grid_cap) {
-    if (grid_cap < 0) return total;  // DDT_GRID_ALL (plain batches only)
+    if (grid_cap < 0) return total;  // one CTA per item (Launchable::grid_mode 2, plain batches only)
     uint32_t cap = (uint32_t)resident;
     if (grid_cap > 0 && (uint32_t)grid_cap < cap) cap = (uint32_t)grid_cap;
     return total < cap ? total : cap;
@@ -789,20 +822,9 @@ static void launch_pdl(void (*k)(Args...), uint32_t grid, cudaStream_t s, const 
     cudaLaunchKernelEx(&cfg, k, args...);
 }
 
-// experiments: DDT_GRID_ALL=1 launches one CTA per item (hardware CTA
-// scheduling) instead of a resident-sized grid walking the items
-static bool grid_all() {
-    static const bool on = [] {
-        const char* e = getenv("DDT_GRID_ALL");
-        return e && e[0] == '1';
-    }();
-    return on;
-}
-
 template <int V>
 static void launch_fused_v(int form, const void* src, uint32_t total, cudaStream_t s, int grid_cap) {
     static int res[4] = {0, 0, 0, 0};
-    if (grid_all() && grid_cap <= 0) grid_cap = -1;
     if (form == 1) {
         if (!res[1]) res[1] = resident_ctas(ddt_fused_param<kParamSmall, V>);
         launch_pdl(ddt_fused_param<kParamSmall, V>, grid_for(total, res[1], grid_cap), s,

@@ -193,7 +193,7 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
     make_launchable(b, !spread, l, sm_count, ub);
     if (l.form != 3) return DDT_OK;
     std::vector<uint8_t> host(device_table_bytes(b));
-    write_device_table(host.data(), b, l.ub);
+    write_device_table(host.data(), b, l.ub, l.ticket);
     return upload(host, &l.dev);
 }
 
@@ -733,6 +733,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             st = add_req(unpackb, r.type, OP_UNPACK, (char*)h->recv_stage + RL.data_off[(size_t)i], r.buf, r.count,
                          nullptr);
         }
+        packb.ticket = unpackb.ticket = queue_ticket(q);
         if (st == DDT_OK && !packb.descs.empty()) st = make_table(packb, h->pack_l, queue_sm_count(q));
         if (st == DDT_OK && !unpackb.descs.empty()) st = make_table(unpackb, h->unpack_l, queue_sm_count(q));
         h->launches = (packb.descs.empty() ? 0 : 1) + (unpackb.descs.empty() ? 0 : 1);
@@ -872,6 +873,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                 if (xb.xinfo[i].signal) xb.xinfo[i].nitems = desc_items(xb.descs[i], kXchgUb);
             // flag-free plans (self messages only) run the plain fused kernel:
             // adaptive item size, like any other batch
+            xb.ticket = queue_ticket(q);  // used only if the plan is flag-free (plain fused kernel)
             st = make_table(xb, h->x_l, queue_sm_count(q), h->x_flags ? kXchgUb : 0);
         }
         size_t ctrl_bytes = sizeof(XCtrl) + sizeof(unsigned long long) * std::max<size_t>(npack, 1);

@@ -74,6 +74,7 @@ struct ddt_queue_s {
     uint32_t* resp_host = nullptr;
     uint32_t* resp_dev = nullptr;
     uint32_t* done_ctr = nullptr;
+    uint32_t* ticket = nullptr;  // device u32[2]: dynamic item tickets of this queue's (stream-ordered) launches
 };
 
 namespace {
@@ -250,6 +251,13 @@ ddt_status_t ddt_queue_create(int device, void* cuda_stream, int32_t capacity, d
             return cuda_fail("context init", e);
         }
         q->sm_count = device_sm_count(device);
+        e = cudaMalloc((void**)&q->ticket, 16);
+        if (e == cudaSuccess) e = cudaMemset(q->ticket, 0, 16);
+        if (e != cudaSuccess) {
+            if (q->ticket) cudaFree(q->ticket);
+            delete q;
+            return cuda_fail("ticket counter", e);
+        }
     }
     *out = q;
     return DDT_OK;
@@ -269,6 +277,7 @@ ddt_status_t ddt_queue_destroy(ddt_queue_t q) {
         if (q->dev_table) cudaFree(q->dev_table);
         if (q->resp_host) cudaFreeHost(q->resp_host);
         if (q->done_ctr) cudaFree(q->done_ctr);
+        if (q->ticket) cudaFree(q->ticket);
     }
     delete q;
     return DDT_OK;
@@ -355,13 +364,14 @@ int32_t ddt_flush(ddt_queue_t q) {
     int32_t nflushed = (int32_t)(q->tail - q->flushed);
     if (!q->scratch.descs.empty()) {
         Launchable& L = q->launch;
+        q->scratch.ticket = (uint64_t)(uintptr_t)q->ticket;
         make_launchable(q->scratch, true, L, q->sm_count);
         if (L.form == 3) {
             size_t tb = device_table_bytes(q->scratch);
             ddt_queue_s::HostSlot* slot = nullptr;
             ddt_status_t s = ensure_host_slot(q, tb, &slot);
             if (s != DDT_OK) return q->sticky = s;
-            write_device_table(slot->p, q->scratch, L.ub);
+            write_device_table(slot->p, q->scratch, L.ub, L.ticket);
             if (q->dev_cap < tb) {
                 if (q->dev_table) cudaFree(q->dev_table);  // synchronizes: old table no longer in use
                 size_t cap = std::max<size_t>(tb, 64 << 10);
@@ -468,11 +478,12 @@ ddt_status_t ddt_plan_create(ddt_queue_t q, ddt_plan_t* out) {
             }
     }
     if (!q->scratch.descs.empty()) {
+        q->scratch.ticket = (uint64_t)(uintptr_t)q->ticket;
         make_launchable(q->scratch, true, p->launch, q->sm_count);
         for (const ReqDesc& d : q->scratch.descs) q->stats.phased += d.ph ? 1 : 0;
         if (p->launch.form == 3) {
             std::vector<uint8_t> host(device_table_bytes(q->scratch));
-            write_device_table(host.data(), q->scratch, p->launch.ub);
+            write_device_table(host.data(), q->scratch, p->launch.ub, p->launch.ticket);
             cudaError_t e = cudaMalloc(&p->launch.dev, host.size());
             if (e == cudaSuccess) e = cudaMemcpy(p->launch.dev, host.data(), host.size(), cudaMemcpyHostToDevice);
             if (e != cudaSuccess) {
@@ -529,6 +540,7 @@ ddt_status_t ddt_queue_get_stats(ddt_queue_t q, ddt_queue_stats_t* out) {
 namespace ddt {
 int queue_device(ddt_queue_s* q) { return q->device; }
 void* queue_stream(ddt_queue_s* q) { return (void*)q->stream; }
+uint64_t queue_ticket(ddt_queue_s* q) { return (uint64_t)(uintptr_t)q->ticket; }
 int queue_sm_count(ddt_queue_s* q) { return q->sm_count; }
 ddt_status_t queue_sticky(ddt_queue_s* q) { return q->sticky; }
 void queue_set_sticky(ddt_queue_s* q, ddt_status_t s) {
