@@ -155,7 +155,7 @@ struct alignas(16) BatchHeader {
 // counter for the next launch (launches sharing a counter are stream-ordered:
 // one counter per queue).  Used by multi-wave batches (>= kTicketMinItemsPerSM
 // items per SM) of at most kTicketMaxReqs requests (batch.cpp grid_mode_for).
-constexpr uint32_t kTicketMinItemsPerSM = 16;
+constexpr uint32_t kTicketMinItemsPerSM = 8;
 constexpr uint32_t kTicketMaxReqs = 64;
 constexpr uint32_t kBatchBlocked = 1u, kBatchGrouped = 2u;
 // Spread batches (batch.cpp spread_items): an explicit item table order[item] =
