@@ -321,6 +321,8 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
     size_t n = std::max(b.descs.size(), b.aux.size());
     out.variant = batch_variant(b);
     out.ub = force_ub > 0 ? force_ub : choose_ub(b, sm_count);
+    const char* v9 = getenv("DDT_NO_V9");  // experiments
+    if (out.variant == 7 && out.ub == 1 && !(v9 && v9[0] == '1')) out.variant = 9;
     out.grid_mode = grid_mode_for(b, out.ub, sm_count);
     out.ticket = out.grid_mode == 1 ? b.ticket : 0;
     out.blob.clear();

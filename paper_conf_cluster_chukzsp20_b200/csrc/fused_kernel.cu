@@ -725,19 +725,21 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
 // phased 16-B units (batch.cpp phase_batch); 8 = 4-B vectors, closed-form or
 // uniform-list layouts, kUnrollNarrow loads in flight per thread (sparse lists
 // such as configs[2] are latency x concurrency bound, not bandwidth bound).
+// 9 = variant 7 for one vector per thread per item (ub = 1: latency-bound
+// halo steps such as configs[1]): no unrolled load slots, a short hot path.
 template <int V> struct VarT {
-    static constexpr int LW = (V == 0 || V == 6 || V == 7) ? -1 : (V == 8 ? 2 : V - 1);
-    static constexpr int UNR = V == 8 ? kUnrollNarrow : kUnroll;
-    static constexpr bool SONLY = (V >= 1 && V <= 5) || V == 7;
+    static constexpr int LW = (V == 0 || V == 6 || V == 7 || V == 9) ? -1 : (V == 8 ? 2 : V - 1);
+    static constexpr int UNR = V == 8 ? kUnrollNarrow : (V == 9 ? 1 : kUnroll);
+    static constexpr bool SONLY = (V >= 1 && V <= 5) || V == 7 || V == 9;
     static constexpr bool GW = V == 6;
-    static constexpr bool PH = V == 7;
+    static constexpr bool PH = V == 7 || V == 9;
     // resident CTAs per SM the register budget must allow.  Plain batches: 5
     // (48 registers) -- a dense multi-request pack reloads its descriptor at
     // almost every item and needs the extra CTAs to keep loads in flight
     // (tools/pack_probe.py: 1 MiB x 1024 packs 4.74 -> 6.08 TB/s from 3 to 5
     // CTAs/SM); exchange kernels (flags, tracing) keep their registers.
-    static constexpr int MINB = V == 7 ? DDT_V7_MINB : (V == 8 ? DDT_V8_MINB : DDT_MINB);
-    static constexpr int XMINB = V == 7 ? DDT_V7_MINB : (V == 8 ? DDT_V8_MINB : DDT_XMINB);
+    static constexpr int MINB = (V == 7 || V == 9) ? DDT_V7_MINB : (V == 8 ? DDT_V8_MINB : DDT_MINB);
+    static constexpr int XMINB = (V == 7 || V == 9) ? DDT_V7_MINB : (V == 8 ? DDT_V8_MINB : DDT_XMINB);
 };
 
 template <int V>
@@ -876,6 +878,7 @@ int launch_fused_form(int form, int variant, const void* src, uint32_t total_ite
     case 6: launch_fused_v<6>(form, src, total_items, s, grid_cap); break;
     case 7: launch_fused_v<7>(form, src, total_items, s, grid_cap); break;
     case 8: launch_fused_v<8>(form, src, total_items, s, grid_cap); break;
+    case 9: launch_fused_v<9>(form, src, total_items, s, grid_cap); break;
     default: launch_fused_v<0>(form, src, total_items, s, grid_cap); break;
     }
     return (int)cudaGetLastError();
@@ -894,6 +897,7 @@ int launch_exchange_form(int form, int variant, const void* src, uint32_t total_
     case 6: launch_exchange_v<6>(form, src, total_items, xa, s, grid_cap); break;
     case 7: launch_exchange_v<7>(form, src, total_items, xa, s, grid_cap); break;
     case 8: launch_exchange_v<8>(form, src, total_items, xa, s, grid_cap); break;
+    case 9: launch_exchange_v<9>(form, src, total_items, xa, s, grid_cap); break;
     default: launch_exchange_v<0>(form, src, total_items, xa, s, grid_cap); break;
     }
     return (int)cudaGetLastError();
