@@ -23,4 +23,12 @@ from .types import Type  # noqa: F401
 from .queue import Queue, Plan  # noqa: F401
 from .halo import Halo, Comm, Windows  # noqa: F401
 
-__all__ = ["DDTError", "Type", "Queue", "Plan", "Halo", "Comm", "Windows", "lib", "DDT_XCHG_NCCL", "DDT_XCHG_P2P"]
+
+
+def reload_env():
+    """Make the library re-read its DDT_* experiment knobs (ddt_reload_env):
+    call after changing one of those environment variables at run time."""
+    lib().ddt_reload_env()
+
+
+__all__ = ["reload_env", "DDTError", "Type", "Queue", "Plan", "Halo", "Comm", "Windows", "lib", "DDT_XCHG_NCCL", "DDT_XCHG_P2P"]

@@ -103,6 +103,7 @@ PROTOTYPES = {
     "ddt_strerror": (ctypes.c_char_p, [I32]),
     "ddt_last_error_message": (ctypes.c_char_p, []),
     "ddt_version": (I32, []),
+    "ddt_reload_env": (None, []),
     "ddt_built_sm": (I32, []),
 }
 

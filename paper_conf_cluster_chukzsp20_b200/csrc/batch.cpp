@@ -35,7 +35,7 @@ static size_t pad16(size_t v) { return (v + 15) & ~(size_t)15; }
 
 // Item order (experiments: DDT_ITEM_ORDER=blocked); cyclic is the default.
 static uint32_t batch_flags(const HostBatch& b) {
-    const char* e = getenv("DDT_ITEM_ORDER");
+    const char* e = DDT_KNOB("DDT_ITEM_ORDER");
     uint32_t f = (e && e[0] == 'b') ? kBatchBlocked : 0u;
     if (!b.gm.empty()) f |= kBatchGrouped;
     return f;
@@ -49,7 +49,7 @@ static int exchange_class(const HostBatch& b, size_t i) {
 }
 
 void group_equal_requests(HostBatch& b, int ub, int max_m) {
-    const char* off = getenv("DDT_NO_GROUP");  // experiments: no interleaving
+    const char* off = DDT_KNOB("DDT_NO_GROUP");  // experiments: no interleaving
     const size_t n = b.descs.size();
     if ((off && off[0] == '1') || n < 2 || max_m < 2) return;
     std::vector<size_t> order;
@@ -136,7 +136,7 @@ static bool try_phase(ReqDesc& S, ReqDesc& D) {
 }
 
 void phase_batch(HostBatch& b) {
-    const char* off = getenv("DDT_NO_PHASE");  // experiments: plain 8-B vectors
+    const char* off = DDT_KNOB("DDT_NO_PHASE");  // experiments: plain 8-B vectors
     if (off && off[0] == '1') return;
     for (const auto* v : {&b.descs, &b.aux})
         for (const ReqDesc& d : *v)
@@ -193,7 +193,7 @@ size_t device_table_bytes(const HostBatch& b) {
 // uniform-list layout, at least one side is a list (the sparse configs[2]
 // shape); items may then hold kUnrollNarrow vectors per thread.
 static bool narrow_list_batch(const HostBatch& b) {
-    const char* off = getenv("DDT_NO_NARROW");  // experiments
+    const char* off = DDT_KNOB("DDT_NO_NARROW");  // experiments
     if (off && off[0] == '1') return false;
     bool list = false;
     for (const auto* v : {&b.descs, &b.aux})
@@ -207,7 +207,7 @@ static bool narrow_list_batch(const HostBatch& b) {
 }
 
 int choose_ub(const HostBatch& b, int sm_count) {
-    const char* env = getenv("DDT_UB");
+    const char* env = DDT_KNOB("DDT_UB");
     if (env && (atoi(env) == 1 || atoi(env) == 2 || atoi(env) == 4 || atoi(env) == 8)) {
         const int u = atoi(env);
         return u == 8 && !narrow_list_batch(b) ? 4 : u;
@@ -259,8 +259,12 @@ uint32_t write_device_table(void* dst, const HostBatch& b, int ub, uint64_t tick
 
 template <int CAP>
 static void to_param(const HostBatch& b, Launchable& out) {
-    out.blob.assign(sizeof(ParamBatch<CAP>), 0);
+    // the kernel reads only the header and the first nreq entries of each
+    // array: no per-flush zero-fill of the ~4-30 KB block (the first resize
+    // zeroes it once)
+    if (out.blob.size() != sizeof(ParamBatch<CAP>)) out.blob.assign(sizeof(ParamBatch<CAP>), 0);
     auto* p = reinterpret_cast<ParamBatch<CAP>*>(out.blob.data());
+    std::memset(&p->h, 0, sizeof(p->h));
     p->h.nreq = (uint32_t)b.descs.size();
     p->h.ub = (uint32_t)out.ub;
     p->h.flags = batch_flags(b);
@@ -304,7 +308,7 @@ static int batch_variant(const HostBatch& b) {
 //     16 x 64 MiB packs 5.5 -> 6.4 TB/s;
 //   * many requests (1024 x 1 MiB): the static cyclic order stays best.
 static int grid_mode_for(const HostBatch& b, int ub, int sm_count) {
-    const char* e = getenv("DDT_GRID_MODE");  // experiments: force 0 / 1 / 2
+    const char* e = DDT_KNOB("DDT_GRID_MODE");  // experiments: force 0 / 1 / 2
     for (const XInfo& x : b.xinfo)
         if (x.signal || x.wait) return 0;
     for (const ReqDesc& d : b.descs)
@@ -321,14 +325,13 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
     size_t n = std::max(b.descs.size(), b.aux.size());
     out.variant = batch_variant(b);
     out.ub = force_ub > 0 ? force_ub : choose_ub(b, sm_count);
-    const char* v9 = getenv("DDT_NO_V9");  // experiments
+    const char* v9 = DDT_KNOB("DDT_NO_V9");  // experiments
     if (out.variant == 7 && out.ub == 1 && !(v9 && v9[0] == '1')) out.variant = 9;
     out.grid_mode = grid_mode_for(b, out.ub, sm_count);
     out.ticket = out.grid_mode == 1 ? b.ticket : 0;
-    out.blob.clear();
-    const char* force = getenv("DDT_FORCE_TABLE");  // experiments: always use the device-table form
+    const char* force = DDT_KNOB("DDT_FORCE_TABLE");  // experiments: always use the device-table form
     if (force && force[0] == '1') allow_param = false;
-    const char* large = getenv("DDT_FORCE_LARGE_PARAM");  // experiments: skip the small parameter form
+    const char* large = DDT_KNOB("DDT_FORCE_LARGE_PARAM");  // experiments: skip the small parameter form
     const bool skip_small = large && large[0] == '1';
     if (allow_param && n <= (size_t)kParamSmall && !skip_small) {
         out.form = 1;
@@ -338,6 +341,7 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
         to_param<kParamLarge>(b, out);
     } else {
         out.form = 3;
+        out.blob.clear();
         std::vector<uint32_t> prefix(b.descs.size() + 1);
         out.total_items = fill_prefix(prefix.data(), b, out.ub);
     }

@@ -14,6 +14,23 @@ namespace ddt {
 
 // ---------------------------------------------------------------- errors
 void set_error(const std::string& msg);
+// Cached getenv for DDT_* knobs (see ddt_reload_env in include/ddt.h): one
+// static slot per call site, re-read only after a reload (lock-free fast
+// path: one relaxed load + compare).  The pointer is valid until the next
+// ddt_reload_env().
+struct KnobSlot {
+    const char* name;
+    std::atomic<uint64_t> gen{0};
+    std::string val;
+    bool set = false;
+    explicit KnobSlot(const char* n) : name(n) {}
+    const char* get();
+};
+#define DDT_KNOB(NAME)                                  \
+    ([]() -> const char* {                              \
+        static ::ddt::KnobSlot ddt_knob_slot_{NAME};    \
+        return ddt_knob_slot_.get();                    \
+    }())
 const char* last_error();
 ddt_status_t cuda_fail(const char* what, int cuda_err);
 

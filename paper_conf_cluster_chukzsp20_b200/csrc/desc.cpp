@@ -53,7 +53,7 @@ int side_lw(ddt_type_s* t, const void* p, int64_t count) {
 // experiments: DDT_NO_L2HINT=1 disables the sparse-side prefetch-size hint
 static bool l2_hint_on() {
     static const bool on = [] {
-        const char* e = getenv("DDT_NO_L2HINT");
+        const char* e = DDT_KNOB("DDT_NO_L2HINT");
         return !(e && e[0] == '1');
     }();
     return on;

@@ -184,8 +184,8 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
     const int ub = force_ub > 0 ? force_ub : choose_ub(b, sm_count);
     uint64_t items = 0;
     for (const auto& d : b.descs) items += desc_items(d, ub);
-    const char* ga = getenv("DDT_GROUP_ALWAYS");  // tests: exercise grouping on small plans
-    const char* sp = getenv("DDT_SPREAD");  // 0: group equal requests instead of spreading every request
+    const char* ga = DDT_KNOB("DDT_GROUP_ALWAYS");  // tests: exercise grouping on small plans
+    const char* sp = DDT_KNOB("DDT_SPREAD");  // 0: group equal requests instead of spreading every request
     const bool many = items > 8ull * (uint64_t)sm_count;
     bool spread = false;
     if (many && !(sp && sp[0] == '0')) spread = spread_items(b, ub);
@@ -594,7 +594,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     // test hook (never set in production): route self messages through the
     // window path instead of DirectIPC, so single-GPU tests and benchmarks
     // exercise and time the multi-GPU protocols
-    const char* svw = getenv("DDT_SELF_VIA_WINDOW");
+    const char* svw = DDT_KNOB("DDT_SELF_VIA_WINDOW");
     const bool self_window = p2p && !direct && svw && svw[0] == '1';
     auto remote = [&](int peer) { return peer != c->rank || self_window; };
 
@@ -608,7 +608,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             const auto& s = sends[i];
             if (s.count * s.type->size == 0 || !remote(s.peer)) continue;
             const int lw_s = std::min(4, side_lw(s.type, s.buf, s.count));
-            const char* nl = getenv("DDT_NO_LL");  // experiments: flag protocol only
+            const char* nl = DDT_KNOB("DDT_NO_LL");  // experiments: flag protocol only
             const int ll = (match[(size_t)i]->ll_ok && lw_s >= 3 && !(nl && nl[0] == '1')) ? 1 : 0;
             send_ll[{s.peer, s.tag}] = ll;
             lists[(size_t)s.peer].push_back({s.tag, ll});
@@ -791,10 +791,10 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             x.parity_stride = d.parity_stride;
             // same vector width on both sides => identical chunking: per-chunk flags
             // (DDT_CHUNK_FLAGS=0: experiments, release every flag at message end)
-            const char* cf = getenv("DDT_CHUNK_FLAGS");
+            const char* cf = DDT_KNOB("DDT_CHUNK_FLAGS");
             x.per_item = (lw == match[(size_t)i]->lw && !(cf && cf[0] == '0')) ? 1u : 0u;
             // the reader of this flag runs on our own device (self window): gpu scope suffices
-            const char* fs = getenv("DDT_FORCE_SYS_SCOPE");  // experiments: emulate a peer GPU's flags
+            const char* fs = DDT_KNOB("DDT_FORCE_SYS_SCOPE");  // experiments: emulate a peer GPU's flags
             x.gpu_scope = (s.peer == c->rank && !(fs && fs[0] == '1')) ? 1u : 0u;
             x.fanout = (uint32_t)match[(size_t)i]->nflags;  // else: all of the receiver's flags at the end
             xb.xinfo.push_back(x);
@@ -860,7 +860,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                 x.parity_stride = RL.parity_stride;
                 x.per_item = 1;
             }
-            const char* fs2 = getenv("DDT_FORCE_SYS_SCOPE");
+            const char* fs2 = DDT_KNOB("DDT_FORCE_SYS_SCOPE");
             x.gpu_scope = (r.peer == c->rank && !(fs2 && fs2[0] == '1')) ? 1u : 0u;  // the writer runs on this GPU
             xb.xinfo.push_back(x);
         }

@@ -28,6 +28,9 @@
 
 #include "ddt_internal.h"
 
+#include <atomic>
+#include <mutex>
+
 using namespace ddt;
 
 struct ddt_queue_s {
@@ -551,3 +554,27 @@ void queue_count_launches(ddt_queue_s* q, int64_t launches, int64_t bytes) {
     q->stats.bytes += bytes;
 }
 }  // namespace ddt
+
+// ---------------------------------------------------------------- knobs
+namespace ddt {
+namespace {
+std::mutex g_knob_mu;
+std::atomic<uint64_t> g_knob_gen{1};
+}  // namespace
+
+const char* KnobSlot::get() {
+    const uint64_t G = g_knob_gen.load(std::memory_order_relaxed);
+    if (gen.load(std::memory_order_acquire) != G) {
+        std::lock_guard<std::mutex> lk(g_knob_mu);
+        if (gen.load(std::memory_order_relaxed) != G) {
+            const char* v = getenv(name);
+            set = v != nullptr;
+            val = v ? v : "";
+            gen.store(G, std::memory_order_release);
+        }
+    }
+    return set ? val.c_str() : nullptr;
+}
+}  // namespace ddt
+
+extern "C" void ddt_reload_env(void) { ddt::g_knob_gen.fetch_add(1); }

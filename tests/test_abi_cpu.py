@@ -27,7 +27,7 @@ def ddt():
 
 def test_exports_every_header_symbol(ddt):
     hdr = open(os.path.join(ROOT, "include", "ddt.h")).read()
-    declared = set(re.findall(r"^\s*(?:ddt_status_t|int64_t|int32_t|const char\*)\s+(ddt_\w+)\s*\(", hdr, re.M))
+    declared = set(re.findall(r"^\s*(?:ddt_status_t|int64_t|int32_t|void|const char\*)\s+(ddt_\w+)\s*\(", hdr, re.M))
     assert len(declared) >= 40
     L = ctypes.CDLL(os.path.join(ROOT, "paper_conf_cluster_chukzsp20_b200", "libddt.so"))
     missing = [s for s in declared if not hasattr(L, s)]

@@ -36,6 +36,7 @@ CLASSES = {
 def build(arrays, dirs, knobs, nvars, local):
     for k, v in knobs.items():
         os.environ[k] = v
+    ddt.reload_env()
     try:
         msgs = halo_messages(0, 1, local, dirs=dirs, nvars=nvars)
         cache = {}
@@ -56,6 +57,7 @@ def build(arrays, dirs, knobs, nvars, local):
     finally:
         for k in knobs:
             os.environ.pop(k, None)
+        ddt.reload_env()
 
 
 def time_steps(plans, K):

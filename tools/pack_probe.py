@@ -42,10 +42,12 @@ def main():
         for ub in (None, 4, 2, 1):
             if ub:
                 os.environ["DDT_UB"] = str(ub)
+            ddt.reload_env()
             for b in range(B):
                 q.pack(t, src[b], 1, dst[b])
             plans["plan" if ub is None else f"plan_ub{ub}"] = ddt.Plan(q)
             os.environ.pop("DDT_UB", None)
+            ddt.reload_env()
         for k, p in plans.items():
             arms[k] = p.launch
         lib_arms = os.environ.get("PROBE_LIB_ARMS", "1") == "1"
