@@ -7,6 +7,7 @@
 #include <cuda_runtime.h>
 #include <chrono>
 #include <cstdio>
+#include <vector>
 
 template <int N> struct P { unsigned char b[N]; };
 template <int N> __global__ void k(const __grid_constant__ P<N> p) {
@@ -54,5 +55,32 @@ int main() {
         printf("{\"param_B\": 4096, \"pdl\": 1, \"event\": 1, \"host_us\": %.3f}\n", launch_us<4096>(s, true, true, e));
         printf("{\"param_B\": 16, \"pdl\": 1, \"event\": 1, \"host_us\": %.3f}\n", launch_us<16>(s, true, true, e));
     }
+    // other driver calls on the flush path
+    const int n = 20000;
+    std::vector<cudaEvent_t> evs(n);
+    auto t0 = std::chrono::steady_clock::now();
+    for (int i = 0; i < n; i++) cudaEventCreateWithFlags(&evs[i], cudaEventDisableTiming);
+    auto t1 = std::chrono::steady_clock::now();
+    printf("{\"call\": \"cudaEventCreateWithFlags\", \"host_us\": %.3f}\n",
+           std::chrono::duration<double, std::micro>(t1 - t0).count() / n);
+    for (int i = 0; i < n; i++) cudaEventRecord(evs[i], s);
+    cudaStreamSynchronize(s);
+    t0 = std::chrono::steady_clock::now();
+    for (int i = 0; i < n; i++) cudaEventQuery(evs[i]);
+    t1 = std::chrono::steady_clock::now();
+    printf("{\"call\": \"cudaEventQuery (complete)\", \"host_us\": %.3f}\n",
+           std::chrono::duration<double, std::micro>(t1 - t0).count() / n);
+    t0 = std::chrono::steady_clock::now();
+    int dev = 0;
+    for (int i = 0; i < n; i++) cudaGetDevice(&dev);
+    t1 = std::chrono::steady_clock::now();
+    printf("{\"call\": \"cudaGetDevice\", \"host_us\": %.3f}\n",
+           std::chrono::duration<double, std::micro>(t1 - t0).count() / n);
+    t0 = std::chrono::steady_clock::now();
+    for (int i = 0; i < n; i++) cudaGetLastError();
+    t1 = std::chrono::steady_clock::now();
+    printf("{\"call\": \"cudaGetLastError\", \"host_us\": %.3f}\n",
+           std::chrono::duration<double, std::micro>(t1 - t0).count() / n);
+    for (auto e : evs) cudaEventDestroy(e);
     return 0;
 }
