@@ -206,6 +206,28 @@ static bool narrow_list_batch(const HostBatch& b) {
     return list && b.xinfo.empty();
 }
 
+// Variant 10 (segment per thread): every request moves 4-B vectors between a
+// packed (contiguous) side and a uniform-list side whose segments hold the
+// same vps <= 4 vectors (<= 16 B: the sparse configs[2] shape), no response
+// slots.  Returns vps, or 0 if the batch does not qualify.
+static int segment_batch_vps(const HostBatch& b) {
+    const char* off = DDT_KNOB("DDT_NO_SEG");  // experiments
+    if ((off && off[0] == '1') || !b.xinfo.empty()) return 0;
+    uint32_t vps = 0;
+    for (const ReqDesc& S : b.descs) {
+        if (!S.nvec) continue;
+        const ReqDesc& D = b.aux[S.aux];
+        if (S.resp || S.lw != 2 || D.lw != 2 || S.ph || D.ph) return 0;
+        const bool s_list = S.kind == K_UNIFORM32 || S.kind == K_UNIFORM64;
+        const bool d_list = D.kind == K_UNIFORM32 || D.kind == K_UNIFORM64;
+        const ReqDesc& L = s_list ? S : D;
+        if (s_list == d_list || (s_list ? D.kind : S.kind) != K_CONTIG) return 0;
+        if (L.vps.d == 0 || L.vps.d > 4 || (vps && L.vps.d != vps)) return 0;
+        vps = L.vps.d;
+    }
+    return (int)vps;
+}
+
 int choose_ub(const HostBatch& b, int sm_count) {
     const char* env = DDT_KNOB("DDT_UB");
     if (env && (atoi(env) == 1 || atoi(env) == 2 || atoi(env) == 4 || atoi(env) == 8)) {
@@ -325,6 +347,19 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
     size_t n = std::max(b.descs.size(), b.aux.size());
     out.variant = batch_variant(b);
     out.ub = force_ub > 0 ? force_ub : choose_ub(b, sm_count);
+    if (const int vps = force_ub > 0 ? 0 : segment_batch_vps(b)) {
+        // an item = kThreads x kSegUnroll whole segments (fewer if that leaves < 2 items per SM)
+        out.variant = 10;
+        out.ub = vps;
+        for (int su : {kSegUnroll, 2}) {
+            uint64_t items = 0;
+            for (const auto& d : b.descs) items += desc_items(d, vps * su);
+            if (items >= 2ull * (uint64_t)sm_count) {
+                out.ub = vps * su;
+                break;
+            }
+        }
+    }
     const char* v9 = DDT_KNOB("DDT_NO_V9");  // experiments
     if (out.variant == 7 && out.ub == 1 && !(v9 && v9[0] == '1')) out.variant = 9;
     out.grid_mode = grid_mode_for(b, out.ub, sm_count);

@@ -23,6 +23,7 @@ constexpr int kThreads = 256;        // threads per CTA of the fused kernel
 constexpr int kUnroll = 4;           // max vectors per thread per item (loads in flight)
 constexpr int kItemVecs = kThreads * kUnroll;  // max vectors per work item
 constexpr int kUnrollNarrow = 8;     // 4-B-vector batches (variant 8): twice the loads in flight
+constexpr int kSegUnroll = 4;        // variant 10: whole segments per thread per item
 // A batch picks ub in {1, 2, 4} vectors per thread per item: small batches use
 // smaller items so that their work spreads over all 148 SMs (latency-bound
 // regime), large batches use kUnroll for memory-level parallelism.

@@ -421,6 +421,60 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
     if (win_s || win_d) __syncthreads();  // the next item may restage the window
 }
 
+// Variant 10: one whole segment of vps (<= 4) 4-B vectors per thread and
+// round (batch.cpp segment_batch_vps): one list lookup per segment instead of
+// one per vector, and the segment's words load back to back from the same
+// thread (one L2 sector fetch, L1 hits after the first).  The item covers
+// vectors [v0, v0 + kThreads * ub) = segments [v0 / vps, ...) (ub = vps * rounds).
+// One side is the uniform list, the other the packed (contiguous) side.
+template <int SR>
+__device__ __forceinline__ void run_seg(const ReqDesc& S, const ReqDesc& D, uint32_t v0, int ub, bool pdlw) {
+    const bool s_list = S.kind != K_CONTIG;
+    const ReqDesc& L = s_list ? S : D;
+    const uint32_t vps = L.vps.d;
+    const uint32_t nsegs = S.nvec / vps;
+    const uint32_t s0 = v0 / vps;
+    const int rounds = ub / (int)vps;
+    const uint8_t* src = reinterpret_cast<const uint8_t*>(S.ptr);
+    uint8_t* dst = reinterpret_cast<uint8_t*>(D.ptr);
+    const bool h64 = S.l2_64 != 0;
+    int64_t loff[SR];
+#pragma unroll
+    for (int u = 0; u < SR; u++) {  // list offsets (independent loads, all issued first)
+        const uint32_t sg = s0 + (uint32_t)(u * kThreads) + threadIdx.x;
+        loff[u] = 0;
+        if (u < rounds && sg < nsegs) {
+            const uint32_t k = divu(sg, L.nseg);
+            const uint32_t j = sg - k * L.nseg.d;
+            const int64_t o = L.kind == K_UNIFORM32 ? (int64_t)__ldg(reinterpret_cast<const int32_t*>(L.list) + j)
+                                                    : (int64_t)__ldg(reinterpret_cast<const long long*>(L.list) + j);
+            loff[u] = (int64_t)k * L.extent + o;  // list offsets are relative to the side's pointer
+        }
+    }
+    if (pdlw) pdl_wait();
+    uint32_t w[SR][4];
+#pragma unroll
+    for (int u = 0; u < SR; u++) {
+        const uint32_t sg = s0 + (uint32_t)(u * kThreads) + threadIdx.x;
+        if (u < rounds && sg < nsegs) {
+            const uint8_t* p = src + (s_list ? loff[u] : (int64_t)sg * vps * 4);
+#pragma unroll
+            for (int c = 0; c < 4; c++)
+                if (c < (int)vps) w[u][c] = ld_vec<true, 2>(p + 4 * c, 2, h64).x;
+        }
+    }
+#pragma unroll
+    for (int u = 0; u < SR; u++) {
+        const uint32_t sg = s0 + (uint32_t)(u * kThreads) + threadIdx.x;
+        if (u < rounds && sg < nsegs) {
+            uint8_t* p = dst + (s_list ? (int64_t)sg * vps * 4 : loff[u]);
+#pragma unroll
+            for (int c = 0; c < 4; c++)
+                if (c < (int)vps) st_vec<2>(p + 4 * c, 2, make_uint4(w[u][c], 0u, 0u, 0u));
+        }
+    }
+}
+
 // Largest r with prefix[r] <= item (prefix strictly increasing, prefix[0] = 0).
 __device__ __forceinline__ uint32_t find_request(const uint32_t* prefix, uint32_t nreq, uint32_t item) {
     uint32_t lo = 0, hi = nreq;
@@ -525,7 +579,7 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // batch is in the parameters: wait for the preceding grid just before the
 // first global-memory access (the first item's data loads).
 template <bool XCHG, int LW, bool SONLY, bool GW, bool PH, bool INPLACE = false, int UNR = kUnroll,
-          bool LAZYW = false>
+          bool LAZYW = false, bool SEG = false>
 __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa) {
     __shared__ ReqDesc sd;
     __shared__ ReqDesc sa;
@@ -641,8 +695,12 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             }
             if (trace && threadIdx.x == 0) tr1 = globaltimer();
         }
-        if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, (int)tv.ub, xa,
-                                                          (uint32_t)epoch, !waited);
+        if constexpr (SEG && !XCHG) {
+            run_seg<kSegUnroll>(*S, *D, v0, (int)tv.ub, !waited);
+        } else {
+            if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, (int)tv.ub, xa,
+                                                              (uint32_t)epoch, !waited);
+        }
         waited = true;
         if constexpr (!XCHG) {
             if (S->resp) {  // scheduler (3): the CTA finishing the request's last item signals it
@@ -727,8 +785,11 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
 // such as configs[2] are latency x concurrency bound, not bandwidth bound).
 // 9 = variant 7 for one vector per thread per item (ub = 1: latency-bound
 // halo steps such as configs[1]): no unrolled load slots, a short hot path.
+// 10 = segment per thread (run_seg): uniform-list <-> packed batches of <= 16-B
+// segments moved as 4-B words (batch.cpp segment_batch_vps).
 template <int V> struct VarT {
-    static constexpr int LW = (V == 0 || V == 6 || V == 7 || V == 9) ? -1 : (V == 8 ? 2 : V - 1);
+    static constexpr bool SEG = V == 10;
+    static constexpr int LW = (V == 0 || V == 6 || V == 7 || V == 9) ? -1 : ((V == 8 || V == 10) ? 2 : V - 1);
     static constexpr int UNR = V == 8 ? kUnrollNarrow : (V == 9 ? 1 : kUnroll);
     static constexpr bool SONLY = (V >= 1 && V <= 5) || V == 7 || V == 9;
     static constexpr bool GW = V == 6;
@@ -738,23 +799,23 @@ template <int V> struct VarT {
     // almost every item and needs the extra CTAs to keep loads in flight
     // (tools/pack_probe.py: 1 MiB x 1024 packs 4.74 -> 6.08 TB/s from 3 to 5
     // CTAs/SM); exchange kernels (flags, tracing) keep their registers.
-    static constexpr int MINB = (V == 7 || V == 9) ? DDT_V7_MINB : (V == 8 ? DDT_V8_MINB : DDT_MINB);
-    static constexpr int XMINB = (V == 7 || V == 9) ? DDT_V7_MINB : (V == 8 ? DDT_V8_MINB : DDT_XMINB);
+    static constexpr int MINB = (V == 7 || V == 9) ? DDT_V7_MINB : ((V == 8 || V == 10) ? DDT_V8_MINB : DDT_MINB);
+    static constexpr int XMINB = (V == 7 || V == 9) ? DDT_V7_MINB : ((V == 8 || V == 10) ? DDT_V8_MINB : DDT_XMINB);
 };
 
 template <int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_dev(const uint8_t* __restrict__ table) {
     pdl_trigger();
     pdl_wait();  // the table may come from a copy just before this launch
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(table),
-                                                                                                  nullptr);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR, false,
+               VarT<V>::SEG>(view_of(table), nullptr);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
     pdl_trigger();
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_PARAM, VarT<V>::UNR, true>(
-        view_of(pb), nullptr);
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_PARAM, VarT<V>::UNR, true,
+               VarT<V>::SEG>(view_of(pb), nullptr);
 }
 
 template <int V>
@@ -879,6 +940,7 @@ int launch_fused_form(int form, int variant, const void* src, uint32_t total_ite
     case 7: launch_fused_v<7>(form, src, total_items, s, grid_cap); break;
     case 8: launch_fused_v<8>(form, src, total_items, s, grid_cap); break;
     case 9: launch_fused_v<9>(form, src, total_items, s, grid_cap); break;
+    case 10: launch_fused_v<10>(form, src, total_items, s, grid_cap); break;
     default: launch_fused_v<0>(form, src, total_items, s, grid_cap); break;
     }
     return (int)cudaGetLastError();

@@ -271,6 +271,39 @@ def test_grid_modes_bit_exact_and_reusable(ddt, mode, monkeypatch):
     qq.destroy()
 
 
+@pytest.mark.parametrize("blk,base,count,shuffled", [(3, "float", 1, False), (3, "float", 2, True),
+                                                     (2, "int32", 3, False), (4, "float", 1, True),
+                                                     (1, "int32", 2, False), (3, "float", 1, "far")])
+def test_segment_per_thread_variant(ddt, blk, base, count, shuffled):
+    """Variant 10 (one whole <= 16-B segment per thread, uniform lists; DESIGN.md
+    §7k) for pack and unpack in one batch each, several segment sizes, count > 1,
+    shuffled block order and int64 offsets ("far": displacements beyond 2^31)."""
+    import torch
+    rng = np.random.default_rng(77 + blk)
+    n = 3000
+    npts = 1 << 15
+    idx = np.sort(rng.choice(npts, n, replace=False))
+    if shuffled is True:
+        rng.shuffle(idx)
+    disp = [int(i) * 4 * blk for i in idx]
+    if shuffled == "far":
+        disp = [d + (1 << 31) for d in disp]
+    spec = ("hindexed", [blk] * n, disp, ("basic", base))
+    cases = [Case(ddt, spec, count=count, misalign=4 * k, seed=700 + k) for k in range(3)]
+    q = ddt.Queue()
+    outs = [c.gpu_pack(q) for c in cases]
+    q.flush()
+    q.wait()
+    for c, (_, _, d) in zip(cases, outs):
+        assert_bytes_equal(host(d), c.expect_pack(), f"segment pack blk={blk}")
+    outs = [c.gpu_unpack(q) for c in cases]
+    q.flush()
+    q.wait()
+    for c, (_, _, d) in zip(cases, outs):
+        assert_bytes_equal(host(d), c.expect_unpack(), f"segment unpack blk={blk}")
+    q.destroy()
+
+
 def test_zero_size_and_empty_requests(ddt, q):
     import torch
     t = ddt.Type.from_spec(("vector", 0, 3, 2, ("basic", "double")))
