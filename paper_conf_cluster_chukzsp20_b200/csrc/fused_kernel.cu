@@ -32,6 +32,9 @@
 #ifndef DDT_INPLACE_PARAM
 #define DDT_INPLACE_PARAM true
 #endif
+#ifndef DDT_INPLACE_DEV
+#define DDT_INPLACE_DEV false
+#endif
 #ifndef DDT_MINB
 #define DDT_MINB 5
 #endif
@@ -807,7 +810,7 @@ template <int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_dev(const uint8_t* __restrict__ table) {
     pdl_trigger();
     pdl_wait();  // the table may come from a copy just before this launch
-    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR, false,
+    fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_DEV, VarT<V>::UNR, false,
                VarT<V>::SEG>(view_of(table), nullptr);
 }
 
