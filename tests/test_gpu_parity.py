@@ -304,6 +304,42 @@ def test_segment_per_thread_variant(ddt, blk, base, count, shuffled):
     q.destroy()
 
 
+def test_pdl_launches_respect_stream_order(ddt):
+    """Programmatic dependent launch keeps every stream
+    dependency: 40 rounds of [torch kernel writes the source] -> [ddt pack
+    flush] -> [ddt unpack flush of that packed buffer] -> [torch kernel reads
+    the result], all on one stream with no host synchronisation, each round's
+    bytes checked afterwards against the oracle (a PDL kernel that ran ahead of
+    its predecessor would read the previous round's values)."""
+    import torch
+    spec = ("subarray", [20, 24, 28], [18, 22, 1], [1, 1, 26], "C", ("basic", "double"))
+    o = oracle.Type(spec)
+    t = ddt.Type.from_spec(spec)
+    lo, hi = o.footprint(1)
+    q = ddt.Queue()
+    src = torch.empty(hi + 64, dtype=torch.uint8, device="cuda")
+    pk = torch.empty(o.size, dtype=torch.uint8, device="cuda")
+    out = torch.empty(hi + 64, dtype=torch.uint8, device="cuda")
+    snaps = []
+    for k in range(40):
+        src.fill_((7 * k + 3) & 0xFF)                # torch kernel writes the source
+        src[k: k + 8].fill_(k)                       # and a second, dependent one
+        out.fill_(0xA5)
+        q.pack(t, src, 1, pk)
+        q.flush()                                    # reads src
+        q.unpack(t, pk, 1, out)
+        q.flush()                                    # reads pk written by the previous kernel
+        snaps.append(out.clone())                    # torch kernel reads the result
+    torch.cuda.synchronize()
+    for k, got in enumerate(snaps):
+        s_host = np.full(hi + 64, (7 * k + 3) & 0xFF, np.uint8)
+        s_host[k: k + 8] = k
+        exp = np.full(hi + 64, 0xA5, np.uint8)
+        oracle.unpack(o, oracle.pack(o, s_host), exp)
+        assert_bytes_equal(host(got), exp, f"round {k}")
+    q.destroy()
+
+
 def test_zero_size_and_empty_requests(ddt, q):
     import torch
     t = ddt.Type.from_spec(("vector", 0, 3, 2, ("basic", "double")))
