@@ -181,14 +181,27 @@ ddt_status_t upload(const std::vector<uint8_t>& host, void** dev) {
 // batch such as configs[1] only pays the extra lookup, 3.5 -> 3.75 us).
 ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub = 0) {
     phase_batch(b);
-    const int ub = force_ub > 0 ? force_ub : choose_ub(b, sm_count);
+    int ub = force_ub > 0 ? force_ub : choose_ub(b, sm_count);
     uint64_t items = 0;
     for (const auto& d : b.descs) items += desc_items(d, ub);
     const char* ga = DDT_KNOB("DDT_GROUP_ALWAYS");  // tests: exercise grouping on small plans
     const char* sp = DDT_KNOB("DDT_SPREAD");  // 0: group equal requests instead of spreading every request
     const bool many = items > 8ull * (uint64_t)sm_count;
     bool spread = false;
-    if (many && !(sp && sp[0] == '0')) spread = spread_items(b, ub);
+    if (many && !(sp && sp[0] == '0')) {
+        // spread plans run one CTA per item (batch.cpp grid_mode_for): with one
+        // vector per thread they get the most CTAs in flight and the one-slot
+        // kernel (variant 9 for phased batches) -- COMB P = 1 116.6 -> 101.6 us
+        // -- when some request has short segments (x faces: DRAM-access bound);
+        // all-dense plans keep the large items (COMB dense faces alone: 16 us at
+        // ub 4, 28.5 us at ub 1)
+        bool sparse = false;
+        for (const ReqDesc& d : b.descs) sparse |= d.l2_64 || b.aux[d.aux].l2_64;
+        const char* su = DDT_KNOB("DDT_SPREAD_UB");  // experiments: item size of spread plans
+        const int sub = force_ub > 0 ? ub : (su ? std::max(1, std::min(4, atoi(su))) : (sparse ? 1 : ub));
+        spread = spread_items(b, sub);
+        if (spread) ub = sub;
+    }
     if (!spread && (many || (ga && ga[0] == '1'))) group_equal_requests(b, ub);
     make_launchable(b, !spread, l, sm_count, ub);
     if (l.form != 3) return DDT_OK;
