@@ -325,7 +325,8 @@ static int batch_variant(const HostBatch& b) {
 // Work distribution of a multi-wave plain batch (>= kTicketMinItemsPerSM
 // items per SM, no exchange flags; exchange batches keep the static order their
 // flag protocol is proven for).  Measured on one B200:
-//   * spread halo plans (COMB): one CTA per item (grid_mode 2) -- 128 -> 116 us;
+//   * spread halo plans (COMB) and sparse batches: one CTA per item (grid_mode 2)
+//     -- COMB 128 -> 116 us, configs[2] 32 x 10^5 x 12 B 55 -> 52 us;
 //   * <= kTicketMaxReqs large requests: dynamic tickets (grid_mode 1) --
 //     16 x 64 MiB packs 5.5 -> 6.4 TB/s;
 //   * many requests (1024 x 1 MiB): the static cyclic order stays best.
@@ -338,7 +339,9 @@ static int grid_mode_for(const HostBatch& b, int ub, int sm_count) {
     uint64_t items = 0;
     for (const ReqDesc& d : b.descs) items += desc_items(d, ub);
     if (items < (uint64_t)kTicketMinItemsPerSM * (uint64_t)sm_count) return 0;
-    int m = !b.order.empty() ? 2 : (b.descs.size() <= (size_t)kTicketMaxReqs ? 1 : 0);
+    bool sparse = false;  // short-segment sides (sparse lists, halo x faces): DRAM-access bound
+    for (const ReqDesc& d : b.descs) sparse |= d.l2_64 || b.aux[d.aux].l2_64;
+    int m = (!b.order.empty() || sparse) ? 2 : (b.descs.size() <= (size_t)kTicketMaxReqs ? 1 : 0);
     if (e && e[0] >= '0' && e[0] <= '2') m = e[0] - '0';
     return (m == 1 && !b.ticket) ? 0 : m;
 }
