@@ -351,10 +351,14 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
     out.variant = batch_variant(b);
     out.ub = force_ub > 0 ? force_ub : choose_ub(b, sm_count);
     if (const int vps = force_ub > 0 ? 0 : segment_batch_vps(b)) {
-        // an item = kThreads x kSegUnroll whole segments (fewer if that leaves < 2 items per SM)
+        // an item = kThreads x r0 whole segments (fewer if that leaves < 2 items per SM)
         out.variant = 10;
         out.ub = vps;
-        for (int su : {kSegUnroll, 2}) {
+        const char* sr = DDT_KNOB("DDT_SEG_ROUNDS");  // experiments: segments per thread per item
+        // 12-16-B segments: 2 per thread (more CTAs in flight; configs[2] sorted 52 -> 50 us,
+        // shuffled 69 -> 58 us); 4-8-B segments: 4 (struct-on-indexed 4-B blocks 75 vs 89 us at 2)
+        const int r0 = sr ? std::max(1, std::min(kSegUnroll, atoi(sr))) : (vps >= 3 ? 2 : kSegUnroll);
+        for (int su : {r0, 1}) {
             uint64_t items = 0;
             for (const auto& d : b.descs) items += desc_items(d, vps * su);
             if (items >= 2ull * (uint64_t)sm_count) {
