@@ -392,6 +392,48 @@ def pack_roofline(ddt, torch, hbm_peak, reps=20):
             "kernel": "ddt_fused_pack_unpack", "bytes_per_launch": 2 * best["S"] * best["B"], "cells": cells}
 
 
+def sparse_roofline(ddt, torch, hbm_peak, flush_buf, reps=20):
+    """configs[2]: fused pack of B = 32 requests of the sparse hindexed layout
+    (10^5 x 12-B blocks each), persistent plan, L2 flushed before every
+    launch; kernel time from CUDA events.  Algorithmic bytes = 2S per request;
+    the DRAM traffic of the same launch (64-B access granularity) comes from
+    the committed ncu capture (profiles/ncu_traffic.json, configs[2])."""
+    from ddt_inputs import config3_spec
+    B = 32
+    spec, nb = config3_spec()
+    t = ddt.Type.from_spec(spec)
+    src = torch.empty((B, nb), dtype=torch.uint8, device="cuda")
+    src.random_(0, 256)
+    dst = torch.empty((B, t.size), dtype=torch.uint8, device="cuda")
+    q = ddt.Queue()
+    q.enqueue_many("pack", t, list(src), 1, list(dst))
+    plan = ddt.Plan(q)
+    stream = torch.cuda.current_stream()
+    for _ in range(3):
+        plan.launch()
+    times = []
+    for k in range(reps):
+        flush_buf.fill_(k & 0xFF)
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        plan.launch()
+        b.record(stream)
+        torch.cuda.synchronize()
+        times.append(a.elapsed_time(b) / 1e3)
+    tmed = statistics.median(times)
+    alg = 2.0 * t.size * B
+    traffic = traffic_from_profiles("ddt_fused_*", "configs[2]")
+    out = {"workload": "configs[2]: 32 x hindexed(10^5 x 12 B), sorted, L2 flushed", "us": round(tmed * 1e6, 2),
+           "alg_gbs": round(alg / tmed / 1e9, 1), "alg_frac": round(alg / tmed / 1e9 / hbm_peak, 3),
+           "traffic": traffic, "bound": "hbm (64-B DRAM access granularity)"}
+    if traffic:
+        out["traffic_gbs"] = round(traffic / tmed / 1e9, 1)
+        out["traffic_frac"] = round(traffic / tmed / 1e9 / hbm_peak, 3)
+    plan.destroy()
+    q.destroy()
+    return out
+
+
 # ------------------------------------------------------------------ CPU oracle
 def oracle_exchange_sample(local, dirs, nvars, P, budget_s):
     """The CPU oracle (test infrastructure, plain C, 1 core) on the same halo
@@ -664,6 +706,7 @@ def main():
             if rank == 0:
                 extras["pack_roofline"] = pack_roofline(ddt, torch, hbm)
                 extras["pack_roofline"]["peak_source"] = peak_src
+                extras["sparse_roofline"] = sparse_roofline(ddt, torch, hbm, flush_buf)
         except Exception as e:
             extras["pack_roofline"] = {"error": f"{type(e).__name__}: {e}"}
         try:
@@ -681,6 +724,7 @@ def main():
                                 "local": list(loc), "messages_per_rank": wl4.nmsgs, "us_per_iter": round(ms4 * 1e3, 2),
                                 "alg_hbm_gbs": round(wl4.alg_bytes / (ms4 / 1e3) / 1e9, 1),
                                 "alg_bytes_per_rank": wl4.alg_bytes,
+                                "dram_traffic_per_launch": traffic_from_profiles("ddt_fused_*", "configs[3]"),
                                 "remote_bytes_out_per_rank": wl4.S_remote,
                                 "nvlink_bound_us": round(wl4.S_remote / 900e9 * 1e6, 2),
                                 "launches_per_iter": wl4.launches, "mode": best_mode,
