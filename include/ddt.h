@@ -158,7 +158,11 @@ ddt_status_t ddt_get_overlaps(ddt_type_t t, int32_t* overlaps);
 /* ------------------------------------------------------------------ queue
  * A queue = the paper's request list + scheduler bound to one
  * device and one CUDA stream (cudaStream_t passed as void*, NULL = legacy
- * default stream).  capacity = ring size (0 => 4096, R11).
+ * default stream).  capacity = ring size (0 => 4096, R11).  Every launch
+ * made through a queue (flushes, its plans, its halo plans) goes to that
+ * stream; when such launches are captured into CUDA graphs, replays must stay
+ * ordered with each other (large batches share the queue's work-ticket
+ * counter, device_desc.h).
  * Errors: DDT_ERR_NODEV, DDT_ERR_CUDA, DDT_ERR_NOMEM, DDT_ERR_ARG.          */
 ddt_status_t ddt_queue_create(int device, void* cuda_stream, int32_t capacity, ddt_queue_t* out);
 /* Waits for in-flight work, then frees the queue. */
