@@ -724,7 +724,8 @@ def main():
                                 "local": list(loc), "messages_per_rank": wl4.nmsgs, "us_per_iter": round(ms4 * 1e3, 2),
                                 "alg_hbm_gbs": round(wl4.alg_bytes / (ms4 / 1e3) / 1e9, 1),
                                 "alg_bytes_per_rank": wl4.alg_bytes,
-                                "dram_traffic_per_launch": traffic_from_profiles("ddt_fused_*", "configs[3]"),
+                                "dram_traffic_per_launch": (traffic_from_profiles("ddt_fused_*", "configs[3]")
+                                                            if P == 1 else None),
                                 "remote_bytes_out_per_rank": wl4.S_remote,
                                 "nvlink_bound_us": round(wl4.S_remote / 900e9 * 1e6, 2),
                                 "launches_per_iter": wl4.launches, "mode": best_mode,
