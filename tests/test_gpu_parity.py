@@ -340,6 +340,31 @@ def test_pdl_launches_respect_stream_order(ddt):
     q.destroy()
 
 
+def test_ring_reclaim_with_many_inflight_batches(ddt):
+    """A 64-slot ring driven by 300 one-request flushes with no host wait: the
+    ring fills repeatedly and enqueue reclaims completed batches (newest-first
+    query + binary search over the in-order batches); every uid ends COMPLETED
+    and every packed result equals the oracle."""
+    import torch
+    qq = ddt.Queue(capacity=64)
+    spec = config1_spec()
+    o = oracle.Type(spec)
+    t = ddt.Type.from_spec(spec)
+    srcs = [random_bytes(8192, 1200 + i) for i in range(8)]
+    d_src = [cuda_bytes(x) for x in srcs]
+    outs = torch.full((300, o.size), SENTINEL, dtype=torch.uint8, device="cuda")
+    uids = []
+    for i in range(300):
+        uids.append(qq.pack(t, d_src[i % 8], 1, outs[i]))
+        assert qq.flush() == 1
+    qq.wait()
+    assert all(qq.query(u) == "completed" for u in uids)
+    got = outs.cpu().numpy()
+    for i in range(300):
+        assert_bytes_equal(got[i], oracle.pack(o, srcs[i % 8]), f"request {i}")
+    qq.destroy()
+
+
 def test_zero_size_and_empty_requests(ddt, q):
     import torch
     t = ddt.Type.from_spec(("vector", 0, 3, 2, ("basic", "double")))
