@@ -115,7 +115,10 @@ struct alignas(16) XInfo {
 // Exchange plans chunk every message in items of kThreads * kXchgUb vectors on
 // both sides, so a receiver's unpack item k depends only on the sender's pack
 // item k (per-chunk flags: unpack of a message overlaps its packing).
-constexpr int kXchgUb = 2;
+#ifndef DDT_XCHG_UB
+#define DDT_XCHG_UB 2
+#endif
+constexpr int kXchgUb = DDT_XCHG_UB;
 
 // General lists: a CTA work item stages the prefix / offset entries of the
 // segments it touches in shared memory (found through the skip table, whose

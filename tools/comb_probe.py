@@ -51,7 +51,8 @@ def build(arrays, dirs, knobs, nvars, local):
         for arrs in arrays:
             sends = [(m["peer"], m["tag"], T(m["send_spec"]), arrs[m["var"]], 1) for m in msgs]
             recvs = [(m["recv_peer"], m["recv_tag"], T(m["recv_spec"]), arrs[m["var"]], 1) for m in msgs]
-            plans.append(ddt.Halo(q, ddt.Comm.single(0), sends, recvs, mode="nccl", graph=True))
+            mode = os.environ.get("PROBE_MODE", "nccl")  # p2p + DDT_SELF_VIA_WINDOW=1: the exchange kernel
+            plans.append(ddt.Halo(q, ddt.Comm.single(0), sends, recvs, mode=mode, graph=(mode == "nccl")))
         S = sum(T(m["send_spec"]).size for m in msgs)
         return q, plans, S, len(msgs)
     finally:
