@@ -368,7 +368,9 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
         }
     }
     const char* v9 = DDT_KNOB("DDT_NO_V9");  // experiments
-    if (out.variant == 7 && out.ub == 1 && !(v9 && v9[0] == '1')) out.variant = 9;
+    bool multi = false;  // a request with its own item size > 1 needs the multi-slot kernel
+    for (const ReqDesc& d : b.descs) multi |= d.xub > 1;
+    if (out.variant == 7 && out.ub == 1 && !multi && !(v9 && v9[0] == '1')) out.variant = 9;
     out.grid_mode = grid_mode_for(b, out.ub, sm_count);
     out.ticket = out.grid_mode == 1 ? b.ticket : 0;
     const char* force = DDT_KNOB("DDT_FORCE_TABLE");  // experiments: always use the device-table form

@@ -133,7 +133,7 @@ int side_lw(ddt_type_s* t, const void* p, int64_t count);
 ddt_status_t alloc_base(const void* p, void** base);
 // Items of a descriptor at ub vectors per thread per item.
 inline uint32_t desc_items(const ReqDesc& d, int ub = kUnroll) {
-    uint64_t per = (uint64_t)kThreads * (uint64_t)ub;
+    uint64_t per = (uint64_t)kThreads * (uint64_t)(d.xub ? d.xub : ub);  // exchange requests carry their own
     uint64_t n = (d.nvec + per - 1) / per;
     return n ? (uint32_t)n : 1u;  // a data-free (signal / wait) request still owns one item
 }

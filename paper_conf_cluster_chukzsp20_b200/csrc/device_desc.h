@@ -75,7 +75,8 @@ struct alignas(16) ReqDesc {
     uint32_t nitems;        // items of this request in its batch (set at flush)
     uint8_t ph;             // phased 16-B units (kPh*), 0 = plain vectors; see below
     uint8_t l2_64;          // 1: short segments (< kSparseSeg B) -> loads carry the .L2::64B prefetch-size hint
-    uint8_t pad3[2];
+    uint8_t xub;            // exchange plans: this request's vectors per thread per item (0 = the batch's ub)
+    uint8_t pad3;
 };
 
 // Phased units (batch.cpp phase_batch).  A closed-form request whose common
@@ -119,6 +120,12 @@ struct alignas(16) XInfo {
 #define DDT_XCHG_UB 2
 #endif
 constexpr int kXchgUb = DDT_XCHG_UB;
+// A flagged message's chunk (item) size is a function of its byte size alone,
+// so sender and receiver -- whose plans differ -- chunk it identically:
+// messages that may travel in LL size (<= kLLMaxBytes) use 1 vector per thread
+// per item (twice the items in flight for latency-bound halos; configs[1]
+// window protocol 7.3 -> 5.7 us), larger ones kXchgUb.
+inline int xchg_ub_for(int64_t bytes) { return bytes <= kLLMaxBytes ? 1 : kXchgUb; }
 
 // General lists: a CTA work item stages the prefix / offset entries of the
 // segments it touches in shared memory (found through the skip table, whose

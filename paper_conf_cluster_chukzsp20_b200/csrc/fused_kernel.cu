@@ -666,7 +666,8 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             }
             cur = r;
         }
-        const uint32_t v0 = local * (uint32_t)(kThreads * tv.ub);
+        const int ubr = XCHG && S->xub ? (int)S->xub : (int)tv.ub;  // exchange requests carry their own item size
+        const uint32_t v0 = local * (uint32_t)(kThreads * ubr);
         bool run = true;
         uint64_t tr0 = 0, tr1 = 0, tr2 = 0;
         if constexpr (XCHG) {
@@ -701,7 +702,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         if constexpr (SEG && !XCHG) {
             run_seg<kSegUnroll>(*S, *D, v0, (int)tv.ub, !waited);
         } else {
-            if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, (int)tv.ub, xa,
+            if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, ubr, xa,
                                                               (uint32_t)epoch, !waited);
         }
         waited = true;

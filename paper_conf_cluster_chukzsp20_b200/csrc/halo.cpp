@@ -70,10 +70,10 @@ RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs, bool reserve_ll 
     L.nflags.assign((size_t)nrecv, 1);
     L.ll_ok.assign((size_t)nrecv, 0);
     int64_t off = 0, nflag = 0;
-    const int64_t chunk = (int64_t)kThreads * kXchgUb;  // vectors per exchange item
     for (size_t k = 0; k < L.order.size(); k++) {
         int i = L.order[k];
         int64_t bytes = recvs[i].count * recvs[i].type->size;
+        const int64_t chunk = (int64_t)kThreads * xchg_ub_for(bytes);  // vectors per exchange item
         off = round_up(off, kAlign);
         L.data_off[(size_t)i] = off;
         int lw = recvs[i].type->committed ? std::min(4, side_lw(recvs[i].type, recvs[i].buf, recvs[i].count)) : 0;
@@ -790,6 +790,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                     st = build_ll(OP_PACK, s.type, dl, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count,
                                   &sd, &dd);
                 if (st != DDT_OK) break;
+                sd.xub = (uint8_t)xchg_ub_for(s.count * s.type->size);  // no flags: free to pick the item size
                 xb.add(sd, dd);
                 XInfo x{};
                 x.parity_stride = d.parity_stride;
@@ -798,6 +799,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             }
             int lw = 0;
             st = add_req(xb, s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, &lw);
+            if (st == DDT_OK) xb.descs.back().xub = (uint8_t)xchg_ub_for(s.count * s.type->size);
             XInfo x{};
             x.signal = (uint64_t)(uintptr_t)(win + 8 * match[(size_t)i]->flag_idx);
             x.counter = npack++;
@@ -864,12 +866,14 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                     st = build_ll(OP_UNPACK, r.type, dl, r.buf, mywin + RL.flags_bytes + RL.data_off[(size_t)i],
                                   r.count, &sd, &dd);
                 if (st != DDT_OK) break;
+                sd.xub = (uint8_t)xchg_ub_for(r.count * r.type->size);
                 xb.add(sd, dd);
                 x.wait = 0;
                 x.parity_stride = RL.parity_stride;
             } else {  // unpack chunk k as soon as the sender's chunk k has landed
                 st = add_req(xb, r.type, OP_UNPACK, mywin + RL.flags_bytes + RL.data_off[(size_t)i], r.buf, r.count,
                              nullptr);
+                if (st == DDT_OK) xb.descs.back().xub = (uint8_t)xchg_ub_for(r.count * r.type->size);
                 x.parity_stride = RL.parity_stride;
                 x.per_item = 1;
             }
