@@ -843,6 +843,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             if (st == DDT_OK && sd.nvec != dd.nvec) st = DDT_ERR_SIZE_MISMATCH;
             if (st != DDT_OK) break;
             sd.op = dd.op = OP_DIRECT;
+            sd.xub = (uint8_t)xchg_ub_for(s.count * s.type->size);  // one done flag per message: any chunking
             xb.add(sd, dd);
             XInfo x{};
             x.signal = (uint64_t)(uintptr_t)((char*)c->peer_windows[s.peer] + 8 * e.flag_idx);
