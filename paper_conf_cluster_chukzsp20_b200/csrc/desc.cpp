@@ -155,18 +155,15 @@ static void contig_desc(const void* p, uint32_t nvec, int lw, ReqDesc* d) {
 
 ddt_status_t build_request(int op, ddt_type_s* t, const DeviceLayout* dl, const void* src, const void* dst,
                            int64_t count, ReqDesc* s, ReqDesc* d) {
-    std::memset(s, 0, sizeof(*s));
-    std::memset(d, 0, sizeof(*d));
     const void* nc = op == OP_PACK ? src : dst;  // the typed side
     const void* pk = op == OP_PACK ? dst : src;  // the packed side
     int lw = std::min(side_lw(t, nc, count), log2i(lowbit16((uint64_t)(uintptr_t)pk)));
-    ReqDesc lay, con;
-    std::memset(&lay, 0, sizeof(lay));
-    ddt_status_t st = layout_desc(t, dl, nc, count, lw, &lay);
+    ReqDesc* lay = op == OP_PACK ? s : d;  // built in place: no temporaries
+    ReqDesc* con = op == OP_PACK ? d : s;
+    std::memset(lay, 0, sizeof(*lay));
+    ddt_status_t st = layout_desc(t, dl, nc, count, lw, lay);
     if (st != DDT_OK) return st;
-    contig_desc(pk, lay.nvec, lw, &con);
-    *s = op == OP_PACK ? lay : con;
-    *d = op == OP_PACK ? con : lay;
+    contig_desc(pk, lay->nvec, lw, con);
     s->op = (uint8_t)op;
     d->op = (uint8_t)op;
     return DDT_OK;

@@ -159,8 +159,8 @@ int64_t claim(ddt_queue_s* q) {
     return q->tail;
 }
 
-int64_t commit_req(ddt_queue_s* q, int op, ddt_type_s* t, ddt_type_s* t2, int64_t bytes, const ReqDesc& d,
-                   const ReqDesc& a) {
+// Publish the Tail slot, whose desc/aux the caller has already written in place.
+int64_t commit_slot(ddt_queue_s* q, int op, ddt_type_s* t, ddt_type_s* t2, int64_t bytes) {
     int64_t uid = q->tail++;
     auto& r = q->ring[(size_t)(uid % q->capacity)];
     r.uid = uid;
@@ -170,9 +170,7 @@ int64_t commit_req(ddt_queue_s* q, int op, ddt_type_s* t, ddt_type_s* t2, int64_
     type_retain(t);
     type_retain(t2);
     r.bytes = bytes;
-    r.desc = d;
     r.desc.uid_lo = (uint32_t)uid;
-    r.aux = a;
     if (q->resp_on && bytes > 0) {
         size_t slot = (size_t)(uid % q->capacity);
         r.desc.resp = (uint64_t)(uintptr_t)(q->resp_dev + slot);
@@ -185,6 +183,14 @@ int64_t commit_req(ddt_queue_s* q, int op, ddt_type_s* t, ddt_type_s* t2, int64_
     return uid;
 }
 
+int64_t commit_req(ddt_queue_s* q, int op, ddt_type_s* t, ddt_type_s* t2, int64_t bytes, const ReqDesc& d,
+                   const ReqDesc& a) {
+    auto& r = q->ring[(size_t)(q->tail % q->capacity)];
+    r.desc = d;
+    r.aux = a;
+    return commit_slot(q, op, t, t2, bytes);
+}
+
 int64_t enqueue(ddt_queue_s* q, int op, ddt_type_s* t, const void* src, int64_t count, void* dst) {
     if (!q || !t || count < 0) return DDT_ERR_ARG;
     if (q->sticky != DDT_OK) return q->sticky;
@@ -194,17 +200,19 @@ int64_t enqueue(ddt_queue_s* q, int op, ddt_type_s* t, const void* src, int64_t 
     if (op == OP_UNPACK && bytes > 0 && instances_overlap(t, count)) return DDT_ERR_OVERLAP;
     int64_t c = claim(q);
     if (c < 0) return c;
-    ReqDesc sd, dd;
-    std::memset(&sd, 0, sizeof(sd));
-    std::memset(&dd, 0, sizeof(dd));
+    // build straight into the free Tail slot (it is only published by commit_slot)
+    auto& r = q->ring[(size_t)(c % q->capacity)];
     if (bytes > 0) {
         DeviceLayout* dl = nullptr;
         ddt_status_t s = type_device_layout(t, q->device, &dl);
         if (s != DDT_OK) return s;
-        s = build_request(op, t, dl, src, dst, count, &sd, &dd);
+        s = build_request(op, t, dl, src, dst, count, &r.desc, &r.aux);
         if (s != DDT_OK) return s;
+    } else {
+        std::memset(&r.desc, 0, sizeof(r.desc));
+        std::memset(&r.aux, 0, sizeof(r.aux));
     }
-    return commit_req(q, op, t, nullptr, bytes, sd, dd);
+    return commit_slot(q, op, t, nullptr, bytes);
 }
 
 ddt_status_t ensure_host_slot(ddt_queue_s* q, size_t bytes, ddt_queue_s::HostSlot** out) {
