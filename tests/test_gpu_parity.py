@@ -388,6 +388,24 @@ def test_oversized_request_rejected(ddt, q):
     assert e.value.code == -10
 
 
+def test_failed_enqueue_publishes_nothing(ddt):
+    """Enqueue builds the descriptors in place in the free Tail slot; a request
+    that fails while being built must leave the ring untouched: the next uid is
+    unchanged and the next request (same slot) packs bit-exactly."""
+    q1 = ddt.Queue(capacity=2)
+    c = Case(ddt, config1_spec(), 3, 8, 0)
+    big = ddt.Type.from_spec(("contiguous", 1 << 33, ("basic", "byte")))
+    u0, _, d0 = c.gpu_pack(q1)
+    assert q1.try_pack(big, 1, 1, 3) == -10  # DDT_ERR_UNSUPPORTED while building the Tail slot
+    u1, _, d1 = c.gpu_pack(q1)
+    assert (u0, u1) == (0, 1)
+    assert q1.flush() == 2
+    q1.wait()
+    for d in (d0, d1):
+        assert_bytes_equal(host(d), c.expect_pack(), "pack after a failed enqueue")
+    q1.destroy()
+
+
 def test_nan_and_negative_zero_survive(ddt, q):
     import torch
     vals = np.array([np.nan, -0.0, np.inf, -np.inf, 5e-324, 1.0] * 40, dtype=np.float64)
