@@ -117,8 +117,11 @@ ddt_status_t ddt_create_hindexed_block(int64_t count, int64_t blocklen, const in
                                        ddt_type_t* out);
 /* struct: block i = blocklens[i] copies of types[i] at byte displacement
  * displs_bytes[i] (+ j * extent(types[i])).  Heterogeneous blocks (e.g. the
- * paper's struct-on-indexed specfem3D_cm layout).  No alignment epsilon
- * is added to the upper bound (reading R2): use ddt_create_resized to pad. */
+ * paper's struct-on-indexed specfem3D_cm layout).  The upper bound carries
+ * MPI's alignment increment epsilon (MPI-3.1 §4.1; reading R2): the extent is
+ * rounded up to a multiple of the largest basic-type alignment (= its size) in
+ * the typemap, e.g. {(double,0),(byte,8)} has extent 16 -- unless a block's
+ * type has explicit bounds (resized / subarray beneath it), which then rule. */
 ddt_status_t ddt_create_struct(int64_t count, const int64_t* blocklens, const int64_t* displs_bytes,
                                const ddt_type_t* types, ddt_type_t* out);
 /* resized (MPI-3.1 §4.1.7): the typemap of `old` with lb / extent replaced;

@@ -33,8 +33,11 @@ Spec tuples (the neutral input language both sides parse independently):
     ("resized", old, lb, extent)
 
 Parity status: every function here is pinned by tests/test_oracle_pins.py
-(numpy slicing / as_strided / concatenation, closed forms, brute-force
-self-describing buffers, round-trip invariants, the config-1 golden file).
+(numpy slicing / as_strided / concatenation, closed forms incl. oldtypes with
+lb != 0, numpy align=True records for the struct alignment epsilon,
+brute-force self-describing buffers, round-trip invariants, the config-1 and
+struct-alignment golden files; run_batch by numpy slicing / assignment on
+shared buffers).
 """
 from __future__ import annotations
 

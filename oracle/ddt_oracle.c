@@ -25,7 +25,14 @@
  *   hindexed(n,B,D,old):for i<n, for j<B[i]: copy of old at D[i] + j*ext(old)
  *   contiguous(n,old):  for i<n: copy of old at i*ext(old)
  *   struct(n,B,D,T[]):  for i<n, for j<B[i]: copy of T[i] at D[i] + j*ext(T[i])
- *                       (byte displacements; no alignment epsilon, DESIGN R2)
+ *                       (byte displacements).  ub carries the alignment
+ *                       increment epsilon (MPI-3.1 §4.1, "ub(Typemap) = max_j
+ *                       (disp_j + sizeof(type_j)) + epsilon", epsilon = the
+ *                       least non-negative increment that rounds the extent to
+ *                       a multiple of max_i k_i, k_i = alignment of basic type
+ *                       i = its size here) unless the typemap carries explicit
+ *                       bounds markers (a resized or subarray type beneath it,
+ *                       MPI-3.1 §4.1.6-4.1.7).  DESIGN.md reading R2.
  *   resized(old,lb,ex): the typemap of old with lb / extent set to (lb, ex)
  *                       (MPI-3.1 §4.1.7); true bounds stay those of the entries
  *   subarray(nd,sizes,subsizes,starts,order,old): C order = dim 0 outermost,
@@ -36,7 +43,8 @@
  *     (MPI-3.1 §4.1.3).
  *   lb / ub: min / max over every placed (non-empty) copy of the oldtype of
  *     copy_disp + lb(old) / copy_disp + ub(old); basic: [0, sizeof).  Empty
- *     type: lb = ub = 0 (reading R3).  No alignment epsilon (R2).
+ *     type: lb = ub = 0 (reading R3).  Alignment epsilon: struct
+ *     only (R2, see above); k is found by enumerating the struct's entries.
  *   true lb / ub: min / max over the actual basic entries.
  *   pack(src,count,T,out): instance k at k*extent(T); entries copied in
  *     typemap order to consecutive packed positions (R1, R8, R9).
@@ -279,6 +287,27 @@ static void orc_bacc_add(orc_bacc *b, int64_t lo, int64_t hi) {
     b->any = 1;
 }
 
+/* Explicit lb / ub markers somewhere in the tree (resized, subarray). */
+static int orc_has_markers(const orc_type *t) {
+    switch (t->kind) {
+    case OK_BASIC: return 0;
+    case OK_RESIZED: case OK_SUBARRAY: return 1;
+    case OK_STRUCT:
+        for (int64_t i = 0; i < t->nblocks; i++)
+            if (orc_has_markers(t->types[i])) return 1;
+        return 0;
+    default: return orc_has_markers(t->old);
+    }
+}
+
+/* max_i k_i over the basic entries of a typemap: every emitted entry is one
+ * basic element whose alignment equals its size (1, 4 or 8 bytes). */
+static void orc_align_emit(void *ctx, int64_t disp, int64_t nbytes) {
+    (void)disp;
+    int64_t *k = (int64_t *)ctx;
+    if (nbytes > *k) *k = nbytes;
+}
+
 static int orc_bounds(const orc_type *t, int64_t *lb, int64_t *ub) {
     if (t->kind == OK_BASIC) { *lb = 0; *ub = t->elem_size; return 1; }
     if (t->kind == OK_SUBARRAY) {
@@ -313,6 +342,13 @@ static int orc_bounds(const orc_type *t, int64_t *lb, int64_t *ub) {
         }
         if (!b.any) { *lb = 0; *ub = 0; return 0; }
         *lb = b.lo; *ub = b.hi;
+        if (!orc_has_markers(t)) { /* epsilon: round the extent up to a multiple of k */
+            int64_t k = 1;
+            orc_walk(t, 0, orc_align_emit, &k);
+            int64_t ext = b.hi - b.lo;
+            while (ext % k != 0) ext++;
+            *ub = b.lo + ext;
+        }
         return 1;
     }
     int64_t olb, oub;

@@ -95,6 +95,8 @@ struct ddt_type_s {
     // closed-form properties (computed at construction)
     bool nonempty = false;
     int64_t size = 0, lb = 0, ub = 0, true_lb = 0, true_ub = 0;
+    int64_t align = 1;    // max alignment (= size) of the basic types in the typemap (struct epsilon, R2)
+    bool sticky = false;  // explicit lb / ub markers beneath (resized, subarray): no epsilon (MPI-3.1 §4.1.6)
     bool has_form = false;
     ddt::Form form;  // normalized strided form if derivable (any number of dims)
 

@@ -131,6 +131,7 @@ static void init_basic() {
         t->ub = sz[i];
         t->true_lb = 0;
         t->true_ub = sz[i];
+        t->align = sz[i];
         t->has_form = true;
         t->form.base = 0;
         t->form.seg_len = sz[i];
@@ -145,6 +146,8 @@ static void derive_from_copies(ddt_type_s* t, int64_t ncopies, int64_t min_disp,
     ddt_type_s* o = t->old;
     t->size = ncopies * o->size;
     t->nonempty = ncopies > 0 && o->nonempty;
+    t->align = o->align;
+    t->sticky = o->sticky;
     if (!t->nonempty) {
         t->lb = t->ub = t->true_lb = t->true_ub = 0;
         t->has_form = true;
@@ -244,6 +247,7 @@ static void derive_subarray(ddt_type_s* t) {
         for (int k = nd - 1; k >= 0; k--) dims.push_back({t->subsizes[k], mult[k]});
     }
     derive_from_copies(t, ncopies, mn, mx, mn, &dims);
+    t->sticky = true;  // defined with explicit bounds (MPI-3.1 §4.1.3)
     // resized: lb 0, extent prod(sizes) * E (true bounds are the entries')
     if (t->nonempty) {
         t->lb = 0;
@@ -252,16 +256,22 @@ static void derive_subarray(ddt_type_s* t) {
 }
 
 // struct: block i = blocklens[i] copies of types[i] at displs[i] + j*ext(types[i])
-// (byte displacements, MPI-3.1 §4.1.2; no alignment epsilon, reading R2).
+// (byte displacements, MPI-3.1 §4.1.2).  Alignment epsilon (reading R2): ub is
+// rounded up so that the extent is a multiple of the largest basic alignment in
+// the typemap, unless a child carries explicit bounds (resized / subarray).
 static void derive_struct(ddt_type_s* t) {
     bool any = false;
     int64_t lb = 0, ub = 0, tlb = 0, tub = 0;
     t->size = 0;
+    t->align = 1;
+    t->sticky = false;
     for (size_t i = 0; i < t->blocklens.size(); i++) {
         const ddt_type_s* o = t->types[i];
         int64_t B = t->blocklens[i];
         t->size += B * o->size;
+        t->sticky |= o->sticky;
         if (B <= 0 || !o->nonempty) continue;
+        t->align = std::max(t->align, o->align);
         int64_t E = type_extent(o), d = t->displs[i];
         int64_t blo = d + o->lb, bhi = d + (B - 1) * E + o->ub;
         int64_t tlo = d + o->true_lb, thi = d + (B - 1) * E + o->true_ub;
@@ -280,6 +290,10 @@ static void derive_struct(ddt_type_s* t) {
     }
     t->lb = lb;
     t->ub = ub;
+    if (!t->sticky) {
+        const int64_t ext = ub - lb;
+        t->ub += (t->align - ext % t->align) % t->align;  // epsilon
+    }
     t->true_lb = tlb;
     t->true_ub = tub;
     // one non-empty block of a closed-form oldtype is itself closed-form
@@ -426,6 +440,8 @@ ddt_status_t ddt_create_resized(ddt_type_t old, int64_t lb, int64_t extent, ddt_
     auto* t = new_derived(T_RESIZED, old);
     t->size = old->size;
     t->nonempty = old->nonempty;
+    t->align = old->align;
+    t->sticky = true;  // explicit lb / ub markers (MPI-3.1 §4.1.7)
     t->lb = lb;
     t->ub = lb + extent;
     t->true_lb = old->true_lb;

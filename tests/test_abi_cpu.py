@@ -124,6 +124,19 @@ def test_closed_forms_match_oracle_enumeration(ddt, spec):
     assert t.overlaps == (len(b) != len(set(b))), spec
 
 
+def test_struct_alignment_golden_library(ddt):
+    """The library's closed-form struct bounds (alignment epsilon, R2) against
+    the hand-derived golden values (tests/golden/struct_alignment.json)."""
+    import json
+    from test_oracle_pins import _spec_from_json
+    g = json.load(open(os.path.join(ROOT, "tests", "golden", "struct_alignment.json")))
+    for case in g["cases"]:
+        t = ddt.Type.from_spec(_spec_from_json(case["spec"]))
+        assert t.size == case["size"], case["name"]
+        assert list(t.extent()) == [case["lb"], case["extent"]], case["name"]
+        assert list(t.true_extent()) == [case["true_lb"], case["true_extent"]], case["name"]
+
+
 def test_layout_kinds(ddt):
     t = ddt.Type.from_spec(config1_spec())
     assert t.layout_kind == "strided" and t.num_segments == 16

@@ -179,6 +179,59 @@ def test_mixed_batch_one_launch_equals_sequential_oracle(ddt, q):
         assert_bytes_equal(host(d), exp, f"batch item {i}")
 
 
+def test_shared_buffer_batch_equals_oracle_run_batch(ddt, q):
+    """One fused launch of 48 packs of mixed layouts into disjoint slices of ONE
+    packed buffer, then one launch of 48 unpacks from ONE packed buffer into
+    disjoint regions of ONE destination array: byte-equal to oracle.run_batch
+    (the requests executed one by one on the host, R6)."""
+    import torch
+    specs = [config1_spec(), ("subarray", [9, 10, 11], [3, 4, 5], [1, 2, 3], "C", ("basic", "double")),
+             ("hindexed", [3, 1, 2], [100, 4, 37], ("basic", "byte")),
+             ("struct", [1, 2, 1], [0, 8, 24], [("basic", "byte"), ("basic", "double"), ("basic", "int32")]),
+             ("vector", 5, 3, -4, ("basic", "int64"))]
+    rng = np.random.default_rng(11)
+    src = random_bytes(1 << 20, 12)
+    ots = [oracle.Type(sp) for sp in specs]
+    tts = [ddt.Type.from_spec(sp) for sp in specs]
+    reqs, pk_off, src_offs = [], 16, []
+    for i in range(48):
+        k = i % len(specs)
+        cnt = int(rng.integers(1, 4))
+        lo, hi = ots[k].footprint(cnt)
+        so = int(rng.integers(0, (1 << 20) - (hi - lo) - 64)) - lo
+        reqs.append(dict(op="pack", type=ots[k], count=cnt, src=src, src_offset=so, dst=None, dst_offset=pk_off, k=k))
+        pk_off += cnt * ots[k].size + int(rng.integers(0, 9))
+    packed_h = np.full(pk_off + 64, SENTINEL, np.uint8)
+    for r in reqs:
+        r["dst"] = packed_h
+    s_d = cuda_bytes(src)
+    p_d = torch.full((pk_off + 64,), SENTINEL, dtype=torch.uint8, device="cuda")
+    l0 = q.stats()["launches"]
+    for r in reqs:
+        q.pack(tts[r["k"]], (s_d, r["src_offset"]), r["count"], (p_d, r["dst_offset"]))
+    assert q.flush() == 48
+    oracle.run_batch([{k: v for k, v in r.items() if k != "k"} for r in reqs])
+    q.wait()
+    assert q.stats()["launches"] - l0 == 1
+    assert_bytes_equal(host(p_d), packed_h, "shared packed buffer")
+    # unpacks: instances placed back to back (disjoint footprints) in one array
+    dst_h = np.full(1 << 21, SENTINEL, np.uint8)
+    ureqs, pos = [], 128
+    for r in reqs:
+        t = r["type"]
+        lo, hi = t.footprint(r["count"])
+        ureqs.append(dict(op="unpack", type=t, count=r["count"], src=packed_h, src_offset=r["dst_offset"],
+                          dst=dst_h, dst_offset=pos - lo, k=r["k"]))
+        pos += (hi - lo) + 8
+    d_d = torch.full((1 << 21,), SENTINEL, dtype=torch.uint8, device="cuda")
+    for r in ureqs:
+        q.unpack(tts[r["k"]], (p_d, r["src_offset"]), r["count"], (d_d, r["dst_offset"]))
+    q.flush()
+    oracle.run_batch([{k: v for k, v in r.items() if k != "k"} for r in ureqs])
+    q.wait()
+    assert_bytes_equal(host(d_d), dst_h, "shared destination array")
+
+
 def test_queue_full_gives_negative_uid_then_recovers(ddt):
     import torch
     q4 = ddt.Queue(capacity=4)

@@ -29,11 +29,21 @@ def _labels(nbytes_elems: int, elem=8):
 
 
 def _spec_from_json(j):
-    if isinstance(j, list) and j and j[0] == "basic":
-        return ("basic", j[1])
-    if isinstance(j, list):
-        return tuple(_spec_from_json(x) if isinstance(x, list) and x and isinstance(x[0], str) else x for x in j)
-    return j
+    """JSON lists -> spec tuples (a spec is a list whose first item is its kind;
+    a struct's oldtypes are a list of specs)."""
+    def is_spec(x):
+        return isinstance(x, list) and bool(x) and isinstance(x[0], str)
+    if not is_spec(j):
+        return j
+    out = [j[0]]
+    for x in j[1:]:
+        if is_spec(x):
+            out.append(_spec_from_json(x))
+        elif isinstance(x, list) and x and all(is_spec(y) for y in x):
+            out.append([_spec_from_json(y) for y in x])
+        else:
+            out.append(x)
+    return tuple(out)
 
 
 # ------------------------------------------------------------ golden config 1
@@ -182,6 +192,97 @@ def test_indexed_matches_concatenation(data):
     parts = [src[off + s: off + s + b * esz] for s, b in zip(starts, bl)]
     expect = np.concatenate(parts) if parts else np.zeros(0, np.uint8)
     np.testing.assert_array_equal(got, expect)
+
+
+@HSET
+@given(c=st.integers(1, 5), b=st.integers(1, 4), stride=st.integers(-5, 6), olb=st.integers(-24, 24),
+       extra=st.integers(0, 24))
+def test_vector_over_nonzero_lb_oldtype_closed_form(c, b, stride, olb, extra):
+    """vector(c, b, stride, old) with old = resized(double, olb, E): the MPI
+    closed form (SURVEY §8(c) pins) lb = min(0,(c-1)S) + min(0,(b-1)E) +
+    lb(old), ub = max(0,(c-1)S) + max(0,(b-1)E) + ub(old), S = stride*E, with
+    lb(old) = olb != 0; the entries (the double at offset 0 of every copy) pin
+    the copy spacing through numpy's as_strided."""
+    E = 8 + extra
+    old = ("resized", ("basic", "double"), olb, E)
+    t = oracle.Type(("vector", c, b, stride, old))
+    lb, ub = _vector_closed_bounds(c, b, stride * E, E, olb=olb, oub=olb + E)
+    assert t.extent() == (lb, ub - lb)
+    lo = min(0, (c - 1) * stride * E)                      # lowest entry byte
+    src = random_bytes(((c - 1) * abs(stride) + b) * E + 64, 13)
+    off = -lo
+    view = np.lib.stride_tricks.as_strided(src[off:], shape=(c, b, 8), strides=(stride * E, E, 1))
+    np.testing.assert_array_equal(oracle.pack(t, src, src_offset=off), view.reshape(-1))
+
+
+@HSET
+@given(st.data())
+def test_indexed_over_nonzero_lb_oldtype_closed_form(data):
+    """indexed(B, D, old), old = resized(float, olb, E), blocks with B_i > 0:
+    lb = min_i(D_i E + min(0,(B_i-1)E)) + lb(old), ub = max_i(D_i E +
+    max(0,(B_i-1)E)) + ub(old) (SURVEY §8(c) pins), lb(old) != 0; the packed
+    bytes are the concatenated blocks (numpy slicing)."""
+    n = data.draw(st.integers(1, 5))
+    bl = [data.draw(st.integers(0, 3)) for _ in range(n)]
+    dl = [data.draw(st.integers(-4, 8)) for _ in range(n)]
+    olb = data.draw(st.integers(-12, 12))
+    E = 4 + data.draw(st.integers(0, 12))
+    t = oracle.Type(("indexed", bl, dl, ("resized", ("basic", "float"), olb, E)))
+    nz = [(d * E, b) for d, b in zip(dl, bl) if b > 0]
+    if nz:
+        lb = min(d + min(0, (b - 1) * E) for d, b in nz) + olb
+        ub = max(d + max(0, (b - 1) * E) for d, b in nz) + olb + E
+    else:
+        lb = ub = 0
+    assert t.extent() == (lb, ub - lb)
+    src = random_bytes(512, 17)
+    off = 200
+    parts = [np.lib.stride_tricks.as_strided(src[off + d * E:], shape=(b, 4), strides=(E, 1)).reshape(-1)
+             for d, b in zip(dl, bl)]
+    expect = np.concatenate(parts) if parts else np.zeros(0, np.uint8)
+    np.testing.assert_array_equal(oracle.pack(t, src, src_offset=off), expect)
+
+
+def test_run_batch_shared_buffers_match_numpy():
+    """oracle.run_batch (a fused batch executed request by request, SURVEY
+    §8(c) step 5): packs of three layouts into disjoint slices of ONE packed
+    buffer, then unpacks of the six faces of a 6x7x8 block from ONE packed
+    buffer into ONE array -- pinned by numpy slicing / assignment."""
+    a = random_bytes(6 * 7 * 8 * 8, 41).view(np.int64).reshape(6, 7, 8)
+    specs = [("subarray", [6, 7, 8], [1, 5, 6], [0, 1, 1], "C", ("basic", "int64")),
+             ("vector", 6, 1, 56, ("basic", "int64")),
+             ("hindexed", [2, 1], [64, 8], ("basic", "int64"))]
+    expect = [a[0:1, 1:6, 1:7].reshape(-1), a.reshape(-1)[0::56][:6], a.reshape(-1)[[8, 9, 1]]]
+    types = [oracle.Type(sp) for sp in specs]
+    packed = np.zeros(sum(t.size for t in types) + 16, np.uint8)
+    reqs, o = [], 8
+    for t in types:
+        reqs.append(dict(op="pack", type=t, count=1, src=a, dst=packed, dst_offset=o))
+        o += t.size
+    oracle.run_batch(reqs)
+    np.testing.assert_array_equal(packed[8:o].view(np.int64), np.concatenate(expect))
+    assert not packed[:8].any() and not packed[o:].any()
+    # unpack: the 6 interior faces of the block from consecutive packed slices
+    faces = [(slice(0, 1), slice(1, 6), slice(1, 7)), (slice(5, 6), slice(1, 6), slice(1, 7)),
+             (slice(1, 5), slice(0, 1), slice(1, 7)), (slice(1, 5), slice(6, 7), slice(1, 7)),
+             (slice(1, 5), slice(1, 6), slice(0, 1)), (slice(1, 5), slice(1, 6), slice(7, 8))]
+    fspecs = [("subarray", [6, 7, 8], [f.stop - f.start for f in fc], [f.start for f in fc], "C", ("basic", "int64"))
+              for fc in faces]
+    ftypes = [oracle.Type(sp) for sp in fspecs]
+    src = random_bytes(sum(t.size for t in ftypes), 42)
+    dst = np.full((6, 7, 8), -1, np.int64)
+    reqs, o = [], 0
+    for t in ftypes:
+        reqs.append(dict(op="unpack", type=t, count=1, src=src, src_offset=o, dst=dst))
+        o += t.size
+    oracle.run_batch(reqs)
+    ref = np.full((6, 7, 8), -1, np.int64)
+    o = 0
+    for fc, t in zip(faces, ftypes):
+        blk = ref[fc]
+        ref[fc] = src[o:o + t.size].view(np.int64).reshape(blk.shape)
+        o += t.size
+    np.testing.assert_array_equal(dst, ref)
 
 
 def test_indexed_typemap_order():
@@ -358,19 +459,22 @@ _NP = {"double": "<f8", "float": "<f4", "int32": "<i4", "int64": "<i8", "byte": 
 
 @HSET
 @given(st.data())
-def test_struct_matches_numpy_structured_dtype(data):
+def test_struct_matches_numpy_aligned_structured_dtype(data):
     """A struct of basic blocks is a numpy structured dtype with explicit field
-    offsets: packing `count` instances copies the fields, in field order, of
-    consecutive records of itemsize = extent (numpy implements the same
-    field-by-name copy)."""
+    offsets.  With ``align=True`` numpy lays records out like a C compiler:
+    itemsize = the end of the last field rounded up to the largest field
+    alignment -- MPI's alignment increment epsilon (MPI-3.1 §4.1: ub =
+    max(disp + sizeof) + epsilon, rounding the extent to a multiple of max k_i;
+    DESIGN R2).  numpy derives that itemsize itself; packing `count` records
+    copies the fields in typemap (not address) order."""
     n = data.draw(st.integers(1, 4))
     names, formats, offsets, bl, d, olds = [], [], [], [], [], []
-    pos = data.draw(st.integers(0, 8))
+    pos = 0
     for i in range(n):
-        base = data.draw(st.sampled_from(["double", "float", "int32", "byte"]))
+        base = data.draw(st.sampled_from(["double", "float", "int32", "int64", "byte"]))
         esz = oracle.BASIC_SIZES[base]
         b = data.draw(st.integers(1, 3))
-        pos = (pos + esz - 1) // esz * esz
+        pos = (pos + esz - 1) // esz * esz          # natural alignment (numpy requires it with align=True)
         names.append(f"f{i}")
         formats.append((_NP[base], (b,)))
         offsets.append(pos)
@@ -379,20 +483,51 @@ def test_struct_matches_numpy_structured_dtype(data):
     perm = data.draw(st.permutations(range(n)))          # typemap order != address order
     spec = ("struct", [bl[i] for i in perm], [d[i] for i in perm], [olds[i] for i in perm])
     t = oracle.Type(spec)
-    lo = min(d)
+    rec = np.dtype({"names": names, "formats": formats, "offsets": offsets}, align=True)
+    assert t.extent() == (0, rec.itemsize)
     hi = max(off + bb * oracle.BASIC_SIZES[o[1]] for off, bb, o in zip(d, bl, olds))
-    assert t.extent() == (lo, hi - lo)
+    assert t.true_extent() == (0, hi)
     count = data.draw(st.integers(1, 3))
-    # numpy record layout: the MPI buffer address is the record start minus lb
-    rec = np.dtype({"names": names, "formats": formats, "offsets": [o - lo for o in offsets], "itemsize": hi - lo})
     src = random_bytes(rec.itemsize * count + 16, 21)
     arr = np.frombuffer(src[: rec.itemsize * count].tobytes(), dtype=rec)
     packed_dt = np.dtype([(names[i], formats[i]) for i in perm])
     expect = np.empty(count, dtype=packed_dt)
     for i in perm:
         expect[names[i]] = arr[names[i]]
-    got = oracle.pack(t, np.concatenate([src, np.zeros(64, np.uint8)]), count, src_offset=-lo)
+    got = oracle.pack(t, src, count)
     np.testing.assert_array_equal(got, expect.view(np.uint8))
+
+
+def test_nested_struct_matches_numpy_nested_aligned_dtype():
+    """A struct holding a struct: the inner record's itemsize (its rounded
+    extent) is the spacing of its copies, and the outer alignment is the
+    largest basic alignment anywhere inside (numpy nested align=True)."""
+    inner_dt = np.dtype([("a", "<f8"), ("b", "u1")], align=True)                  # 16
+    outer_dt = np.dtype([("c", "u1"), ("s", inner_dt, (2,)), ("e", "<i4")], align=True)
+    inner = ("struct", [1, 1], [0, 8], [("basic", "double"), ("basic", "byte")])
+    off = [outer_dt.fields[k][1] for k in ("c", "s", "e")]
+    spec = ("struct", [1, 2, 1], off, [("basic", "byte"), inner, ("basic", "int32")])
+    t = oracle.Type(spec)
+    assert oracle.Type(inner).extent() == (0, inner_dt.itemsize)
+    assert t.extent() == (0, outer_dt.itemsize)
+    src = random_bytes(outer_dt.itemsize * 3, 77)
+    arr = np.frombuffer(src.tobytes(), dtype=outer_dt)
+    expect = b"".join(r["c"].tobytes() + b"".join(x["a"].tobytes() + x["b"].tobytes() for x in r["s"])
+                      + r["e"].tobytes() for r in arr)
+    assert oracle.pack(t, src, 3).tobytes() == expect
+
+
+def test_struct_alignment_golden():
+    """Hand-derived values (tests/golden/struct_alignment.json, each case cites
+    its source): MPI-3.1 §4.1's own example {(double,0),(char,8)} has extent 16."""
+    g = json.load(open(os.path.join(GOLD, "struct_alignment.json")))
+    for case in g["cases"]:
+        t = oracle.Type(_spec_from_json(case["spec"]))
+        assert t.size == case["size"], case["name"]
+        assert list(t.extent()) == [case["lb"], case["extent"]], case["name"]
+        assert list(t.true_extent()) == [case["true_lb"], case["true_extent"]], case["name"]
+        if "typemap_count2" in case:
+            assert t.typemap(2)[0].tolist() == case["typemap_count2"], case["name"]
 
 
 @HSET
