@@ -14,10 +14,12 @@ face (Alg 3, §IV-B).  Inputs larger than L2:
 steps rotate over R = 96 independent arrays + plans (DRAM footprint > 2x L2),
 so no step finds its data in L2.  W warm-up steps, then exactly K steps back to
 back between barrier + synchronize, timed by one CUDA-event pair; at N = 1 the
-K steps are one captured CUDA graph (a solver's captured time-step loop), at
-N > 1 they are issued from the host.  value = device time / K, max over ranks.
-modes.*.isolated_flushed_us adds the single-exchange view: events around each
-step, a 256 MiB L2 flush before it (includes that step's launch latency).
+K steps are one captured CUDA graph at every N (a solver's captured time-step
+loop; the P2P exchange keeps its epoch on the device), and a 256 MiB L2 read
+sweep runs right before the start event.  value = device time / K, max over
+ranks.  modes.*.isolated_flushed_us adds the single-exchange view: events
+around each step, an L2 read sweep before it (includes that step's launch
+latency).
 
 Extra measurements on the same JSON line (rank 0):
   pack_roofline  -- config 5 dense vector pack (S >= 1 MiB, B*S = 1 GiB cells):
@@ -180,7 +182,7 @@ def timed_steps(torch, wl, K, W, flush_buf, dist_on, sampler=None, flush=True):
     t0 = time.time()
     for k in range(K):
         if flush:
-            flush_buf.fill_(k & 0xFF)  # evict the working set from the 126 MB L2
+            l2_evict(torch, flush_buf)  # evict the working set from the 126 MB L2 (clean lines only)
         ev[k][0].record(stream)
         wl.step()
         ev[k][1].record(stream)
@@ -195,13 +197,28 @@ def timed_steps(torch, wl, K, W, flush_buf, dist_on, sampler=None, flush=True):
     return per, t1 - t0
 
 
-def run_steps(torch, wl, K, W, dist_on, sampler=None, capture=False):
+def l2_evict(torch, flush_buf):
+    """Evict the 126 MB L2 with a READ sweep of a 256 MiB buffer (one small
+    reduction kernel on the current stream): afterwards L2 holds only clean
+    lines of this buffer, so the next kernel finds none of its data in L2 and
+    pays no write-back of lines dirtied earlier (a fill_ flush would leave
+    126 MB of dirty lines to be written back during the timed region)."""
+    flush_buf.max()
+
+
+def run_steps(torch, wl, K, W, dist_on, sampler=None, capture=False, flush_buf=None):
     """The contract's timing: W untimed warm-up steps, then EXACTLY K steps back
     to back over the round-robin replicas, bracketed by barrier + synchronize on
     both sides and timed by one CUDA-event pair on the launching stream.
     capture=True records the K steps as one CUDA graph first (a time-step loop
     captured once, the way a solver would), so the per-step time is device time,
-    not Python launch rate.  Returns (ms per step, wall seconds)."""
+    not Python launch rate.  flush_buf: an L2 read sweep is enqueued just before
+    the start event, so (a) every replica the timed steps touch is cold in L2 --
+    including the replicas the untimed first replay (graph upload) just touched,
+    whatever K is -- and (b) the host submits the timed graph while the sweep
+    runs, so the K-step time does not contain the idle-GPU graph-launch latency
+    (the driver's K = 20 and a K = 500 run then agree).  Returns (ms per step,
+    wall seconds)."""
     stream = torch.cuda.current_stream()
     for _ in range(W):
         wl.step()
@@ -220,6 +237,8 @@ def run_steps(torch, wl, K, W, dist_on, sampler=None, capture=False):
         dist.barrier()
     torch.cuda.synchronize()
     t0 = time.time()
+    if flush_buf is not None:
+        l2_evict(torch, flush_buf)
     a.record(stream)
     if g is not None:
         g.replay()
@@ -321,7 +340,7 @@ def e2e_zero_copy(torch, ddt, rank, P, local, dirs, nvars, comm, mode, K, dist_o
     return ms, h2d, d2h
 
 
-def latency_floor(ddt, torch, K, R=96):
+def latency_floor(ddt, torch, K, flush_buf, R=96):
     """The launch + dependent-DRAM-round-trip floor of ONE fused launch, timed
     exactly like the configs[1] step: a K-step CUDA graph over R rotating
     buffers, each step one fused pack of the configs[0] vector (512 B, one
@@ -345,7 +364,7 @@ def latency_floor(ddt, torch, K, R=96):
         def step(self):
             plans[self.k % R].launch()
             self.k += 1
-    ms, _ = run_steps(torch, _W(), K, 10, False, None, capture=True)
+    ms, _ = run_steps(torch, _W(), K, 10, False, None, capture=True, flush_buf=flush_buf)
     for p in plans:
         p.destroy()
     q.destroy()
@@ -413,7 +432,7 @@ def sparse_roofline(ddt, torch, hbm_peak, flush_buf, reps=20):
         plan.launch()
     times = []
     for k in range(reps):
-        flush_buf.fill_(k & 0xFF)
+        l2_evict(torch, flush_buf)  # read sweep: no dirty lines left to write back inside the timed launch
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record(stream)
         plan.launch()
@@ -435,16 +454,34 @@ def sparse_roofline(ddt, torch, hbm_peak, flush_buf, reps=20):
 
 
 # ------------------------------------------------------------------ CPU oracle
-def oracle_exchange_sample(local, dirs, nvars, P, budget_s):
-    """The CPU oracle (test infrastructure, plain C, 1 core) on the same halo
-    workload, all P ranks simulated in one process; returns us per iteration
-    (transfer = in-process, pack + unpack timed)."""
+def host_cores():
+    return len(os.sched_getaffinity(0))
+
+
+def cpu_model():
+    try:
+        return next((ln.split(":", 1)[1].strip() for ln in open("/proc/cpuinfo") if ln.startswith("model name")), "?")
+    except Exception:
+        return "?"
+
+
+def oracle_exchange_sample(local, dirs, nvars, P, budget_s, threads=1, random_init=True, max_iters=None):
+    """The CPU oracle (test infrastructure, plain C) on the same halo workload,
+    all P ranks simulated in one process; returns (us per iteration, iterations,
+    threads used).  threads > 1: the messages of an exchange are split over a
+    thread pool ("a threaded run splitting requests across all
+    cores"; ctypes releases the GIL inside the C oracle) -- all packs, then all
+    unpacks (each writes its own ghost region); the oracle itself is untouched.
+    Transfer is in-process; pack + unpack are timed."""
     import oracle
+    from concurrent.futures import ThreadPoolExecutor
     shape = tuple(n + 2 for n in local)
     arrays, msgs = {}, []
     for r in range(P):
         for v in range(nvars):
-            arrays[(r, v)] = random_bytes(int(np.prod(shape)) * 8, seed(2, r * 10 + v)).view(np.int64).reshape(shape)
+            nb = int(np.prod(shape)) * 8
+            arrays[(r, v)] = (random_bytes(nb, seed(2, r * 10 + v)) if random_init
+                              else np.zeros(nb, np.uint8)).view(np.int64).reshape(shape)
     by_key = {}
     for r in range(P):
         for m in halo_messages(r, P, local, dirs=dirs, nvars=nvars):
@@ -462,15 +499,28 @@ def oracle_exchange_sample(local, dirs, nvars, P, budget_s):
             rm = by_key[(m["peer"], r, m["tag"])]
             msgs.append(dict(src_rank=r, dst_rank=m["peer"], var=m["var"], send=T(m["send_spec"]),
                              recv=T(rm["recv_spec"])))
+    threads = max(1, min(threads, len(msgs)))
+    ex = ThreadPoolExecutor(threads) if threads > 1 else None
+
+    def one():
+        if ex is None:
+            oracle.exchange(arrays, msgs)
+            return
+        packed = list(ex.map(lambda m: oracle.pack(m["send"], arrays[(m["src_rank"], m["var"])]), msgs))
+        list(ex.map(lambda mp: oracle.unpack(mp[0]["recv"], mp[1], arrays[(mp[0]["dst_rank"], mp[0]["var"])]),
+                    zip(msgs, packed)))
+    one()  # untimed: first touch of the arrays, type tables
     n = 0
     t0 = time.perf_counter()
     while True:
-        oracle.exchange(arrays, msgs)
+        one()
         n += 1
         el = time.perf_counter() - t0
-        if el >= budget_s:
+        if el >= budget_s or (max_iters and n >= max_iters):
             break
-    return el / n * 1e6, n
+    if ex is not None:
+        ex.shutdown()
+    return el / n * 1e6, n, threads
 
 
 def oracle_per_config(budget_s):
@@ -552,8 +602,9 @@ def main():
     config = {"workload": "configs[1]: 3D subarray face halo, 128^3 doubles per rank, 6 neighbors, dense layout",
               "per_rank_interior": list(local), "proc_grid": list(grid), "ghost": 1, "messages_per_rank": 6,
               "dtype_elem": "double (moved as raw bytes)",
-              "l2": ("inputs larger than L2: steps rotate over R independent arrays + plans whose DRAM "
-                     "footprint (R x ~4 MB) is > 2x the 126 MB L2")}
+              "l2": ("inputs larger than L2: steps rotate over R independent arrays + plans (R x ~4 MB > 2x "
+                     "the 126 MB L2), and L2 is evicted by a read sweep right before the timed steps, so no "
+                     "timed step finds its data in L2 at any K")}
 
     if args.impl == "reference":
         if rank != 0:
@@ -562,35 +613,45 @@ def main():
         # each step = one configs[1] exchange of ONE rank's messages (6 faces of a
         # 128^3 block: the per-rank work is the same at every N -- weak scaling).
         import oracle
+        from concurrent.futures import ThreadPoolExecutor
         shape = tuple(n + 2 for n in local)
         a = random_bytes(int(np.prod(shape)) * 8, seed(2, 0)).view(np.int64).reshape(shape)
         msgs = halo_messages(0, 1, local, dirs=FACE_DIRS)
         by_tag = {m["recv_tag"]: m for m in msgs}
         omsgs = [dict(src_rank=0, dst_rank=0, var=0, send=oracle.Type(m["send_spec"]),
                       recv=oracle.Type(by_tag[m["tag"]]["recv_spec"])) for m in msgs]
-        arrays = {(0, 0): a}
+        nc = host_cores()
+        thr = max(1, min(nc, len(omsgs)))  # the messages of a step split over the host's cores
+        ex = ThreadPoolExecutor(thr)
+
+        def step():
+            packed = list(ex.map(lambda m: oracle.pack(m["send"], a), omsgs))
+            list(ex.map(lambda mp: oracle.unpack(mp[0]["recv"], mp[1], a), zip(omsgs, packed)))
         budget = max(5.0, min(args.cpu_budget * 6, 120.0))
         t_start = time.perf_counter()
         for _ in range(args.warmup):
-            oracle.exchange(arrays, omsgs)
+            step()
             if time.perf_counter() - t_start > budget / 4:
                 break
         times = []
         t_start = time.perf_counter()
         for _ in range(args.steps):
             t0 = time.perf_counter()
-            oracle.exchange(arrays, omsgs)
+            step()
             times.append(time.perf_counter() - t0)
             if time.perf_counter() - t_start > budget:
                 break
+        ex.shutdown()
         per = sum(times) / len(times) * 1e6
         line = {"impl": "reference", "metric": METRIC, "value": round(per, 2), "unit": "us/iter", "n_gpus": N,
                 "steps": len(times), "warmup": args.warmup, "ms_per_step": round(per / 1e3, 4),
                 "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
                 "data": "synthetic (PCG64 random 64-bit patterns)", "config": dict(config, impl="cpu oracle"),
-                "cpu_baseline": {"value": round(per, 2), "unit": "us/iter", "cores": 1, "kind": "oracle",
-                                 "sample": f"{len(times)} timed oracle exchanges of one rank's 6 faces "
-                                           f"(plain C, 1 thread, {budget:.0f} s cap)"},
+                "cpu_baseline": {"value": round(per, 2), "unit": "us/iter", "cores": thr, "kind": "oracle",
+                                 "sample": (f"{len(times)} timed oracle exchanges of one rank's 6 faces (plain C "
+                                            f"oracle, messages split over {thr} threads on a {nc}-core host, "
+                                            f"{budget:.0f} s cap)"),
+                                 "cpu_model": cpu_model()},
                 "e2e": {"value": round(per, 2), "unit": "us/iter", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
         print(json.dumps(line), flush=True)
         return
@@ -626,10 +687,10 @@ def main():
     # K-step loop can be captured from it (capture needs a non-default stream)
     stream = torch.cuda.Stream()
     torch.cuda.set_stream(stream)
-    # N = 1: every message is a self message -> one DirectIPC kernel per step,
-    # capturable; N > 1: P2P plans carry a host-counted epoch as a kernel
-    # argument (not capturable), so steps are issued from the host
-    capture = not dist_on
+    # every plan is capturable (N = 1: one DirectIPC kernel per step; N > 1:
+    # the P2P exchange kernel keeps its epoch on the device, NCCL mode captures
+    # its send/recv), so the K steps are one captured CUDA graph at every N;
+    # a mode whose capture fails falls back to host-issued steps (reported)
     R = int(os.environ.get("DDT_BENCH_REPLICAS", "96"))
 
     results = {}
@@ -644,15 +705,27 @@ def main():
             # plan metadata: host all-gather over the process group; NCCL comm
             # only for the NCCL-mode data path
             c = ddt.Comm.from_torch(dev, nccl=(mode == "nccl")) if dist_on else ddt.Comm.single(dev)
-            wl = HaloWorkload(ddt, torch, rank, P, local, FACE_DIRS, 1, mode, c, 2, replicas=R, graph=not capture)
-            ms, wall = run_steps(torch, wl, args.steps, args.warmup, dist_on, sampler, capture=capture)
+            wl = HaloWorkload(ddt, torch, rank, P, local, FACE_DIRS, 1, mode, c, 2, replicas=R, graph=False)
+            capture = os.environ.get("DDT_BENCH_NO_CAPTURE") != "1"
+            try:
+                ms, wall = run_steps(torch, wl, args.steps, args.warmup, dist_on, sampler, capture=capture,
+                                     flush_buf=flush_buf)
+            except Exception as ce:  # capture refused: host-issued steps instead
+                if not capture:
+                    raise
+                torch.cuda.synchronize()
+                capture = False
+                capture_err = f"{type(ce).__name__}: {ce}"
+                ms, wall = run_steps(torch, wl, args.steps, args.warmup, dist_on, sampler, capture=False,
+                                     flush_buf=flush_buf)
             ms = max_over_ranks(torch, ms, dist_on)
             # the single-exchange view: events around each step, L2 flushed before it
             per, _ = timed_steps(torch, wl, max(50, args.steps // 5), 3, flush_buf, dist_on, None)
             iso_ms = max_over_ranks(torch, sum(per) / len(per), dist_on)
             qs = np.percentile(np.asarray(per), [10, 50, 90])
             results[mode] = dict(wl=wl, mean_ms=ms, iso_ms=iso_ms, iso_p50_ms=float(qs[1]), iso_p10_ms=float(qs[0]),
-                                 iso_p90_ms=float(qs[2]), comm=c, wall=wall)
+                                 iso_p90_ms=float(qs[2]), comm=c, wall=wall, capture=capture,
+                                 capture_err=None if capture else locals().get("capture_err"))
         except Exception as e:  # report, keep the other mode
             results[mode] = dict(error=f"{type(e).__name__}: {e}")
     ok = {m: r for m, r in results.items() if "error" not in r}
@@ -693,7 +766,7 @@ def main():
 
     if rank == 0 and not dist_on:
         try:
-            fl = latency_floor(ddt, torch, K)
+            fl = latency_floor(ddt, torch, K, flush_buf)
             roof["latency_floor"] = {"us": round(fl, 3), "value_over_floor": round(best["mean_ms"] * 1e3 / fl, 2),
                                      "what": "same K-step graph harness, one fused launch moving 512 B (configs[0] "
                                              "vector pack) from cold buffers: launch + one dependent DRAM round trip"}
@@ -737,10 +810,20 @@ def main():
 
     cpu = None
     if rank == 0 and N == 1 and not args.no_extras:
-        us, n = oracle_exchange_sample(local, FACE_DIRS, 1, 1, args.cpu_budget)
-        cpu = {"value": round(us, 2), "unit": "us/iter", "cores": 1, "kind": "oracle",
-               "sample": f"{n} iterations of the configs[1] face exchange (pack + unpack of 6 faces, P=1) "
-                         f"over ~{args.cpu_budget:.0f} s, plain C oracle, 1 thread",
+        nc = host_cores()
+        us_all, n_all, thr = oracle_exchange_sample(local, FACE_DIRS, 1, 1, args.cpu_budget / 2, threads=nc)
+        us1, n1, _ = oracle_exchange_sample(local, FACE_DIRS, 1, 1, args.cpu_budget / 4, threads=1)
+        # configs[3] COMB (P = 1: 104 + 104 messages over 4 x 514^3 arrays), all cores
+        usc, nc_it, thc = oracle_exchange_sample((512, 512, 512), ALL_DIRS, 4, 1, args.cpu_budget / 2, threads=nc,
+                                                 random_init=False, max_iters=50)
+        cpu = {"value": round(us_all, 2), "unit": "us/iter", "cores": thr, "kind": "oracle",
+               "sample": (f"{n_all} iterations of the configs[1] face exchange (pack + unpack of 6 faces, P=1) "
+                          f"over ~{args.cpu_budget / 2:.0f} s, plain C oracle, the 6 messages split over {thr} "
+                          f"threads (host has {nc} cores: at most one thread per message)"),
+               "cpu_model": cpu_model(), "host_cores": nc,
+               "one_core": {"value": round(us1, 2), "unit": "us/iter", "iterations": n1},
+               "comb26_allcores": {"value": round(usc, 2), "unit": "us/iter", "threads": thc, "iterations": nc_it,
+                                   "workload": "configs[3] P=1: 512^3 x 4 vars, 26 directions (104+104 msgs)"},
                "other_configs": oracle_per_config(max(3.0, args.cpu_budget / 2))}
 
     if rank == 0:
@@ -749,9 +832,11 @@ def main():
             "steps": K, "warmup": args.warmup, "ms_per_step": round(best["mean_ms"], 5),
             "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
             "data": "synthetic (seeded random int64 bit patterns)",
-            "config": dict(config, mode=best_mode, replicas=R,
-                           launch=("K-step CUDA graph (captured time-step loop)" if capture
-                                   else "host-issued, one ddt_exchange per step")),
+            "config": dict(config, mode=best_mode, replicas=R, distinct_replicas_timed=min(K, R),
+                           launch=("K-step CUDA graph (captured time-step loop)" if best["capture"]
+                                   else "host-issued, one ddt_exchange per step"),
+                           l2_evict=("256 MiB read sweep enqueued before the start event (L2 holds none of the "
+                                     "timed steps' data, no dirty lines to write back)")),
             "e2e": {"value": round(e2e_ms * 1e3, 2), "unit": "us/iter", "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": d2h,
                     "flow": e2e_note or (f"zero-copy ({e2e_mode} plan): ddt_exchange on a plan over pinned HOST "

@@ -81,6 +81,7 @@ void group_equal_requests(HostBatch& b, int ub, int max_m) {
     for (uint32_t m : gm) any |= m > 1;
     if (!any) return;
     HostBatch out;
+    out.ticket = b.ticket;
     for (size_t k : order) {
         out.add(b.descs[k], b.aux[b.descs[k].aux]);
         if (!b.xinfo.empty()) out.xinfo.push_back(b.xinfo[k]);
@@ -330,12 +331,27 @@ static int batch_variant(const HostBatch& b) {
 //   * <= kTicketMaxReqs large requests: dynamic tickets (grid_mode 1) --
 //     16 x 64 MiB packs 5.5 -> 6.4 TB/s;
 //   * many requests (1024 x 1 MiB): the static cyclic order stays best.
+// Exchange batches (flags / LL windows) always claim items by ticket, in item
+// order (fused_kernel.cu): a resident-sized grid (1) for one-wave plans, one
+// CTA per item (2) for multi-wave ones (DDT_XGRID_MODE forces either).
+static bool is_exchange_batch(const HostBatch& b) {
+    for (const XInfo& x : b.xinfo)
+        if (x.signal || x.wait) return true;
+    for (const ReqDesc& d : b.descs)
+        if (d.kind == K_LL || d.op == OP_SIGNAL) return true;
+    return false;
+}
+
 static int grid_mode_for(const HostBatch& b, int ub, int sm_count) {
     const char* e = DDT_KNOB("DDT_GRID_MODE");  // experiments: force 0 / 1 / 2
-    for (const XInfo& x : b.xinfo)
-        if (x.signal || x.wait) return 0;
-    for (const ReqDesc& d : b.descs)
-        if (d.kind == K_LL || d.op == OP_SIGNAL) return 0;
+    if (is_exchange_batch(b)) {
+        const char* xe = DDT_KNOB("DDT_XGRID_MODE");
+        uint64_t items = 0;
+        for (const ReqDesc& d : b.descs) items += desc_items(d, d.xub ? d.xub : ub);
+        int m = items > (uint64_t)kTicketMinItemsPerSM * (uint64_t)sm_count ? 2 : 1;
+        if (xe && (xe[0] == '1' || xe[0] == '2')) m = xe[0] - '0';
+        return m;
+    }
     uint64_t items = 0;
     for (const ReqDesc& d : b.descs) items += desc_items(d, ub);
     if (items < (uint64_t)kTicketMinItemsPerSM * (uint64_t)sm_count) return 0;
@@ -373,6 +389,12 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
     if (out.variant == 7 && out.ub == 1 && !multi && !(v9 && v9[0] == '1')) out.variant = 9;
     out.grid_mode = grid_mode_for(b, out.ub, sm_count);
     out.ticket = out.grid_mode == 1 ? b.ticket : 0;
+    if (is_exchange_batch(b)) {  // exchange kernels claim by ticket (DDT_XSTATIC=1: static cyclic order, A/B only)
+        const char* xs = DDT_KNOB("DDT_XSTATIC");
+        const bool st = xs && xs[0] == '1';
+        out.ticket = st ? 0 : b.ticket;
+        if (st) out.grid_mode = 0;
+    }
     const char* force = DDT_KNOB("DDT_FORCE_TABLE");  // experiments: always use the device-table form
     if (force && force[0] == '1') allow_param = false;
     const char* large = DDT_KNOB("DDT_FORCE_LARGE_PARAM");  // experiments: skip the small parameter form
@@ -399,6 +421,7 @@ int launch_fused(const Launchable& l, void* stream, int grid_cap) {
 
 int launch_exchange(const Launchable& l, const XArgs& xa, void* stream, int grid_cap) {
     const void* src = l.form == 3 ? l.dev : (const void*)l.blob.data();
+    if (l.grid_mode == 2 && grid_cap <= 0) grid_cap = -1;  // one CTA per item (ticket-claimed)
     return launch_exchange_form(l.form, l.variant, src, l.total_items, xa, stream, grid_cap);
 }
 

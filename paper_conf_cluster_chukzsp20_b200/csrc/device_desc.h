@@ -192,9 +192,17 @@ constexpr int kParamLarge = 32;
 static_assert(sizeof(ParamBatch<kParamLarge>) <= 32000, "kernel parameter limit");
 
 // Control block of the fused exchange kernel (device memory, zeroed at create).
+// The exchange epoch lives here, on the device: every CTA of a launch reads
+// `epoch` (after griddepcontrol.wait, so the previous launch of the plan has
+// completed) and runs exchange epoch + 1; the last CTA to exit stores it.  No
+// per-launch kernel argument changes, so a plan's launches can be captured
+// into a CUDA graph and replayed (a K-step time loop).  Every rank runs the
+// same sequence of exchanges, so the epochs of all ranks advance in lockstep.
 struct XCtrl {
     unsigned int trace_n;         // trace records written (tracing on)
     unsigned int pad;
+    unsigned int ticket[2];       // item tickets {next, exited} (claim order = item order)
+    unsigned long long epoch;     // exchanges completed by this plan
     unsigned long long counters[1];  // [nsend] monotonic per-message item counters
 };
 
@@ -206,15 +214,13 @@ struct TraceRec {
     unsigned long long t0, t1, t2, t3;
 };
 
-// Per-launch arguments of the fused exchange kernel.  The epoch (1, 2, ...) is
-// counted by the host -- every rank runs the same sequence of exchanges -- so
-// no CTA reads or advances device state before its first item.
+// Arguments of the fused exchange kernel: fixed for the plan's lifetime (the
+// epoch is device-resident, XCtrl::epoch), so launches are graph-capturable.
 struct TraceRec;
 struct XArgs {
     XCtrl* ctrl;
     int* err_flag;               // host-mapped: a wait timed out
     unsigned long long timeout_ns;
-    unsigned long long epoch;
     TraceRec* trace;             // 0 = tracing off
     unsigned long long trace_cap;
 };

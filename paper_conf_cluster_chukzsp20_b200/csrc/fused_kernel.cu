@@ -570,10 +570,12 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // message's epoch flag in the peer's window when the message is complete (the
 // paper's "GPU thread signals completion", across GPUs); unpack
 // items with a flag wait for it (the receiver callback of P:247, on the GPU).
-// Items are ordered [pack / direct ..., unpack ...] and every CTA walks its
-// items in increasing order, so a CTA only ever waits after finishing all of
-// its own pack items; with grid <= resident CTAs nothing waits on work that
-// cannot run (deadlock freedom without a global ticket).
+// Items are ordered [items that never wait ..., items that wait ...] and CTAs
+// CLAIM items from a global atomic ticket (XCtrl::ticket), so every item that
+// signals is claimed -- by a CTA that is running and never blocks before
+// finishing it -- before any waiting item is claimed.  Progress therefore
+// needs no co-residency: the grid may exceed the resident CTAs (one CTA per
+// item), and a kernel on another stream may hold any number of SMs.
 // INPLACE: the batch rides in the kernel parameters (constant bank): every
 // thread reads its request's descriptors in place (uniform constant loads),
 // with no shared-memory staging and no barrier before the first data load --
@@ -592,9 +594,12 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
     XCtrl* ctrl = nullptr;
     TraceRec* trace = nullptr;
     if constexpr (XCHG) {
-        epoch = xa->epoch;
         ctrl = xa->ctrl;
         trace = xa->trace;
+        // the previous launch of this plan completed before griddepcontrol.wait
+        // returned (kernel entry); no CTA of this launch stores the epoch
+        // before every CTA has read it (the store is the last CTA's exit)
+        epoch = *reinterpret_cast<volatile unsigned long long*>(&ctrl->epoch) + 1ull;
     }
     constexpr int kWords = (int)(sizeof(ReqDesc) / 16);
     constexpr int kXWords = (int)(sizeof(XInfo) / 16);
@@ -614,7 +619,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
     // dynamic tickets (device_desc.h): thread 0 fetches the next item's ticket
     // while the CTA moves the current one (two shared slots, one barrier per item)
     __shared__ uint32_t s_tk[2];
-    const bool dyn = !XCHG && tv.ticket != nullptr;
+    const bool dyn = tv.ticket != nullptr;  // exchange plans always claim by ticket
     int par = 0;
     if (dyn) {
         if (!waited) {  // the counter is reset by the previous grid: wait for it first
@@ -624,6 +629,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         if (threadIdx.x == 0) s_tk[0] = atomicAdd(tv.ticket, 1u);
         __syncthreads();
         first = s_tk[0];
+        last = tv.total;
     }
     for (uint32_t item = first; item < last;) {
         if (dyn && threadIdx.x == 0) s_tk[par ^ 1] = atomicAdd(tv.ticket, 1u);
@@ -768,11 +774,17 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             item += step;
         }
     }
-    if (dyn && threadIdx.x == 0) {  // the last CTA out resets the counter for the next launch
+    // the last CTA out resets the ticket counter for the next launch and, in an
+    // exchange, stores the epoch it ran (exchange kernels count exits on their
+    // control block even in the static item order, DDT_XSTATIC experiments)
+    unsigned int* tk = tv.ticket;
+    if constexpr (XCHG) tk = ctrl->ticket;
+    if ((dyn || XCHG) && threadIdx.x == 0) {
         __threadfence();
-        if (atomicAdd(tv.ticket + 1, 1u) == gridDim.x - 1) {
-            tv.ticket[0] = 0u;
-            tv.ticket[1] = 0u;
+        if (atomicAdd(tk + 1, 1u) == gridDim.x - 1) {
+            tk[0] = 0u;
+            tk[1] = 0u;
+            if constexpr (XCHG) ctrl->epoch = epoch;  // this exchange is complete on this rank
             __threadfence();
         }
     }
@@ -911,10 +923,9 @@ static void launch_exchange_v(int form, const void* src, uint32_t total, const X
                               int grid_cap) {
     static int res[4] = {0, 0, 0, 0};
     // programmatic serialisation: the launch overlaps the previous kernel's
-    // tail; every CTA waits (griddepcontrol.wait) before its first table, flag
-    // or data access, and all of this grid's CTAs are resident before the next
-    // PDL grid can be scheduled, so the co-residency argument for the flag
-    // waits (grid <= resident CTAs) is unchanged
+    // tail; every CTA waits (griddepcontrol.wait) before its first table, flag,
+    // epoch or data access.  grid_cap < 0: one CTA per item (items are claimed
+    // by ticket, so the grid may exceed the resident CTAs)
     if (form == 1) {
         if (!res[1]) res[1] = resident_ctas(ddt_exchange_param<kParamSmall, V>);
         launch_pdl(ddt_exchange_param<kParamSmall, V>, grid_for(total, res[1], grid_cap), s,

@@ -130,6 +130,7 @@ struct ddt_halo_s {
     void* send_stage = nullptr;
     void* recv_stage = nullptr;
     std::vector<Xfer> xfers;
+    bool self_nccl = false;       // test hook DDT_SELF_VIA_NCCL: self messages through staging + NCCL
     Launchable pack_l, unpack_l;  // NCCL mode: pack (+ direct self copies), unpack
     // P2P mode
     Launchable x_l;               // P2P mode: the single fused exchange kernel
@@ -139,7 +140,6 @@ struct ddt_halo_s {
     uint64_t timeout_ns = 10ull * 1000 * 1000 * 1000;
     int grid_cap = 0;
     bool x_flags = false;         // P2P plan has remote messages (flags); else the plain fused kernel runs
-    uint64_t epoch = 0;           // exchanges issued (every rank issues the same sequence)
     void* trace = nullptr;        // device TraceRec buffer (tracing on) and its capacity
     int64_t trace_cap = 0;
     std::vector<void*> ipc_opened;  // peers' receive buffers mapped for pack-free writes
@@ -394,11 +394,10 @@ ddt_status_t record_exchange(ddt_halo_s* h) {
     if (h->mode != DDT_XCHG_NCCL) {
         int e;
         if (h->x_flags) {
-            XArgs xa{};
+            XArgs xa{};  // the epoch is device-resident (XCtrl::epoch): nothing here varies per launch
             xa.ctrl = reinterpret_cast<XCtrl*>(h->ctrl);
             xa.err_flag = h->err_dev;
             xa.timeout_ns = h->timeout_ns;
-            xa.epoch = ++h->epoch;  // flags hold the epoch; windows alternate halves by its parity
             xa.trace = reinterpret_cast<TraceRec*>(h->trace);
             xa.trace_cap = (unsigned long long)h->trace_cap;
             e = launch_exchange(h->x_l, xa, h->stream, h->grid_cap);
@@ -413,13 +412,13 @@ ddt_status_t record_exchange(ddt_halo_s* h) {
         if (e) return cuda_fail("pack launch", e);
     }
     bool remote = false;
-    for (auto& x : h->xfers) remote |= x.peer != h->rank;
+    for (auto& x : h->xfers) remote |= x.peer != h->rank || h->self_nccl;
     if (remote) {
         const NcclApi* n = nccl();
         if (!n) return DDT_ERR_UNSUPPORTED;
         int r = n->GroupStart();
         for (auto& x : h->xfers) {
-            if (x.peer == h->rank || r != 0) continue;
+            if ((x.peer == h->rank && !h->self_nccl) || r != 0) continue;
             if (x.send_bytes)
                 r = n->Send((char*)h->send_stage + x.send_off, (size_t)x.send_bytes, kNcclUint8, x.peer, h->comm,
                             h->stream);
@@ -461,34 +460,6 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     if (c->nranks > 1 && mode == DDT_XCHG_NCCL && !c->nccl_comm) return DDT_ERR_ARG;
     if (p2p && (!c->peer_windows || c->window_bytes <= 0)) return DDT_ERR_ARG;
     if (queue_sticky(q) != DDT_OK) return queue_sticky(q);
-    // validate messages
-    std::map<std::pair<int, int>, int> seen_s, seen_r;
-    for (int i = 0; i < nsend; i++) {
-        auto& s = sends[i];
-        if (!s.type || s.count < 0 || s.peer < 0 || s.peer >= c->nranks) return DDT_ERR_ARG;
-        if (!s.type->committed) return DDT_ERR_STATE;
-        if (s.count * s.type->size > 0 && !s.buf) return DDT_ERR_ARG;
-        if (!seen_s.emplace(std::make_pair(s.peer, s.tag), i).second) return DDT_ERR_ARG;
-    }
-    for (int i = 0; i < nrecv; i++) {
-        auto& r = recvs[i];
-        if (!r.type || r.count < 0 || r.peer < 0 || r.peer >= c->nranks) return DDT_ERR_ARG;
-        if (!r.type->committed) return DDT_ERR_STATE;
-        if (r.count * r.type->size > 0 && !r.buf) return DDT_ERR_ARG;
-        if (r.count * r.type->size > 0 && instances_overlap(r.type, r.count)) return DDT_ERR_OVERLAP;
-        if (!seen_r.emplace(std::make_pair(r.peer, r.tag), i).second) return DDT_ERR_ARG;
-    }
-    if (p2p) {  // symmetric pattern required by the parity double buffering / ready handshake
-        for (auto& kv : seen_s)
-            if (kv.first.first != c->rank) {
-                bool back = false;
-                for (auto& rv : seen_r) back |= rv.first.first == kv.first.first;
-                if (!back) {
-                    set_error("P2P exchange needs a symmetric pattern (send to p => receive from p)");
-                    return DDT_ERR_ARG;
-                }
-            }
-    }
     auto* h = new (std::nothrow) ddt_halo_s();
     if (!h) return DDT_ERR_NOMEM;
     h->q = q;
@@ -500,19 +471,82 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     h->comm = c->nccl_comm;
     h->ag = c->host_allgather;
     h->ag_ctx = c->host_ctx;
+    DevGuard g(h->device);
+    // validate messages.  Every check below is local to this rank; its status
+    // is agreed (min over ranks) before the collective metadata rounds, so a
+    // rank that rejects its arguments fails together with its peers instead of
+    // leaving them blocked in the directory all-gather.
+    ddt_status_t vst = DDT_OK;
+    auto fail = [&](ddt_status_t e, const char* why) {
+        if (vst == DDT_OK) {
+            vst = e;
+            if (why) set_error(why);
+        }
+    };
+    std::map<std::pair<int, int>, int> seen_s, seen_r;
+    for (int i = 0; i < nsend; i++) {
+        auto& s = sends[i];
+        if (!s.type || s.count < 0 || s.peer < 0 || s.peer >= c->nranks) {
+            fail(DDT_ERR_ARG, "bad send argument");
+            continue;
+        }
+        if (!s.type->committed) fail(DDT_ERR_STATE, "send type not committed");
+        else if (s.count * s.type->size > 0 && !s.buf) fail(DDT_ERR_ARG, "null send buffer");
+        if (!seen_s.emplace(std::make_pair(s.peer, s.tag), i).second) fail(DDT_ERR_ARG, "duplicate (peer, tag) send");
+    }
+    for (int i = 0; i < nrecv; i++) {
+        auto& r = recvs[i];
+        if (!r.type || r.count < 0 || r.peer < 0 || r.peer >= c->nranks) {
+            fail(DDT_ERR_ARG, "bad receive argument");
+            continue;
+        }
+        if (!r.type->committed) fail(DDT_ERR_STATE, "receive type not committed");
+        else if (r.count * r.type->size > 0 && !r.buf) fail(DDT_ERR_ARG, "null receive buffer");
+        else if (r.count * r.type->size > 0 && instances_overlap(r.type, r.count))
+            fail(DDT_ERR_OVERLAP, "overlapping receive typemap");
+        if (!seen_r.emplace(std::make_pair(r.peer, r.tag), i).second) fail(DDT_ERR_ARG, "duplicate (peer, tag) receive");
+    }
+    if (p2p && vst == DDT_OK) {
+        // symmetric pattern of NON-EMPTY messages, required by the parity double
+        // buffering / ready handshake: a rank that sends data to p must also
+        // wait for data from p each exchange, or it could run two epochs ahead
+        // and overwrite the window half p is still unpacking (zero-byte
+        // messages produce no items and synchronise nothing)
+        std::map<int, int> out_nz, in_nz;
+        for (int i = 0; i < nsend; i++)
+            if (sends[i].peer != c->rank && sends[i].count * sends[i].type->size > 0) out_nz[sends[i].peer]++;
+        for (int i = 0; i < nrecv; i++)
+            if (recvs[i].peer != c->rank && recvs[i].count * recvs[i].type->size > 0) in_nz[recvs[i].peer]++;
+        for (auto& kv : out_nz)
+            if (!in_nz.count(kv.first))
+                fail(DDT_ERR_ARG, "P2P exchange needs a symmetric pattern (non-empty send to p => non-empty "
+                                  "receive from p)");
+        for (auto& kv : in_nz)
+            if (!out_nz.count(kv.first))
+                fail(DDT_ERR_ARG, "P2P exchange needs a symmetric pattern (non-empty receive from p => non-empty "
+                                  "send to p)");
+    }
+    RecvLayout RL;
+    if (vst == DDT_OK) {
+        RL = layout_recvs(nrecv, recvs, mode == DDT_XCHG_P2P);
+        if (p2p && c->window_bytes < RL.window_bytes) fail(DDT_ERR_ARG, "window smaller than ddt_halo_window_bytes()");
+    }
+    {
+        const std::string why = vst != DDT_OK ? last_error() : "";
+        ddt_status_t all = agree(h, vst);
+        if (all != DDT_OK) {
+            if (vst == DDT_OK) set_error("halo create failed on a peer rank");
+            else set_error(why);
+            delete h;  // nothing retained yet
+            return all;
+        }
+    }
     h->sends.assign(sends, sends + nsend);
     h->recvs.assign(recvs, recvs + nrecv);
     for (auto& s : h->sends) type_retain(s.type);
     for (auto& r : h->recvs) type_retain(r.type);
-    DevGuard g(h->device);
 
-    // ---- receive layout and directories (receiver -> each sender)
-    RecvLayout RL = layout_recvs(nrecv, recvs, mode == DDT_XCHG_P2P);
-    if (p2p && c->window_bytes < RL.window_bytes) {
-        free_halo(h);
-        set_error("window smaller than ddt_halo_window_bytes()");
-        return DDT_ERR_ARG;
-    }
+    // ---- receive layout (above) and directories (receiver -> each sender)
     const int P = c->nranks;
     std::vector<std::vector<int64_t>> dir_out((size_t)P), dir_in;
     for (int p = 0; p < P; p++) {
@@ -610,6 +644,11 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     const char* svw = DDT_KNOB("DDT_SELF_VIA_WINDOW");
     const bool self_window = p2p && !direct && svw && svw[0] == '1';
     auto remote = [&](int peer) { return peer != c->rank || self_window; };
+    // the same for NCCL mode (needs an NCCL communicator, e.g. a 1-rank one):
+    // self messages go pack -> staging -> ncclSend/ncclRecv to self -> unpack
+    const char* svn = DDT_KNOB("DDT_SELF_VIA_NCCL");
+    h->self_nccl = mode == DDT_XCHG_NCCL && c->nccl_comm && svn && svn[0] == '1';
+    auto remote_n = [&](int peer) { return peer != c->rank || h->self_nccl; };
 
     // ---- second metadata round (window mode): sender -> receiver, which
     // messages travel in the LL format (receiver offered it, sender can do 8-B)
@@ -689,7 +728,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         // send staging: one region per remote peer reproducing the receiver's layout
         std::map<int, std::pair<int64_t, int64_t>> span;  // peer -> (first_off, end_off) in the peer's layout
         for (int i = 0; i < nsend; i++) {
-            if (sends[i].peer == c->rank) continue;
+            if (!remote_n(sends[i].peer)) continue;
             int64_t a = match[(size_t)i]->data_off, b = a + match[(size_t)i]->bytes;
             auto it = span.find(sends[i].peer);
             if (it == span.end()) span[sends[i].peer] = {a, b};
@@ -709,7 +748,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         // my receive spans per remote peer
         std::map<int, std::pair<int64_t, int64_t>> rspan;
         for (int i = 0; i < nrecv; i++) {
-            if (recvs[i].peer == c->rank) continue;
+            if (!remote_n(recvs[i].peer)) continue;
             int64_t a = RL.data_off[(size_t)i], b = a + recvs[i].count * recvs[i].type->size;
             auto it = rspan.find(recvs[i].peer);
             if (it == rspan.end()) rspan[recvs[i].peer] = {a, b};
@@ -733,7 +772,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         for (int i = 0; i < nsend && st == DDT_OK; i++) {
             const auto& s = sends[i];
             if (s.count * s.type->size == 0) continue;
-            if (s.peer == c->rank) {
+            if (!remote_n(s.peer)) {
                 st = add_direct(packb, s, recvs[self_recv(s.tag)], false);
                 continue;
             }
@@ -742,7 +781,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         }
         for (int i = 0; i < nrecv && st == DDT_OK; i++) {
             const auto& r = recvs[i];
-            if (r.count * r.type->size == 0 || r.peer == c->rank) continue;
+            if (r.count * r.type->size == 0 || !remote_n(r.peer)) continue;
             st = add_req(unpackb, r.type, OP_UNPACK, (char*)h->recv_stage + RL.data_off[(size_t)i], r.buf, r.count,
                          nullptr);
         }
@@ -885,15 +924,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         for (const auto& x : xb.xinfo) h->x_flags |= x.signal != 0 || x.wait != 0;
         for (size_t i = 0; i < xb.descs.size(); i++)  // LL windows need the exchange kernel (and its epoch)
             h->x_flags |= xb.descs[i].kind == K_LL || xb.aux[xb.descs[i].aux].kind == K_LL;
-        if (st == DDT_OK && !xb.descs.empty()) {
-            // exchange plans chunk every message alike on both sides (kXchgUb)
-            for (size_t i = 0; i < xb.descs.size(); i++)
-                if (xb.xinfo[i].signal) xb.xinfo[i].nitems = desc_items(xb.descs[i], kXchgUb);
-            // flag-free plans (self messages only) run the plain fused kernel:
-            // adaptive item size, like any other batch
-            xb.ticket = queue_ticket(q);  // used only if the plan is flag-free (plain fused kernel)
-            st = make_table(xb, h->x_l, queue_sm_count(q), h->x_flags ? kXchgUb : 0);
-        }
+        // control block (device epoch, item tickets, message counters) first:
+        // the table carries its ticket address
         size_t ctrl_bytes = sizeof(XCtrl) + sizeof(unsigned long long) * std::max<size_t>(npack, 1);
         if (st == DDT_OK) {
             cudaError_t e = cudaMalloc(&h->ctrl, ctrl_bytes);
@@ -904,6 +936,18 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                 e = cudaHostGetDevicePointer((void**)&h->err_dev, h->err_host, 0);
             }
             if (e != cudaSuccess) st = cuda_fail("exchange control block", e);
+        }
+        if (st == DDT_OK && !xb.descs.empty()) {
+            // exchange plans chunk every message alike on both sides (kXchgUb)
+            for (size_t i = 0; i < xb.descs.size(); i++)
+                if (xb.xinfo[i].signal) xb.xinfo[i].nitems = desc_items(xb.descs[i], kXchgUb);
+            // exchange kernels claim items from the plan's own ticket (item
+            // order = claim order: deadlock freedom without co-residency);
+            // flag-free plans (self messages only) run the plain fused kernel
+            // with the queue's ticket and an adaptive item size
+            xb.ticket = h->x_flags ? (uint64_t)(uintptr_t)((char*)h->ctrl + offsetof(XCtrl, ticket))
+                                   : queue_ticket(q);
+            st = make_table(xb, h->x_l, queue_sm_count(q), h->x_flags ? kXchgUb : 0);
         }
         h->launches = xb.descs.empty() ? 0 : 1;
     }
@@ -958,17 +1002,9 @@ ddt_status_t ddt_exchange(ddt_halo_t h) {
         return DDT_ERR_TIMEOUT;
     }
     DevGuard g(h->device);
-    // a flagged P2P plan passes the epoch as a kernel argument: launched directly
-    // (a captured graph would freeze it); every other plan may replay a graph
-    if (h->mode != DDT_XCHG_NCCL && h->x_flags && h->stream) {
-        cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
-        if (cudaStreamIsCapturing(h->stream, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone) {
-            set_error("a P2P plan with remote messages cannot be captured into a CUDA graph (its epoch is a "
-                      "per-launch kernel argument): launch it directly or use DDT_XCHG_NCCL");
-            return DDT_ERR_STATE;
-        }
-    }
-    if (h->use_graph && h->stream && !(h->mode != DDT_XCHG_NCCL && h->x_flags)) {
+    // every plan may be captured (the P2P epoch is device-resident) and, with
+    // ddt_halo_set_graph, replays its own captured graph
+    if (h->use_graph && h->stream) {
         if (!h->gexec) {
             cudaError_t e = cudaStreamBeginCapture(h->stream, cudaStreamCaptureModeThreadLocal);
             if (e != cudaSuccess) return cuda_fail("graph capture begin", e);

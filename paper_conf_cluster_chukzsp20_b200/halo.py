@@ -87,8 +87,20 @@ class Comm:
         self._cb = _c_allgather(gather) if gather is not None else None
 
     @staticmethod
-    def single(device: int = 0) -> "Comm":
-        return Comm(0, 1, device)
+    def single(device: int = 0, nccl: bool = False) -> "Comm":
+        """One rank.  nccl=True also creates a 1-rank NCCL communicator (NCCL
+        send/recv to self: the DDT_SELF_VIA_NCCL test hook routes self messages
+        through the NCCL-mode staging + transfer path on one GPU)."""
+        c = Comm(0, 1, device)
+        if nccl:
+            uid = ctypes.create_string_buffer(128)
+            check(lib().ddt_nccl_unique_id(uid), "ddt_nccl_unique_id")
+            comm = P()
+            import torch
+            with torch.cuda.device(device):
+                check(lib().ddt_nccl_comm_create(1, uid, 0, ctypes.byref(comm)), "ddt_nccl_comm_create")
+            c.nccl_comm = comm
+        return c
 
     @staticmethod
     def from_torch(device: int, group=None, nccl: bool = True) -> "Comm":

@@ -64,3 +64,25 @@ def assert_bytes_equal(got: np.ndarray, exp: np.ndarray, what=""):
         bad = np.nonzero(got != exp)[0]
         raise AssertionError(f"{what}: {bad.size} bytes differ; first at {bad[:8].tolist()} "
                              f"got {got[bad[:8]].tolist()} expected {exp[bad[:8]].tolist()}")
+
+
+def occupier():
+    """ctypes handle of tests/c/occupy.cu (built here with nvcc for sm_100a on
+    first use; test support, not part of the library)."""
+    import ctypes
+    import os
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    src = os.path.join(root, "tests", "c", "occupy.cu")
+    out = os.path.join(root, "build", "occupy.so")
+    if not os.path.exists(out) or os.path.getmtime(out) < os.path.getmtime(src):
+        os.makedirs(os.path.dirname(out), exist_ok=True)
+        tmp = out + f".tmp{os.getpid()}"
+        subprocess.check_call(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O2",
+                               "-shared", "-Xcompiler", "-fPIC", "-o", tmp, src])
+        os.replace(tmp, out)
+    L = ctypes.CDLL(out)
+    L.occupy_launch.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p,
+                                ctypes.c_longlong]
+    L.occupy_launch.restype = ctypes.c_int
+    return L

@@ -129,32 +129,3 @@ def test_p2p_wait_times_out_instead_of_hanging():
             if p.is_alive():
                 p.kill()
     assert res == {0: True, 1: True}, res
-
-
-@pytest.mark.filterwarnings("ignore:The CUDA Graph is empty")
-def test_flagged_p2p_plan_refuses_capture(ddt, monkeypatch):
-    """A P2P plan with flags (here: self messages forced through the window
-    path) carries its epoch as a kernel argument, so capturing it into a user
-    graph would freeze the epoch: ddt_exchange returns DDT_ERR_STATE instead.
-    Plans without flags capture fine (bench.py's N = 1 K-step graph)."""
-    import torch
-    from ddt_inputs import halo_messages, FACE_DIRS
-    monkeypatch.setenv("DDT_SELF_VIA_WINDOW", "1")
-    s = torch.cuda.Stream()
-    with torch.cuda.stream(s):
-        a = torch.zeros((6, 6, 6), dtype=torch.int64, device="cuda")
-        msgs = halo_messages(0, 1, (4, 4, 4), dirs=FACE_DIRS)
-        sends = [(m["peer"], m["tag"], ddt.Type.from_spec(m["send_spec"]), a, 1) for m in msgs]
-        recvs = [(m["recv_peer"], m["recv_tag"], ddt.Type.from_spec(m["recv_spec"]), a, 1) for m in msgs]
-        q = ddt.Queue()
-        h = ddt.Halo(q, ddt.Comm.single(0), sends, recvs, mode="p2p", graph=False)
-        h.exchange()  # direct launch works
-        torch.cuda.synchronize()
-        g = torch.cuda.CUDAGraph()
-        with pytest.raises(ddt.DDTError) as e:
-            with torch.cuda.graph(g, stream=s):
-                h.exchange()
-        assert e.value.code == -2
-        torch.cuda.synchronize()
-        h.destroy()
-        q.destroy()

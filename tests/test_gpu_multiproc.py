@@ -107,3 +107,159 @@ def test_p2p_exchange_multiprocess_one_gpu(world, dirs_name, iters, mode, group)
             if p.is_alive():
                 p.kill()
     assert len(res) == world and all(res.values()), res
+
+
+def _worker_bytes(rank, world, port, opts, q):
+    """Like _worker, but every rank's arrays live in uint8 device buffers at a
+    byte offset (odd ranks at 4 mod 8 when opts['mis']: sender and receiver
+    vector widths then differ, so messages are released whole -- the fan-out
+    path), with optional env knobs, element type and local size."""
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    for k, v in opts.get("env", {}).items():
+        os.environ[k] = v
+    ok = False
+    try:
+        init(rank, world, port)
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(0)
+        import paper_conf_cluster_chukzsp20_b200 as ddt
+        from ddt_inputs import (halo_messages, proc_grid, global_block, padded_block, ghost_mask, random_bytes,
+                                FACE_DIRS, ALL_DIRS)
+        dirs = FACE_DIRS if opts["dirs"] == "faces" else ALL_DIRS
+        P, local, nvars, base = world, tuple(opts["local"]), opts.get("nvars", 2), opts.get("base", "double")
+        esz, dt = (8, np.int64) if base == "double" else (4, np.int32)
+        grid = proc_grid(P)
+        G = tuple(n * g for n, g in zip(local, grid))
+        shape = tuple(n + 2 for n in local)
+        nbytes = int(np.prod(shape)) * esz
+        off = 4 if (opts.get("mis") and rank % 2 == 1) else 0
+        bufs = [torch.full((nbytes + 64,), 0xA5, dtype=torch.uint8, device="cuda") for _ in range(nvars)]
+        msgs = halo_messages(rank, P, local, dirs=dirs, nvars=nvars, base=base)
+        cache = {}
+
+        def T(spec):
+            if repr(spec) not in cache:
+                cache[repr(spec)] = ddt.Type.from_spec(spec)
+            return cache[repr(spec)]
+        sends = [(m["peer"], m["tag"], T(m["send_spec"]), (bufs[m["var"]], off), 1) for m in msgs]
+        recvs = [(m["recv_peer"], m["recv_tag"], T(m["recv_spec"]), (bufs[m["var"]], off), 1) for m in msgs]
+        comm = ddt.Comm.from_torch(0, nccl=False)
+        qq = ddt.Queue()
+        graph = opts.get("graph", False)
+        h = ddt.Halo(qq, comm, sends, recvs, mode=opts.get("mode", "p2p"), graph=graph)
+        gm = ghost_mask(local, dirs)
+        ok = True
+        for it in range(opts.get("iters", 3)):
+            globs = [random_bytes(int(np.prod(G)) * esz, 700 + 10 * it + v).view(dt).reshape(G) for v in range(nvars)]
+            for v in range(nvars):
+                a = np.full(shape, -1, dt)  # ghosts != any expected value pattern
+                a[1:-1, 1:-1, 1:-1] = global_block(globs[v], rank, P)
+                bufs[v][off:off + nbytes].copy_(torch.from_numpy(a.view(np.uint8).reshape(-1)))
+            torch.cuda.synchronize()
+            dist.barrier()
+            h.exchange()
+            torch.cuda.synchronize()
+            dist.barrier()
+            for v in range(nvars):
+                got = bufs[v][off:off + nbytes].cpu().numpy().view(dt).reshape(shape)
+                exp = padded_block(globs[v], rank, P)
+                ok &= bool(np.array_equal(got[gm], exp[gm]))
+                ok &= bool(np.array_equal(got[1:-1, 1:-1, 1:-1], exp[1:-1, 1:-1, 1:-1]))
+        h.destroy()
+        dist.barrier()
+        comm.close()
+        qq.destroy()
+        dist.destroy_process_group()
+    except Exception as e:
+        print(f"rank {rank}: {type(e).__name__}: {e}", flush=True)
+        ok = False
+    q.put((rank, ok))
+
+
+def _spawn(target, world, extra, timeout=400):
+    import torch.multiprocessing as mp
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = free_port()
+    procs = [ctx.Process(target=target, args=(r, world, port) + extra + (q,)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    try:
+        for _ in range(world):
+            r, ok = q.get(timeout=timeout)
+            res[r] = ok
+    finally:
+        for p in procs:
+            p.join(timeout=60)
+            if p.is_alive():
+                p.kill()
+    return res
+
+
+@pytest.mark.timeout(900)
+@pytest.mark.parametrize("world,opts", [
+    # the per-chunk flag protocol for every message (no LL)
+    (2, dict(dirs="all", local=(6, 5, 7), env={"DDT_NO_LL": "1"}, iters=4)),
+    (4, dict(dirs="all", local=(6, 5, 7), env={"DDT_NO_LL": "1"}, iters=3)),
+    (8, dict(dirs="faces", local=(6, 5, 7), env={"DDT_NO_LL": "1"}, iters=2)),
+    # messages > 512 KB (528 KiB z faces): per-chunk flags at 2 vectors per thread per item
+    (2, dict(dirs="faces", local=(4, 260, 260), nvars=1, iters=3)),
+    (2, dict(dirs="faces", local=(4, 260, 260), nvars=1, iters=4, graph=True)),
+    # 4-B elements (4-B vectors, LL does not apply)
+    (2, dict(dirs="all", local=(6, 10, 12), base="float", iters=3)),
+    (4, dict(dirs="all", local=(6, 10, 12), base="float", iters=3)),
+    # sender / receiver widths differ (odd ranks at 4 mod 8): whole-message fan-out + counters
+    (2, dict(dirs="all", local=(6, 10, 12), mis=True, iters=3)),
+    (4, dict(dirs="all", local=(12, 20, 24), mis=True, iters=3)),
+    (2, dict(dirs="faces", local=(4, 260, 260), nvars=1, mis=True, iters=3)),
+    # configs[1] at full size with P = 2 (remote z faces + self faces), both window formats
+    (2, dict(dirs="faces", local=(128, 128, 128), nvars=1, iters=2)),
+    (2, dict(dirs="faces", local=(128, 128, 128), nvars=1, iters=2, env={"DDT_NO_LL": "1"})),
+    (2, dict(dirs="faces", local=(128, 128, 128), nvars=1, iters=2, mode="p2p_direct")),
+    # one CTA per item forced for the exchange kernel (ticket-claimed)
+    (2, dict(dirs="all", local=(12, 20, 24), iters=3, env={"DDT_XGRID_MODE": "2"})),
+])
+def test_exchange_protocols_multiprocess(world, opts):
+    res = _spawn(_worker_bytes, world, (opts,))
+    assert len(res) == world and all(res.values()), res
+
+
+def _bad_args_worker(rank, world, port, q):
+    """Rank 1 passes an invalid message (peer out of range); rank 0 is valid.
+    Both must fail ddt_halo_create (the local checks are agreed before any
+    collective metadata round), neither may hang."""
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    res = "none"
+    try:
+        init(rank, world, port)
+        import torch
+        torch.cuda.set_device(0)
+        import paper_conf_cluster_chukzsp20_b200 as ddt
+        from ddt_inputs import halo_messages, FACE_DIRS
+        local = (4, 5, 6)
+        a = torch.zeros(tuple(n + 2 for n in local), dtype=torch.int64, device="cuda")
+        msgs = halo_messages(rank, world, local, dirs=FACE_DIRS)
+        sends = [(m["peer"], m["tag"], ddt.Type.from_spec(m["send_spec"]), a, 1) for m in msgs]
+        recvs = [(m["recv_peer"], m["recv_tag"], ddt.Type.from_spec(m["recv_spec"]), a, 1) for m in msgs]
+        if rank == 1:
+            p, t, ty, b, c = sends[0]
+            sends[0] = (world + 3, t, ty, b, c)
+        comm = ddt.Comm.from_torch(0, nccl=False)
+        qq = ddt.Queue()
+        try:
+            ddt.Halo(qq, comm, sends, recvs, mode="p2p", graph=False)
+            res = "created"
+        except Exception as e:
+            res = f"error:{e}"
+    except Exception as e:
+        res = f"setup:{type(e).__name__}: {e}"
+    q.put((rank, res))
+
+
+@pytest.mark.timeout(300)
+def test_halo_create_fails_on_every_rank_together():
+    res = _spawn(_bad_args_worker, 2, (), timeout=200)
+    assert len(res) == 2, res
+    assert all(v.startswith("error:") for v in res.values()), res
