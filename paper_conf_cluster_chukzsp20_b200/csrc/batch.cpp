@@ -245,11 +245,12 @@ int choose_ub(const HostBatch& b, int sm_count) {
     return 1;
 }
 
-uint32_t write_device_table(void* dst, const HostBatch& b, int ub, uint64_t ticket) {
+uint32_t write_device_table(void* dst, const HostBatch& b, int ub, uint64_t ticket, uint32_t claim) {
     size_t n = b.descs.size();
     auto* h = reinterpret_cast<BatchHeader*>(dst);
     std::memset(h, 0, sizeof(*h));
     h->ticket = ticket;
+    h->claim = claim;
     auto* prefix = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(dst) + sizeof(BatchHeader));
     uint32_t items = fill_prefix(prefix, b, ub);
     size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
@@ -293,6 +294,7 @@ static void to_param(const HostBatch& b, Launchable& out) {
     p->h.flags = batch_flags(b);
     p->h.total_items = fill_prefix(p->prefix, b, out.ub);
     p->h.ticket = out.ticket;
+    p->h.claim = out.claim;
     std::copy(b.gm.begin(), b.gm.end(), p->gm);
     std::copy(b.descs.begin(), b.descs.end(), p->descs);
     std::copy(b.aux.begin(), b.aux.end(), p->aux);
@@ -332,8 +334,9 @@ static int batch_variant(const HostBatch& b) {
 //     16 x 64 MiB packs 5.5 -> 6.4 TB/s;
 //   * many requests (1024 x 1 MiB): the static cyclic order stays best.
 // Exchange batches (flags / LL windows) always claim items by ticket, in item
-// order (fused_kernel.cu): a resident-sized grid (1) for one-wave plans, one
-// CTA per item (2) for multi-wave ones (DDT_XGRID_MODE forces either).
+// order (fused_kernel.cu): one CTA per item (2) for one-wave plans, a
+// resident-sized grid claiming chunks of items (1) for multi-wave ones
+// (DDT_XGRID_MODE forces either).
 static bool is_exchange_batch(const HostBatch& b) {
     for (const XInfo& x : b.xinfo)
         if (x.signal || x.wait) return true;
@@ -348,7 +351,7 @@ static int grid_mode_for(const HostBatch& b, int ub, int sm_count) {
         const char* xe = DDT_KNOB("DDT_XGRID_MODE");
         uint64_t items = 0;
         for (const ReqDesc& d : b.descs) items += desc_items(d, d.xub ? d.xub : ub);
-        int m = items > (uint64_t)kTicketMinItemsPerSM * (uint64_t)sm_count ? 2 : 1;
+        int m = items > (uint64_t)kTicketMinItemsPerSM * (uint64_t)sm_count ? 1 : 2;
         if (xe && (xe[0] == '1' || xe[0] == '2')) m = xe[0] - '0';
         return m;
     }
@@ -389,11 +392,14 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
     if (out.variant == 7 && out.ub == 1 && !multi && !(v9 && v9[0] == '1')) out.variant = 9;
     out.grid_mode = grid_mode_for(b, out.ub, sm_count);
     out.ticket = out.grid_mode == 1 ? b.ticket : 0;
-    if (is_exchange_batch(b)) {  // exchange kernels claim by ticket (DDT_XSTATIC=1: static cyclic order, A/B only)
-        const char* xs = DDT_KNOB("DDT_XSTATIC");
-        const bool st = xs && xs[0] == '1';
-        out.ticket = st ? 0 : b.ticket;
-        if (st) out.grid_mode = 0;
+    out.claim = 0;
+    if (is_exchange_batch(b)) {
+        // exchange kernels claim from the plan's tick (b.ticket = &XCtrl::tick):
+        // one item per CTA (grid_mode 2, claim 0) or chunks of DDT_XCLAIM
+        // (default kXClaim) consecutive items over a resident grid (grid_mode 1)
+        out.ticket = b.ticket;
+        const char* xc = DDT_KNOB("DDT_XCLAIM");
+        out.claim = out.grid_mode == 2 ? 0u : (uint32_t)(xc ? std::max(1, atoi(xc)) : kXClaim);
     }
     const char* force = DDT_KNOB("DDT_FORCE_TABLE");  // experiments: always use the device-table form
     if (force && force[0] == '1') allow_param = false;

@@ -167,9 +167,10 @@ struct Launchable {
     int ub = kUnroll;           // vectors per thread per item
     uint64_t ticket = 0;        // dynamic item tickets in use (device counter), 0 = static order
     int grid_mode = 0;          // 0: resident grid, static item order; 1: resident grid, tickets; 2: one CTA per item
+    uint32_t claim = 0;         // exchange batches: items per ticket claim (0 = one item per CTA)
 };
 size_t device_table_bytes(const HostBatch& b);
-uint32_t write_device_table(void* dst, const HostBatch& b, int ub, uint64_t ticket = 0);
+uint32_t write_device_table(void* dst, const HostBatch& b, int ub, uint64_t ticket = 0, uint32_t claim = 0);
 // Items per thread for a batch: the largest of {4, 2, 1} that still gives
 // >= 2 items per SM, so latency-bound batches use every SM.
 int choose_ub(const HostBatch& b, int sm_count);

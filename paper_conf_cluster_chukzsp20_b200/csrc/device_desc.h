@@ -156,8 +156,8 @@ struct alignas(16) BatchHeader {
     uint32_t ub;            // vectors per thread per item (1, 2 or 4)
     uint32_t flags;         // bit 0: blocked item order (else cyclic over CTAs); bit 1: grouped (gm[] present)
     uint32_t order_offset;  // 0, or byte offset of the explicit item table (kBatchSpread)
-    uint32_t pad0;
-    uint64_t ticket;        // 0: static item order; else device u32[2] {next, exited}: dynamic item tickets
+    uint32_t claim;         // exchange batches: items per claim (0 = one item per CTA, grid == total_items)
+    uint64_t ticket;        // plain: 0 = static order, else device u32[2] {next, exited}; exchange: XCtrl::tick
 };
 // Dynamic item tickets (multi-wave plain batches): a resident-sized grid takes
 // items in increasing order from an atomic counter instead of the static
@@ -169,6 +169,8 @@ struct alignas(16) BatchHeader {
 constexpr uint32_t kTicketMinItemsPerSM = 8;
 constexpr uint32_t kTicketMaxReqs = 64;
 constexpr uint32_t kBatchBlocked = 1u, kBatchGrouped = 2u;
+// Items per ticket claim of a multi-wave exchange launch (resident grid).
+constexpr uint32_t kXClaim = 4;
 // Spread batches (batch.cpp spread_items): an explicit item table order[item] =
 // (request << kSpreadShift) | chunk, ordered so that every request's chunks are
 // spread evenly over the whole launch (chunk c of a request of n items sits at
@@ -192,17 +194,22 @@ constexpr int kParamLarge = 32;
 static_assert(sizeof(ParamBatch<kParamLarge>) <= 32000, "kernel parameter limit");
 
 // Control block of the fused exchange kernel (device memory, zeroed at create).
-// The exchange epoch lives here, on the device: every CTA of a launch reads
-// `epoch` (after griddepcontrol.wait, so the previous launch of the plan has
-// completed) and runs exchange epoch + 1; the last CTA to exit stores it.  No
-// per-launch kernel argument changes, so a plan's launches can be captured
-// into a CUDA graph and replayed (a K-step time loop).  Every rank runs the
-// same sequence of exchanges, so the epochs of all ranks advance in lockstep.
+//
+// Item claiming and the exchange epoch (fused_kernel.cu): CTAs claim items of
+// an exchange launch from the monotonic 64-bit counter `tick` (never reset), in
+// item order.  Every launch of a plan takes the same, fixed number of tickets
+// (its "span"): with one item per CTA (claim == 0) each of the total_items
+// CTAs claims once, span = total_items; with a resident grid looping over
+// chunks of `claim` items, every CTA claims until one claim lands past the
+// last chunk, span = claim * (ceil(total / claim) + grid).  So ticket t
+// belongs to launch t / span -- the exchange epoch is t / span + 1, on the
+// device, with no exit counter, no reset and no per-launch kernel argument:
+// launches are graph-capturable, and every rank (running the same sequence of
+// exchanges) derives the same epoch.
 struct XCtrl {
     unsigned int trace_n;         // trace records written (tracing on)
     unsigned int pad;
-    unsigned int ticket[2];       // item tickets {next, exited} (claim order = item order)
-    unsigned long long epoch;     // exchanges completed by this plan
+    unsigned long long tick;      // item tickets claimed so far (monotonic)
     unsigned long long counters[1];  // [nsend] monotonic per-message item counters
 };
 
@@ -215,7 +222,7 @@ struct TraceRec {
 };
 
 // Arguments of the fused exchange kernel: fixed for the plan's lifetime (the
-// epoch is device-resident, XCtrl::epoch), so launches are graph-capturable.
+// epoch derives from the claimed tickets, XCtrl), so launches are graph-capturable.
 struct TraceRec;
 struct XArgs {
     XCtrl* ctrl;

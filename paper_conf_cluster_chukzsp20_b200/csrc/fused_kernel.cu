@@ -39,7 +39,7 @@
 #define DDT_MINB 5
 #endif
 #ifndef DDT_XMINB
-#define DDT_XMINB 1
+#define DDT_XMINB 4
 #endif
 #ifndef DDT_V8_MINB
 #define DDT_V8_MINB 6
@@ -490,7 +490,7 @@ __device__ __forceinline__ uint32_t find_request(const uint32_t* prefix, uint32_
 }
 
 struct TableView {
-    uint32_t nreq, total, ub, flags;
+    uint32_t nreq, total, ub, flags, claim;
     const uint32_t* prefix;
     const uint32_t* gm;       // group size per request (kBatchGrouped)
     const ReqDesc* descs;
@@ -507,6 +507,7 @@ __device__ __forceinline__ TableView view_of(const uint8_t* t) {
     v.total = h->total_items;
     v.ub = h->ub;
     v.flags = h->flags;
+    v.claim = h->claim;
     v.prefix = reinterpret_cast<const uint32_t*>(t + sizeof(BatchHeader));
     v.gm = reinterpret_cast<const uint32_t*>(t + sizeof(BatchHeader) + ((((size_t)h->nreq + 1) * 4 + 15) & ~(size_t)15));
     v.descs = reinterpret_cast<const ReqDesc*>(t + h->desc_offset);
@@ -524,6 +525,7 @@ __device__ __forceinline__ TableView view_of(const ParamBatch<CAP>& p) {
     v.total = p.h.total_items;
     v.ub = p.h.ub;
     v.flags = p.h.flags;
+    v.claim = p.h.claim;
     v.prefix = p.prefix;
     v.gm = p.gm;
     v.descs = p.descs;
@@ -571,11 +573,13 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // paper's "GPU thread signals completion", across GPUs); unpack
 // items with a flag wait for it (the receiver callback of P:247, on the GPU).
 // Items are ordered [items that never wait ..., items that wait ...] and CTAs
-// CLAIM items from a global atomic ticket (XCtrl::ticket), so every item that
-// signals is claimed -- by a CTA that is running and never blocks before
-// finishing it -- before any waiting item is claimed.  Progress therefore
-// needs no co-residency: the grid may exceed the resident CTAs (one CTA per
-// item), and a kernel on another stream may hold any number of SMs.
+// CLAIM items (or chunks of consecutive items) from a global atomic ticket
+// (XCtrl::tick) and run them in increasing order, so every item that signals
+// is claimed -- by a CTA that is running and never blocks before finishing it
+// -- before any waiting item is claimed.  Progress therefore needs no
+// co-residency: the grid may exceed the resident CTAs (one CTA per item), and
+// a kernel on another stream may hold any number of SMs.  The ticket also
+// gives the launch's epoch (device_desc.h XCtrl).
 // INPLACE: the batch rides in the kernel parameters (constant bank): every
 // thread reads its request's descriptors in place (uniform constant loads),
 // with no shared-memory staging and no barrier before the first data load --
@@ -596,10 +600,6 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
     if constexpr (XCHG) {
         ctrl = xa->ctrl;
         trace = xa->trace;
-        // the previous launch of this plan completed before griddepcontrol.wait
-        // returned (kernel entry); no CTA of this launch stores the epoch
-        // before every CTA has read it (the store is the last CTA's exit)
-        epoch = *reinterpret_cast<volatile unsigned long long*>(&ctrl->epoch) + 1ull;
     }
     constexpr int kWords = (int)(sizeof(ReqDesc) / 16);
     constexpr int kXWords = (int)(sizeof(XInfo) / 16);
@@ -619,7 +619,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
     // dynamic tickets (device_desc.h): thread 0 fetches the next item's ticket
     // while the CTA moves the current one (two shared slots, one barrier per item)
     __shared__ uint32_t s_tk[2];
-    const bool dyn = tv.ticket != nullptr;  // exchange plans always claim by ticket
+    const bool dyn = !XCHG && tv.ticket != nullptr;
     int par = 0;
     if (dyn) {
         if (!waited) {  // the counter is reset by the previous grid: wait for it first
@@ -630,6 +630,32 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         __syncthreads();
         first = s_tk[0];
         last = tv.total;
+    }
+    // exchange: claim items (chunks of xclaim, or one item per CTA) from the
+    // plan's monotonic tick in item order; the first claim also fixes the
+    // epoch (device_desc.h XCtrl).  Thread 0 prefetches the next chunk's claim.
+    __shared__ unsigned long long s_xt[2];
+    unsigned long long* xtick = nullptr;
+    uint32_t xclaim = 0;
+    uint64_t xspan = 0, xend = 0;
+    if constexpr (XCHG) {
+        xtick = reinterpret_cast<unsigned long long*>(tv.ticket);
+        xclaim = tv.claim;
+        const uint64_t nch = xclaim ? ((uint64_t)tv.total + xclaim - 1) / xclaim : (uint64_t)tv.total;
+        xspan = xclaim ? (uint64_t)xclaim * (nch + gridDim.x) : (uint64_t)tv.total;
+        xend = xclaim ? (uint64_t)xclaim * nch : (uint64_t)tv.total;
+        if (threadIdx.x == 0) s_xt[0] = atomicAdd(xtick, xclaim ? (unsigned long long)xclaim : 1ull);
+        __syncthreads();
+        const uint64_t t = s_xt[0];
+        epoch = t / xspan + 1ull;
+        const uint64_t loc = t % xspan;
+        if (loc >= xend) {
+            first = last = 0;  // this CTA's one failing claim: nothing to do
+        } else {
+            first = (uint32_t)loc;
+            last = xclaim ? min(tv.total, (uint32_t)loc + xclaim) : (uint32_t)loc + 1u;
+            if (xclaim && threadIdx.x == 0) s_xt[1] = atomicAdd(xtick, (unsigned long long)xclaim);  // prefetch
+        }
     }
     for (uint32_t item = first; item < last;) {
         if (dyn && threadIdx.x == 0) s_tk[par ^ 1] = atomicAdd(tv.ticket, 1u);
@@ -770,21 +796,26 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             __syncthreads();  // the prefetched ticket is visible; every thread is past this item
             par ^= 1;
             item = s_tk[par];
+        } else if (XCHG) {
+            if (++item >= last) {  // chunk done: take the prefetched claim
+                if (!xclaim) break;
+                __syncthreads();   // the prefetched claim is visible; every thread is past this item
+                par ^= 1;
+                const uint64_t loc = s_xt[par] % xspan;
+                if (loc >= xend) break;
+                item = (uint32_t)loc;
+                last = min(tv.total, (uint32_t)loc + xclaim);
+                if (threadIdx.x == 0) s_xt[par ^ 1] = atomicAdd(xtick, (unsigned long long)xclaim);
+            }
         } else {
             item += step;
         }
     }
-    // the last CTA out resets the ticket counter for the next launch and, in an
-    // exchange, stores the epoch it ran (exchange kernels count exits on their
-    // control block even in the static item order, DDT_XSTATIC experiments)
-    unsigned int* tk = tv.ticket;
-    if constexpr (XCHG) tk = ctrl->ticket;
-    if ((dyn || XCHG) && threadIdx.x == 0) {
+    if (dyn && threadIdx.x == 0) {  // the last CTA out resets the counter for the next launch
         __threadfence();
-        if (atomicAdd(tk + 1, 1u) == gridDim.x - 1) {
-            tk[0] = 0u;
-            tk[1] = 0u;
-            if constexpr (XCHG) ctrl->epoch = epoch;  // this exchange is complete on this rank
+        if (atomicAdd(tv.ticket + 1, 1u) == gridDim.x - 1) {
+            tv.ticket[0] = 0u;
+            tv.ticket[1] = 0u;
             __threadfence();
         }
     }
@@ -816,7 +847,13 @@ template <int V> struct VarT {
     // (tools/pack_probe.py: 1 MiB x 1024 packs 4.74 -> 6.08 TB/s from 3 to 5
     // CTAs/SM); exchange kernels (flags, tracing) keep their registers.
     static constexpr int MINB = (V == 7 || V == 9) ? DDT_V7_MINB : ((V == 8 || V == 10) ? DDT_V8_MINB : DDT_MINB);
-    static constexpr int XMINB = (V == 7 || V == 9) ? DDT_V7_MINB : ((V == 8 || V == 10) ? DDT_V8_MINB : DDT_XMINB);
+    // exchange kernels: every request moves at most kXchgUb vectors per thread
+    // per item (sender and receiver chunk alike), so two load slots suffice;
+    // >= 4 resident CTAs per SM (<= 64 registers) keep one-CTA-per-item
+    // exchange launches in as few waves as possible (96 registers / 2 CTAs
+    // per SM before: configs[1] through the window protocol 7.2 -> see DESIGN)
+    static constexpr int XUNR = UNR < kXchgUb ? UNR : kXchgUb;
+    static constexpr int XMINB = (V == 8 || V == 10) ? DDT_V8_MINB : DDT_XMINB;
 };
 
 template <int V>
@@ -839,7 +876,7 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_dev(const uint8_t* __restrict__ table, const XArgs xa) {
     pdl_trigger();
     pdl_wait();  // before any table read, flag or data access
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(table), &xa);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::XUNR>(view_of(table), &xa);
 }
 
 template <int CAP, int V>
@@ -847,7 +884,7 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, const XArgs xa) {
     pdl_trigger();
     pdl_wait();
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::UNR>(view_of(pb), &xa);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::XUNR>(view_of(pb), &xa);
 }
 
 // ------------------------------------------------------------------ host side

@@ -206,7 +206,7 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
     make_launchable(b, !spread, l, sm_count, ub);
     if (l.form != 3) return DDT_OK;
     std::vector<uint8_t> host(device_table_bytes(b));
-    write_device_table(host.data(), b, l.ub, l.ticket);
+    write_device_table(host.data(), b, l.ub, l.ticket, l.claim);
     return upload(host, &l.dev);
 }
 
@@ -924,8 +924,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         for (const auto& x : xb.xinfo) h->x_flags |= x.signal != 0 || x.wait != 0;
         for (size_t i = 0; i < xb.descs.size(); i++)  // LL windows need the exchange kernel (and its epoch)
             h->x_flags |= xb.descs[i].kind == K_LL || xb.aux[xb.descs[i].aux].kind == K_LL;
-        // control block (device epoch, item tickets, message counters) first:
-        // the table carries its ticket address
+        // control block (item tick -> epoch, message counters) first: the
+        // table carries the tick's address
         size_t ctrl_bytes = sizeof(XCtrl) + sizeof(unsigned long long) * std::max<size_t>(npack, 1);
         if (st == DDT_OK) {
             cudaError_t e = cudaMalloc(&h->ctrl, ctrl_bytes);
@@ -945,7 +945,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             // order = claim order: deadlock freedom without co-residency);
             // flag-free plans (self messages only) run the plain fused kernel
             // with the queue's ticket and an adaptive item size
-            xb.ticket = h->x_flags ? (uint64_t)(uintptr_t)((char*)h->ctrl + offsetof(XCtrl, ticket))
+            xb.ticket = h->x_flags ? (uint64_t)(uintptr_t)((char*)h->ctrl + offsetof(XCtrl, tick))
                                    : queue_ticket(q);
             st = make_table(xb, h->x_l, queue_sm_count(q), h->x_flags ? kXchgUb : 0);
         }
