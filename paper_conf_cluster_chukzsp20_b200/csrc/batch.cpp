@@ -150,18 +150,76 @@ void phase_batch(HostBatch& b) {
     }
 }
 
-bool spread_items(HostBatch& b, int ub) {
+// Two closed-form sides walk the same lattice of segments with bases less
+// than one innermost stride apart (same rows).
+static bool same_lattice(const ReqDesc& a, const ReqDesc& c) {
+    if (a.kind != K_STRIDED || c.kind != K_STRIDED || a.ndim != c.ndim || a.ndim == 0 || a.lw != c.lw ||
+        a.vps.d != c.vps.d || a.extent != c.extent || a.ph || c.ph)
+        return false;
+    for (int k = 0; k < a.ndim; k++)
+        if (a.radix[k].d != c.radix[k].d || a.stride[k] != c.stride[k]) return false;
+    const int64_t pa = (int64_t)a.ptr + a.base, pc = (int64_t)c.ptr + c.base;
+    const int64_t d = pa > pc ? pa - pc : pc - pa;
+    return d < (a.stride[0] < 0 ? -a.stride[0] : a.stride[0]);
+}
+
+// Pair requests whose both sides walk the same short-segment lattice (see
+// device_desc.h kSpreadShift): partners become adjacent, the first carries
+// pair = 1.  Spread (non-exchange, plain) batches only.  DDT_NO_PAIR=1: off.
+static void pair_requests(HostBatch& b) {
+    const char* off = DDT_KNOB("DDT_NO_PAIR");
+    if ((off && off[0] == '1') || !b.gm.empty()) return;
     const size_t n = b.descs.size();
-    if (n < 2 || n > (1u << (32 - kSpreadShift))) return false;
+    std::vector<int> partner(n, -1);
+    bool any = false;
+    for (size_t i = 0; i < n; i++) {
+        const ReqDesc& A = b.descs[i];
+        if (partner[i] >= 0 || A.resp || !(A.l2_64 || b.aux[A.aux].l2_64) || A.nvec == 0) continue;
+        for (size_t j = i + 1; j < n; j++) {
+            const ReqDesc& B = b.descs[j];
+            if (partner[j] >= 0 || B.resp || B.nvec != A.nvec || B.op != A.op) continue;
+            if (!same_lattice(A, B) || !same_lattice(b.aux[A.aux], b.aux[B.aux])) continue;
+            partner[i] = (int)j;
+            partner[j] = (int)i;
+            any = true;
+            break;
+        }
+    }
+    if (!any) return;
+    HostBatch out;
+    out.ticket = b.ticket;
+    for (size_t i = 0; i < n; i++) {
+        if (partner[i] >= 0 && (size_t)partner[i] < i) continue;  // placed with its partner
+        ReqDesc d = b.descs[i];
+        d.pair = partner[i] >= 0 ? 1 : 0;
+        out.add(d, b.aux[b.descs[i].aux]);
+        if (!b.xinfo.empty()) out.xinfo.push_back(b.xinfo[i]);
+        if (partner[i] >= 0) {
+            out.add(b.descs[(size_t)partner[i]], b.aux[b.descs[(size_t)partner[i]].aux]);
+            if (!b.xinfo.empty()) out.xinfo.push_back(b.xinfo[(size_t)partner[i]]);
+        }
+    }
+    b = std::move(out);
+}
+
+bool spread_items(HostBatch& b, int ub, bool allow_pair) {
+    if (b.descs.size() < 2 || b.descs.size() > (1u << (32 - kSpreadShift))) return false;
     for (const XInfo& x : b.xinfo)
         if (x.signal || x.wait) return false;
     for (const ReqDesc& d : b.descs)
         if (d.kind == K_LL || d.op == OP_SIGNAL) return false;
+    if (allow_pair) pair_requests(b);
+    const size_t n = b.descs.size();
+    auto unpair = [&]() {
+        for (ReqDesc& d : b.descs) d.pair = 0;
+        return false;
+    };
     std::vector<uint32_t> items(n);
     uint64_t total = 0;
     for (size_t r = 0; r < n; r++) {
-        items[r] = desc_items(b.descs[r], ub);
-        if (items[r] > (1u << kSpreadShift)) return false;
+        // the second member of a pair runs inside its partner's items
+        items[r] = (r > 0 && b.descs[r - 1].pair) ? 0u : desc_items(b.descs[r], ub);
+        if (items[r] > (1u << kSpreadShift)) return unpair();
         total += items[r];
     }
     // chunk c of request r at relative position (2c + 1) / (2 n_r); ties by r
@@ -253,6 +311,7 @@ uint32_t write_device_table(void* dst, const HostBatch& b, int ub, uint64_t tick
     h->claim = claim;
     auto* prefix = reinterpret_cast<uint32_t*>(reinterpret_cast<char*>(dst) + sizeof(BatchHeader));
     uint32_t items = fill_prefix(prefix, b, ub);
+    if (!b.order.empty()) items = (uint32_t)b.order.size();  // spread: the item table (pairs share items)
     size_t off = sizeof(BatchHeader) + pad16((n + 1) * 4);
     if (!b.gm.empty()) {
         std::memcpy(reinterpret_cast<char*>(dst) + off, b.gm.data(), n * 4);
@@ -416,6 +475,7 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
         out.blob.clear();
         std::vector<uint32_t> prefix(b.descs.size() + 1);
         out.total_items = fill_prefix(prefix.data(), b, out.ub);
+        if (!b.order.empty()) out.total_items = (uint32_t)b.order.size();
     }
 }
 

@@ -76,7 +76,7 @@ struct alignas(16) ReqDesc {
     uint8_t ph;             // phased 16-B units (kPh*), 0 = plain vectors; see below
     uint8_t l2_64;          // 1: short segments (< kSparseSeg B) -> loads carry the .L2::64B prefetch-size hint
     uint8_t xub;            // exchange plans: this request's vectors per thread per item (0 = the batch's ub)
-    uint8_t pad3;
+    uint8_t pair;           // spread plans: 1 = request r + 1 runs in this request's items (batch.cpp pair_requests)
 };
 
 // Phased units (batch.cpp phase_batch).  A closed-form request whose common
@@ -178,6 +178,11 @@ constexpr uint32_t kXClaim = 4;
 // DRAM-activation-bound 8-B x-face cells overlap the bandwidth-bound dense
 // rows instead of following them.  Non-exchange batches only.
 constexpr int kSpreadShift = 20;
+// Paired requests (batch.cpp pair_requests): two requests that walk the same
+// lattice of short segments a few bytes apart -- the +x and -x faces of a halo
+// variable touch the two ends of the same rows -- run in the same items, the
+// same thread moving vector v of both (loads of both, then stores of both), so
+// each DRAM row is opened once for all four x-face accesses instead of twice.
 
 // A small batch carried in the kernel parameters.
 template <int CAP>

@@ -478,6 +478,51 @@ __device__ __forceinline__ void run_seg(const ReqDesc& S, const ReqDesc& D, uint
     }
 }
 
+// A paired item (device_desc.h, batch.cpp pair_requests): requests A and B
+// walk the same lattice of short (unphased) segments a few bytes apart; each
+// thread loads vector v of both, then stores both, so the DRAM rows they share
+// are opened once.  Same vector width on all four sides.
+template <int LW, bool SONLY>
+__device__ __forceinline__ void run_pair(const ReqDesc& SA, const ReqDesc& DA, const ReqDesc& SB, const ReqDesc& DB,
+                                         uint32_t v0, int ub, bool pdlw) {
+    // up to two slots in flight (four loads per thread); spread plans pair at
+    // ub <= 2 (halo.cpp make_table)
+    constexpr int PU = 2;
+    const int lw = LW >= 0 ? LW : SA.lw;
+    const uint32_t nvec = SA.nvec;
+    const uint8_t* sa = reinterpret_cast<const uint8_t*>(SA.ptr);
+    const uint8_t* sb = reinterpret_cast<const uint8_t*>(SB.ptr);
+    const bool ha = SA.l2_64 != 0, hb = SB.l2_64 != 0;
+    for (int u0 = 0; u0 < ub; u0 += PU) {
+        uint4 a[PU], b[PU];
+#pragma unroll
+        for (int k = 0; k < PU; k++) {
+            const uint32_t v = v0 + (uint32_t)((u0 + k) * kThreads) + threadIdx.x;
+            if (u0 + k < ub && v < nvec) {
+                const uint8_t* pa = sa + vec_offset<LW, SONLY>(SA, v);
+                const uint8_t* pb = sb + vec_offset<LW, SONLY>(SB, v);
+                if (pdlw) {
+                    pdl_wait();
+                    pdlw = false;
+                }
+                a[k] = ld_vec<true, LW>(pa, lw, ha);
+                b[k] = ld_vec<true, LW>(pb, lw, hb);
+            }
+        }
+        uint8_t* da = reinterpret_cast<uint8_t*>(DA.ptr);
+        uint8_t* db = reinterpret_cast<uint8_t*>(DB.ptr);
+#pragma unroll
+        for (int k = 0; k < PU; k++) {
+            const uint32_t v = v0 + (uint32_t)((u0 + k) * kThreads) + threadIdx.x;
+            if (u0 + k < ub && v < nvec) {
+                st_vec<LW>(da + vec_offset<LW, SONLY>(DA, v), lw, a[k]);
+                st_vec<LW>(db + vec_offset<LW, SONLY>(DB, v), lw, b[k]);
+            }
+        }
+    }
+    if (pdlw) pdl_wait();
+}
+
 // Largest r with prefix[r] <= item (prefix strictly increasing, prefix[0] = 0).
 __device__ __forceinline__ uint32_t find_request(const uint32_t* prefix, uint32_t nreq, uint32_t item) {
     uint32_t lo = 0, hi = nreq;
@@ -588,10 +633,11 @@ __device__ __forceinline__ uint64_t globaltimer() {
 // batch is in the parameters: wait for the preceding grid just before the
 // first global-memory access (the first item's data loads).
 template <bool XCHG, int LW, bool SONLY, bool GW, bool PH, bool INPLACE = false, int UNR = kUnroll,
-          bool LAZYW = false, bool SEG = false>
+          bool LAZYW = false, bool SEG = false, bool PAIR = false>
 __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa) {
     __shared__ ReqDesc sd;
     __shared__ ReqDesc sa;
+    __shared__ ReqDesc sd2, sa2;  // the partner of a paired request (plain device-table batches)
     __shared__ XInfo sx;
     __shared__ int s_ok;
     uint64_t epoch = 0;
@@ -685,6 +731,12 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             copy_words(&sd, tv.descs + r, kWords, 0);
             if constexpr (XCHG) copy_words(&sx, tv.xinfo + r, kXWords, 32);
             copy_words(&sa, tv.aux + r, kWords, 64);  // destination descriptor (aux[r], see HostBatch::add)
+            if constexpr (!XCHG && PAIR) {
+                if (tv.order && tv.descs[r].pair) {  // paired request: its partner r + 1 too
+                    copy_words(&sd2, tv.descs + r + 1, kWords, 128);
+                    copy_words(&sa2, tv.aux + r + 1, kWords, 192);
+                }
+            }
             __syncthreads();
             if constexpr (XCHG) {
                 if (sx.parity_stride) {  // double-buffered window: pack writes it, unpack reads it
@@ -698,7 +750,8 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             }
             cur = r;
         }
-        const int ubr = XCHG && S->xub ? (int)S->xub : (int)tv.ub;  // exchange requests carry their own item size
+        // exchange requests and the dense requests of spread plans carry their own item size
+        const int ubr = S->xub ? (int)S->xub : (int)tv.ub;
         const uint32_t v0 = local * (uint32_t)(kThreads * ubr);
         bool run = true;
         uint64_t tr0 = 0, tr1 = 0, tr2 = 0;
@@ -733,6 +786,8 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         }
         if constexpr (SEG && !XCHG) {
             run_seg<kSegUnroll>(*S, *D, v0, (int)tv.ub, !waited);
+        } else if (!XCHG && PAIR && S->pair) {
+            run_pair<LW, SONLY>(sd, sa, sd2, sa2, v0, ubr, !waited);
         } else {
             if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, ubr, xa,
                                                               (uint32_t)epoch, !waited);
@@ -847,6 +902,9 @@ template <int V> struct VarT {
     // (tools/pack_probe.py: 1 MiB x 1024 packs 4.74 -> 6.08 TB/s from 3 to 5
     // CTAs/SM); exchange kernels (flags, tracing) keep their registers.
     static constexpr int MINB = (V == 7 || V == 9) ? DDT_V7_MINB : ((V == 8 || V == 10) ? DDT_V8_MINB : DDT_MINB);
+    // paired requests (device-table spread plans): the one-slot variants only
+    // (batch.cpp kPairVariants), so the register budget of the others is untouched
+    static constexpr bool PAIR = V == 9 || V == 7 || V == 4;
     // exchange kernels: every request moves at most kXchgUb vectors per thread
     // per item (sender and receiver chunk alike), so two load slots suffice;
     // >= 4 resident CTAs per SM (<= 64 registers) keep one-CTA-per-item
@@ -861,7 +919,7 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_dev(const u
     pdl_trigger();
     pdl_wait();  // the table may come from a copy just before this launch
     fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_DEV, VarT<V>::UNR, false,
-               VarT<V>::SEG>(view_of(table), nullptr);
+               VarT<V>::SEG, VarT<V>::PAIR>(view_of(table), nullptr);
 }
 
 template <int CAP, int V>

@@ -186,7 +186,8 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
     for (const auto& d : b.descs) items += desc_items(d, ub);
     const char* ga = DDT_KNOB("DDT_GROUP_ALWAYS");  // tests: exercise grouping on small plans
     const char* sp = DDT_KNOB("DDT_SPREAD");  // 0: group equal requests instead of spreading every request
-    const bool many = items > 8ull * (uint64_t)sm_count;
+    const char* sa = DDT_KNOB("DDT_SPREAD_ALWAYS");  // tests: spread (and pair) small plans too
+    const bool many = items > 8ull * (uint64_t)sm_count || (sa && sa[0] == '1' && force_ub <= 0);
     bool spread = false;
     if (many && !(sp && sp[0] == '0')) {
         // spread plans run one CTA per item (batch.cpp grid_mode_for): with one
@@ -199,11 +200,27 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
         for (const ReqDesc& d : b.descs) sparse |= d.l2_64 || b.aux[d.aux].l2_64;
         const char* su = DDT_KNOB("DDT_SPREAD_UB");  // experiments: item size of spread plans
         const int sub = force_ub > 0 ? ub : (su ? std::max(1, std::min(4, atoi(su))) : (sparse ? 1 : ub));
+        // dense requests of a sparse plan may keep larger items of their own
+        // (ReqDesc::xub): DDT_SPREAD_DENSE_UB (experiments)
+        const char* du = DDT_KNOB("DDT_SPREAD_DENSE_UB");
+        const int dub = du ? std::max(0, std::min(4, atoi(du))) : 0;
+        if (sparse && dub > sub && force_ub <= 0)
+            for (ReqDesc& d : b.descs)
+                if (!d.l2_64 && !b.aux[d.aux].l2_64 && d.op != OP_SIGNAL) d.xub = (uint8_t)dub;
         spread = spread_items(b, sub);
+        if (!spread)
+            for (ReqDesc& d : b.descs) d.xub = 0;
         if (spread) ub = sub;
     }
     if (!spread && (many || (ga && ga[0] == '1'))) group_equal_requests(b, ub);
     make_launchable(b, !spread, l, sm_count, ub);
+    bool paired = false;
+    for (const ReqDesc& d : b.descs) paired |= d.pair != 0;
+    if (paired && !pair_variant(l.variant)) {  // the chosen instance cannot run pairs: undo them
+        for (ReqDesc& d : b.descs) d.pair = 0;
+        spread_items(b, ub, false);
+        make_launchable(b, false, l, sm_count, ub);
+    }
     if (l.form != 3) return DDT_OK;
     std::vector<uint8_t> host(device_table_bytes(b));
     write_device_table(host.data(), b, l.ub, l.ticket, l.claim);

@@ -75,12 +75,16 @@ def _check(arrs, local, dirs, before=None):
     ((5, 6, 7), ALL_DIRS, 2, 4),
     ((9, 4, 3), FACE_DIRS, 1, 2),
 ])
-@pytest.mark.parametrize("group", [False, True])
+@pytest.mark.parametrize("group", [False, True, "spread"])
 def test_halo_small(ddt, mode, graph, local, dirs, nvars, cfg, group, monkeypatch):
     """group=True: equal-size requests interleaved chunk by chunk even though the
-    plan is one wave (the default only groups multi-wave plans)."""
+    plan is one wave (the default only groups multi-wave plans); "spread": the
+    multi-wave plain-plan form (explicit spread item table, one CTA per item,
+    +x / -x style requests paired in the same items) forced on a small plan."""
     import torch
-    if group:
+    if group == "spread":
+        monkeypatch.setenv("DDT_SPREAD_ALWAYS", "1")
+    elif group:
         monkeypatch.setenv("DDT_GROUP_ALWAYS", "1")
     q, arrs, h, comm = _setup(ddt, local, dirs, nvars, mode, graph, cfg)
     for it in range(4):

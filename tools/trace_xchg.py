@@ -7,22 +7,24 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
 import paper_conf_cluster_chukzsp20_b200 as ddt  # noqa: E402
-from ddt_inputs import halo_messages, FACE_DIRS  # noqa: E402
+from ddt_inputs import halo_messages, FACE_DIRS, ALL_DIRS  # noqa: E402
 
 torch.cuda.set_device(0)
-local = (128, 128, 128)
-a = torch.zeros((130, 130, 130), dtype=torch.int64, device="cuda")
-msgs = halo_messages(0, 1, local, dirs=FACE_DIRS)
-sends = [(m["peer"], m["tag"], ddt.Type.from_spec(m["send_spec"]), a, 1) for m in msgs]
-recvs = [(m["recv_peer"], m["recv_tag"], ddt.Type.from_spec(m["recv_spec"]), a, 1) for m in msgs]
+comb = len(sys.argv) > 1 and sys.argv[1] == "comb"
+local = (512, 512, 512) if comb else (128, 128, 128)
+nvars = 4 if comb else 1
+arrs = [torch.zeros(tuple(n + 2 for n in local), dtype=torch.int64, device="cuda") for _ in range(nvars)]
+msgs = halo_messages(0, 1, local, dirs=ALL_DIRS if comb else FACE_DIRS, nvars=nvars)
+sends = [(m["peer"], m["tag"], ddt.Type.from_spec(m["send_spec"]), arrs[m["var"]], 1) for m in msgs]
+recvs = [(m["recv_peer"], m["recv_tag"], ddt.Type.from_spec(m["recv_spec"]), arrs[m["var"]], 1) for m in msgs]
 h = ddt.Halo(ddt.Queue(), ddt.Comm.single(0), sends, recvs, mode="p2p", graph=False)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 for _ in range(5):
     h.exchange()
 torch.cuda.synchronize()
 for it in range(3):
-    read = h.trace(8192)
-    flush.fill_(it)
+    read = h.trace(200000)
+    flush.max()
     torch.cuda.synchronize()
     h.exchange()
     r = read()
@@ -30,7 +32,7 @@ for it in range(3):
     ph = {k: (r[k] - t) / 1e3 for k in ("t0", "t1", "t2", "t3")}
     pack = r["op"] == 0
     unp = r["op"] == 1
-    print(f"iter {it}: records {len(r)}  span {ph['t3'].max():.2f} us")
+    print(f"iter {it}: records {len(r)}  span {ph['t3'].max():.2f} us  CTAs {len(set(r['cta'].tolist()))}")
     for name, m in (("pack", pack), ("unpack", unp)):
         if m.any():
             print(f"  {name:6s} start [{ph['t0'][m].min():.2f}, {ph['t0'][m].max():.2f}]  wait-done max {ph['t1'][m].max():.2f}"

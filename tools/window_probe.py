@@ -20,6 +20,10 @@ from ddt_inputs import FACE_DIRS, ALL_DIRS  # noqa: E402
 
 VARIANTS = {
     "direct": {},
+    "direct_nopair": {"DDT_NO_PAIR": "1"},
+    "direct_ub2": {"DDT_SPREAD_UB": "2"},
+    "direct_dense4": {"DDT_SPREAD_DENSE_UB": "4"},
+    "direct_dense2": {"DDT_SPREAD_DENSE_UB": "2"},
     "window": {"DDT_SELF_VIA_WINDOW": "1"},
     "window_xgrid1": {"DDT_SELF_VIA_WINDOW": "1", "DDT_XGRID_MODE": "1"},
     "window_xgrid2": {"DDT_SELF_VIA_WINDOW": "1", "DDT_XGRID_MODE": "2"},
@@ -33,7 +37,7 @@ def build(cfg, names):
     wls = {}
     base_env = dict(os.environ)
     for n in names:
-        for k in ("DDT_SELF_VIA_WINDOW", "DDT_XGRID_MODE", "DDT_XCLAIM", "DDT_NO_LL"):
+        for k in ("DDT_SELF_VIA_WINDOW", "DDT_XGRID_MODE", "DDT_XCLAIM", "DDT_NO_LL", "DDT_NO_PAIR", "DDT_SPREAD_UB", "DDT_SPREAD_DENSE_UB"):
             os.environ.pop(k, None)
         os.environ.update(VARIANTS[n])
         ddt.reload_env()
