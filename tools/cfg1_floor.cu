@@ -10,7 +10,19 @@
 //   faces8   : one thread per 8-B cell (98,304 threads)
 //   phased   : z / y face rows as 8-B head + 63 x 16-B + 8-B tail, x-face
 //              cells 8 B (66,048 threads; what the library's variant 7 does)
+//   tma3d    : z / y faces moved by the Tensor Memory Accelerator -- a 3-D
+//              tensor map over the 130^3 array, boxes of 128 x 4 rows loaded
+//              (cp.async.bulk.tensor ... mbarrier::complete_tx) into shared
+//              memory and stored to the ghost plane (cp.async.bulk.tensor
+//              global.shared::cta), one elected thread per CTA; x faces by
+//              threads (one thread per row, both cells: TMA boxes need a
+//              16-B inner extent, an x-face cell is 8 B)
+//   bulk1d   : z / y face rows as one 1-D bulk copy (cp.async.bulk, no tensor
+//              map) of the 16-B-aligned 1008-B body + 8-B head / tail by
+//              threads; x faces as in tma3d
 // Prints one JSON line per kernel.  Build: nvcc -gencode arch=compute_100a,code=sm_100a -O3 -o cfg1_floor cfg1_floor.cu
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_runtime.h>
 #include <cstdio>
 #include <cstdint>
@@ -136,6 +148,127 @@ __global__ void xpair_pdl(double* __restrict__ a) {
         pdl_wait();
     }
 }
+// ---- TMA / bulk-async variants
+__device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t n) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(n) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect(uint64_t* b, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t phase) {
+    uint32_t done = 0;
+    while (!done)
+        asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                     : "=r"(done) : "r"(smem_u32(b)), "r"(phase) : "memory");
+}
+__device__ __forceinline__ void bulk_commit_wait() {
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+constexpr int kRowsPerCta = 4;                    // rows of 128 doubles per TMA box
+constexpr int kDenseCtas = 4 * 128 / kRowsPerCta;  // 4 dense faces x 128 rows
+constexpr int kXCtas = (16384 + 255) / 256;        // x faces: one thread per row (both cells)
+
+// face f, row block rb -> box origin of the source and destination (x, y, z)
+__device__ __forceinline__ void face_box(int f, int rb, int& sx, int& sy, int& sz, int& dy, int& dz) {
+    const int r0 = 1 + rb * kRowsPerCta;
+    sx = 1;
+    if (f == 0) { sy = r0; sz = 1; dy = r0; dz = 129; }
+    else if (f == 1) { sy = r0; sz = 128; dy = r0; dz = 0; }
+    else if (f == 2) { sy = 1; sz = r0; dy = 129; dz = r0; }
+    else { sy = 128; sz = r0; dy = 0; dz = r0; }
+}
+
+__device__ __forceinline__ void xpair_thread(double* __restrict__ a, int c) {
+    const int z = 1 + c / 128, y = 1 + c % 128;
+    const double v1 = __ldg(a + idx(z, y, 1)), v2 = __ldg(a + idx(z, y, 128));
+    a[idx(z, y, 129)] = v1;
+    a[idx(z, y, 0)] = v2;
+}
+
+__device__ __forceinline__ void tma_load3(const CUtensorMap* m, void* dst, uint64_t* bar, int x, int y, int z) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4}], [%5];"
+        ::"r"(smem_u32(dst)), "l"(m), "r"(x), "r"(y), "r"(z), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void tma_store3(const CUtensorMap* m, const void* src, int x, int y, int z) {
+    asm volatile("cp.async.bulk.tensor.3d.global.shared::cta.bulk_group [%0, {%1, %2, %3}], [%4];"
+                 ::"l"(m), "r"(x), "r"(y), "r"(z), "r"(smem_u32(src)) : "memory");
+}
+
+// two tensor maps per array: boxes (128, 4, 1) for z faces, (128, 1, 4) for y faces
+__global__ void __launch_bounds__(256) tma3d_pdl(double* __restrict__ a, const CUtensorMap* __restrict__ mz,
+                                                 const CUtensorMap* __restrict__ my) {
+    pdl_trigger();
+    __shared__ alignas(128) unsigned char buf[128 * 8 * kRowsPerCta];
+    __shared__ alignas(8) uint64_t bar;
+    const int b = blockIdx.x;
+    if (b < kDenseCtas) {
+        if (threadIdx.x == 0) {
+            const int f = b / (128 / kRowsPerCta), rb = b % (128 / kRowsPerCta);
+            int sx, sy, sz, dy, dz;
+            face_box(f, rb, sx, sy, sz, dy, dz);
+            // the tensor map operand must be the __grid_constant__ parameter's own
+            // address (a pointer select makes the compiler copy the maps to local
+            // memory, which TMA cannot read: illegal instruction)
+            mbar_init(&bar, 1);
+            pdl_wait();
+            mbar_expect(&bar, sizeof(buf));
+            const CUtensorMap* m = f < 2 ? mz : my;  // tensor maps in global memory (64-B aligned)
+            tma_load3(m, buf, &bar, sx, sy, sz);
+            mbar_wait(&bar, 0);
+            tma_store3(m, buf, sx, dy, dz);
+            bulk_commit_wait();
+        } else {
+            pdl_wait();
+        }
+    } else {
+        const int c = (b - kDenseCtas) * 256 + threadIdx.x;
+        pdl_wait();
+        if (c < 16384) xpair_thread(a, c);
+    }
+}
+
+// 1-D bulk copies: each dense row = head (8 B) + 16-B-aligned body (1008 B) + tail (8 B)
+__global__ void __launch_bounds__(256) bulk1d_pdl(double* __restrict__ a) {
+    pdl_trigger();
+    __shared__ alignas(128) unsigned char buf[kRowsPerCta][1024];
+    __shared__ alignas(8) uint64_t bar;
+    const int b = blockIdx.x;
+    if (b < kDenseCtas) {
+        const int f = b / (128 / kRowsPerCta), rb = b % (128 / kRowsPerCta);
+        long long s[kRowsPerCta], d[kRowsPerCta];
+        for (int k = 0; k < kRowsPerCta; k++) face_rows(f, rb * kRowsPerCta + k, s[k], d[k]);
+        if (threadIdx.x == 0) {
+            mbar_init(&bar, 1);
+            pdl_wait();
+            mbar_expect(&bar, kRowsPerCta * 1008);
+            for (int k = 0; k < kRowsPerCta; k++)
+                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                             ::"r"(smem_u32(buf[k])), "l"(reinterpret_cast<const char*>(a + s[k]) + 16), "r"(1008),
+                             "r"(smem_u32(&bar)) : "memory");
+            mbar_wait(&bar, 0);
+            for (int k = 0; k < kRowsPerCta; k++)
+                asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+                             ::"l"(reinterpret_cast<char*>(a + d[k]) + 16), "r"(smem_u32(buf[k])), "r"(1008)
+                             : "memory");
+            bulk_commit_wait();
+        } else if (threadIdx.x <= 2 * kRowsPerCta) {  // heads and tails (x = 1 and x = 128)
+            pdl_wait();
+            const int k = (threadIdx.x - 1) / 2, x = (threadIdx.x - 1) % 2 ? 128 : 1;
+            a[d[k] + x] = __ldg(a + s[k] + x);
+        } else {
+            pdl_wait();
+        }
+    } else {
+        const int c = (b - kDenseCtas) * 256 + threadIdx.x;
+        pdl_wait();
+        if (c < 16384) xpair_thread(a, c);
+    }
+}
+
 template <class... A>
 static void launch_pdl(void (*k)(A...), int grid, cudaStream_t s, A... args) {
     cudaLaunchConfig_t cfg = {};
@@ -183,24 +316,118 @@ static double graph_us(F launch, int R, int K) {
     return best * 1e3 / K;
 }
 
-int main() {
-    const int R = 96, K = 500;
-    double* arr[R];
+int main(int argc, char** argv) {
+    setvbuf(stdout, NULL, _IONBF, 0);
+    const bool tma_only = argc > 1;  // diagnostic: skip the thread kernels
+    const int R = argc > 1 ? 2 : 96, K = 500;
+    double* arr[96];
     for (int r = 0; r < R; r++) {
         cudaMalloc(&arr[r], PLANE * N * sizeof(double));
         cudaMemset(arr[r], r, PLANE * N * sizeof(double));
     }
     const int g8 = (6 * 16384 + 255) / 256, gp = (4 * 128 * 65 + 2 * 16384 + 255) / 256;
-    double te = graph_us([&](cudaStream_t s, int r) { empty_k<<<gp, 256, 0, s>>>(arr[r]); }, R, K);
-    double t8 = graph_us([&](cudaStream_t s, int r) { faces8<<<g8, 256, 0, s>>>(arr[r]); }, R, K);
-    double tp = graph_us([&](cudaStream_t s, int r) { phased<<<gp, 256, 0, s>>>(arr[r]); }, R, K);
+    double te = 0, t8 = 0, tp = 0, teb = 0, t8b = 0, tep = 0, tpp = 0, txp = 0;
     Big big{};
-    double teb = graph_us([&](cudaStream_t s, int r) { empty_big<<<gp, 256, 0, s>>>(arr[r], big); }, R, K);
-    double t8b = graph_us([&](cudaStream_t s, int r) { faces8_big<<<g8, 256, 0, s>>>(arr[r], big); }, R, K);
     const int gx = (4 * 128 * 65 + 16384 + 255) / 256;
-    double tep = graph_us([&](cudaStream_t s, int r) { launch_pdl(empty_pdl, gp, s, arr[r]); }, R, K);
-    double tpp = graph_us([&](cudaStream_t s, int r) { launch_pdl(phased_pdl, gp, s, arr[r]); }, R, K);
-    double txp = graph_us([&](cudaStream_t s, int r) { launch_pdl(xpair_pdl, gx, s, arr[r]); }, R, K);
+    if (!tma_only) {
+    te = graph_us([&](cudaStream_t s, int r) { empty_k<<<gp, 256, 0, s>>>(arr[r]); }, R, K);
+    fprintf(stderr, "done te %.3f\n", te);
+    t8 = graph_us([&](cudaStream_t s, int r) { faces8<<<g8, 256, 0, s>>>(arr[r]); }, R, K);
+    fprintf(stderr, "done t8 %.3f\n", t8);
+    tp = graph_us([&](cudaStream_t s, int r) { phased<<<gp, 256, 0, s>>>(arr[r]); }, R, K);
+    fprintf(stderr, "done tp %.3f\n", tp);
+    teb = graph_us([&](cudaStream_t s, int r) { empty_big<<<gp, 256, 0, s>>>(arr[r], big); }, R, K);
+    fprintf(stderr, "done teb %.3f\n", teb);
+    t8b = graph_us([&](cudaStream_t s, int r) { faces8_big<<<g8, 256, 0, s>>>(arr[r], big); }, R, K);
+    fprintf(stderr, "done t8b %.3f\n", t8b);
+    tep = graph_us([&](cudaStream_t s, int r) { launch_pdl(empty_pdl, gp, s, arr[r]); }, R, K);
+    fprintf(stderr, "done tep %.3f\n", tep);
+    tpp = graph_us([&](cudaStream_t s, int r) { launch_pdl(phased_pdl, gp, s, arr[r]); }, R, K);
+    fprintf(stderr, "done tpp %.3f\n", tpp);
+    txp = graph_us([&](cudaStream_t s, int r) { launch_pdl(xpair_pdl, gx, s, arr[r]); }, R, K);
+    fprintf(stderr, "done txp %.3f\n", txp);
+    }
+    // TMA: tensor maps per replica array
+    PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
+    cudaDriverEntryPointQueryResult qr;
+    cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void**)&enc, cudaEnableDefault, &qr);
+    static CUtensorMap mz[96], my[96];
+    for (int r = 0; r < R && enc; r++) {
+        cuuint64_t dims[3] = {130, 130, 130};
+        cuuint64_t strides[2] = {130 * 8, 130 * 130 * 8};
+        cuuint32_t boxz[3] = {128, (cuuint32_t)kRowsPerCta, 1}, boxy[3] = {128, 1, (cuuint32_t)kRowsPerCta};
+        cuuint32_t es[3] = {1, 1, 1};
+        CUresult c1 = enc(&mz[r], CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, arr[r], dims, strides, boxz, es,
+                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        CUresult c2 = enc(&my[r], CU_TENSOR_MAP_DATA_TYPE_FLOAT64, 3, arr[r], dims, strides, boxy, es,
+                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+        if (c1 != CUDA_SUCCESS || c2 != CUDA_SUCCESS) { printf("tensor map encode failed %d %d\n", c1, c2); return 1; }
+    }
+    printf("{\"tensor_maps\": %s}\n", enc ? "\"ok\"" : "\"no entry point\"");
+    CUtensorMap* dmaps = nullptr;  // [2R]: z-face and y-face maps of each replica, in global memory
+    cudaMalloc(&dmaps, sizeof(CUtensorMap) * 2 * R);
+    for (int r = 0; r < R; r++) {
+        cudaMemcpy(dmaps + 2 * r, &mz[r], sizeof(CUtensorMap), cudaMemcpyHostToDevice);
+        cudaMemcpy(dmaps + 2 * r + 1, &my[r], sizeof(CUtensorMap), cudaMemcpyHostToDevice);
+    }
+    {  // 1-D bulk copies first (no tensor maps)
+        launch_pdl(bulk1d_pdl, kDenseCtas + kXCtas, 0, arr[0]);
+        cudaError_t se = cudaDeviceSynchronize();
+        fprintf(stderr, "bulk1d: sync %s\n", cudaGetErrorString(se));
+        if (se != cudaSuccess) return 3;
+    }
+    const int gt = kDenseCtas + kXCtas;
+    auto launch_tma = [&](cudaStream_t s, int r) {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(gt);
+        cfg.blockDim = dim3(256);
+        cfg.stream = s;
+        cudaLaunchAttribute at[1];
+        at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+        at[0].val.programmaticStreamSerializationAllowed = 1;
+        cfg.attrs = at;
+        cfg.numAttrs = 1;
+        double* ap = arr[r];
+        const CUtensorMap* pz = dmaps + 2 * r;
+        const CUtensorMap* py = dmaps + 2 * r + 1;
+        void* args[3] = {&ap, &pz, &py};
+        cudaError_t e = cudaLaunchKernelExC(&cfg, (const void*)tma3d_pdl, args);
+        if (e != cudaSuccess) fprintf(stderr, "tma launch: %s\n", cudaGetErrorString(e));
+    };
+    // the tma3d kernel faults (illegal instruction): the halo rows start at
+    // x = 1, 8 mod 16, and a tensor box's innermost start must be 16-B aligned
+    // on B200 (tools/tma_min.cu) -- so it is not timed; bulk1d is
+    (void)launch_tma;
+    double ttma = -1.0;
+    fprintf(stderr, "done ttma %.3f\n", ttma);
+    double tbulk = graph_us([&](cudaStream_t s, int r) { launch_pdl(bulk1d_pdl, gt, s, arr[r]); }, R, K);
+    fprintf(stderr, "done tbulk %.3f\n", tbulk);
+    // correctness of the TMA / bulk kernels against the thread kernel on one array
+    {
+        const size_t n = PLANE * N;
+        double *h0 = new double[n], *h1 = new double[n], *h2 = new double[n];
+        for (size_t i = 0; i < n; i++) h0[i] = (double)(i * 2654435761ull % 1000003);
+        auto run = [&](int which, double* out) {
+            cudaMemcpy(arr[0], h0, n * 8, cudaMemcpyHostToDevice);
+            if (which == 0) launch_pdl(xpair_pdl, gx, 0, arr[0]);
+            else if (which == 1) launch_pdl(bulk1d_pdl, gt, 0, arr[0]);
+            else launch_pdl(bulk1d_pdl, gt, 0, arr[0]);
+            cudaDeviceSynchronize();
+            cudaMemcpy(out, arr[0], n * 8, cudaMemcpyDeviceToHost);
+        };
+        run(0, h1);
+        run(1, h2);
+        size_t bad1 = 0, bad2 = 0;
+        for (size_t i = 0; i < n; i++) bad1 += h1[i] != h2[i];
+        run(2, h2);
+        for (size_t i = 0; i < n; i++) bad2 += h1[i] != h2[i];
+        printf("{\"check\": \"bulk1d vs threads\", \"differing\": %zu, \"again\": %zu}\n", bad1, bad2);
+        delete[] h0; delete[] h1; delete[] h2;
+    }
+    printf("{\"kernel\": \"tma3d_pdl\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gt, ttma);
+    printf("{\"kernel\": \"bulk1d_pdl\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gt, tbulk);
     printf("{\"kernel\": \"empty_pdl\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gp, tep);
     printf("{\"kernel\": \"phased_pdl\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gp, tpp);
     printf("{\"kernel\": \"xpair_pdl\", \"ctas\": %d, \"us_per_step\": %.3f}\n", gx, txp);
