@@ -35,13 +35,17 @@ def test_bench_n1():
     _check(_line(r.stdout), 1)
 
 
-def test_bench_n2_shared_gpu():
+@pytest.mark.parametrize("mode,port", [("p2p", 29533), ("p2p_direct", 29534)])
+def test_bench_n2_shared_gpu(mode, port):
+    """N = 2: the K steps of the flagged P2P exchange are one captured CUDA graph
+    (device-resident epoch), as at N = 1."""
     env = dict(os.environ, DDT_BENCH_BACKEND="gloo", DDT_BENCH_SHARE_GPU="1", DDT_BENCH_REPLICAS="4")
     r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
-                        "--master-addr", "127.0.0.1", "--master-port", "29533", "bench.py", "--gpus", "2",
-                        "--steps", "10", "--warmup", "3", "--no-extras", "--mode", "p2p"],
+                        "--master-addr", "127.0.0.1", "--master-port", str(port), "bench.py", "--gpus", "2",
+                        "--steps", "10", "--warmup", "3", "--no-extras", "--mode", mode],
                        cwd=ROOT, capture_output=True, text=True, timeout=900, env=env)
     assert r.returncode == 0, (r.stdout[-2000:], r.stderr[-3000:])
     d = _line(r.stdout)
     _check(d, 2)
-    assert d["config"]["mode"] == "p2p"
+    assert d["config"]["mode"] == mode
+    assert d["config"]["launch"].startswith("K-step CUDA graph"), d["config"]["launch"]
