@@ -294,50 +294,66 @@ def e2e_steps(torch, wl, K, dist_on):
     return ms, nb, nb
 
 
-def e2e_zero_copy(torch, ddt, rank, P, local, dirs, nvars, comm, mode, K, dist_on):
+def e2e_zero_copy(torch, ddt, rank, P, local, dirs, nvars, comm, mode, K, dist_on, breakdown=False):
     """Zero-copy flow with HOST arrays: the halo plan is built on pinned host
     arrays (include/ddt.h: data buffers may be page-locked host memory), so
     each ddt_exchange's fused kernels read the send faces from host memory and
     write the received ghosts into host memory over PCIe (remote messages
     travel through device staging + NCCL): per step exactly the halo bytes
     cross the bus, and the step's result is in host memory when the stream
-    completes.  Returns (ms per step, host->device bytes, device->host bytes)."""
+    completes.  Returns (ms per step, host->device bytes, device->host bytes,
+    breakdown) -- breakdown (rank 0, N = 1): the same flow for the dense (y / z)
+    faces alone and the x faces (one 8-B cell per row: one PCIe transaction per
+    cell) alone, with their bytes."""
     shape = tuple(n + 2 for n in local)
     g = torch.Generator().manual_seed(seed(2, rank))
     hosts = [torch.randint(-2**62, 2**62, shape, dtype=torch.int64, generator=g).pin_memory() for _ in range(nvars)]
-    msgs = halo_messages(rank, P, local, dirs=dirs, nvars=nvars)
     cache = {}
 
     def T(spec):
         if repr(spec) not in cache:
             cache[repr(spec)] = ddt.Type.from_spec(spec)
         return cache[repr(spec)]
-    q = ddt.Queue()
-    sends = [(m["peer"], m["tag"], T(m["send_spec"]), hosts[m["var"]], 1) for m in msgs]
-    recvs = [(m["recv_peer"], m["recv_tag"], T(m["recv_spec"]), hosts[m["var"]], 1) for m in msgs]
-    h = ddt.Halo(q, comm, sends, recvs, mode=mode, graph=False)
-    stream = torch.cuda.current_stream()
-    for _ in range(3):
-        h.exchange()
-    if dist_on:
-        import torch.distributed as dist
-        dist.barrier()
-    torch.cuda.synchronize()
-    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    s.record(stream)
-    for _ in range(K):
-        h.exchange()
-    e.record(stream)
-    torch.cuda.synchronize()
-    ms = s.elapsed_time(e) / K
+
+    def run(msgs, K):
+        q = ddt.Queue()
+        sends = [(m["peer"], m["tag"], T(m["send_spec"]), hosts[m["var"]], 1) for m in msgs]
+        recvs = [(m["recv_peer"], m["recv_tag"], T(m["recv_spec"]), hosts[m["var"]], 1) for m in msgs]
+        h = ddt.Halo(q, comm, sends, recvs, mode=mode, graph=False)
+        stream = torch.cuda.current_stream()
+        for _ in range(3):
+            h.exchange()
+        if dist_on:
+            import torch.distributed as dist
+            dist.barrier()
+        torch.cuda.synchronize()
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s.record(stream)
+        for _ in range(K):
+            h.exchange()
+        e.record(stream)
+        torch.cuda.synchronize()
+        ms = s.elapsed_time(e) / K
+        if dist_on:
+            import torch.distributed as dist
+            dist.barrier()
+        h.destroy()
+        q.destroy()
+        return ms
+
+    msgs = halo_messages(rank, P, local, dirs=dirs, nvars=nvars)
+    ms = run(msgs, K)
     h2d = sum(T(m["send_spec"]).size for m in msgs)   # send faces read from host memory
     d2h = sum(T(m["recv_spec"]).size for m in msgs)   # ghost faces written to host memory
-    if dist_on:
-        import torch.distributed as dist
-        dist.barrier()
-    h.destroy()
-    q.destroy()
-    return ms, h2d, d2h
+    bd = None
+    if breakdown:
+        bd = {}
+        for name, keep in (("dense_yz_faces", lambda d: d[2] == 0), ("x_faces", lambda d: d[2] != 0)):
+            sub = [m for m in msgs if keep(m["dir"])]
+            t = run(sub, K)
+            b = sum(T(m["send_spec"]).size for m in sub)
+            bd[name] = {"us": round(t * 1e3, 2), "bytes_each_way": b, "GBps_each_way": round(b / (t / 1e3) / 1e9, 2)}
+    return ms, h2d, d2h, bd
 
 
 def latency_floor(ddt, torch, K, flush_buf, R=96):
@@ -585,7 +601,7 @@ def main():
     ap.add_argument("--steps", type=int, default=500)
     ap.add_argument("--warmup", type=int, default=50)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--mode", default="auto", choices=["auto", "p2p", "p2p_direct", "nccl"])
+    ap.add_argument("--mode", default="auto", choices=["auto", "p2p", "p2p_direct", "nccl", "nccl_early"])
     ap.add_argument("--no-extras", action="store_true")
     ap.add_argument("--cpu-budget", type=float, default=10.0)
     args = ap.parse_args()
@@ -697,14 +713,14 @@ def main():
     # N = 1: every message is a self message (one DirectIPC launch in every mode);
     # N > 1: the three data paths differ -- measure all, report the fastest
     if args.mode == "auto":
-        modes = ["nccl", "p2p"] if not dist_on else ["p2p_direct", "p2p", "nccl"]
+        modes = ["nccl", "p2p"] if not dist_on else ["p2p_direct", "p2p", "nccl", "nccl_early"]
     else:
         modes = [args.mode]
     for mode in modes:
         try:
             # plan metadata: host all-gather over the process group; NCCL comm
             # only for the NCCL-mode data path
-            c = ddt.Comm.from_torch(dev, nccl=(mode == "nccl")) if dist_on else ddt.Comm.single(dev)
+            c = ddt.Comm.from_torch(dev, nccl=mode.startswith("nccl")) if dist_on else ddt.Comm.single(dev)
             wl = HaloWorkload(ddt, torch, rank, P, local, FACE_DIRS, 1, mode, c, 2, replicas=R, graph=False)
             capture = os.environ.get("DDT_BENCH_NO_CAPTURE") != "1"
             try:
@@ -741,21 +757,21 @@ def main():
     staged_ms = max_over_ranks(torch, staged_ms, dist_on)
     # zero-copy e2e: NCCL or P2P-window plan (P2P_DIRECT opens the receive
     # buffers through CUDA IPC, which host memory does not support)
-    e2e_mode = "nccl" if best_mode == "nccl" else "p2p"
+    e2e_mode = "nccl" if best_mode.startswith("nccl") else "p2p"
     e2e_note = None
     try:
-        e2e_ms, h2d, d2h = e2e_zero_copy(torch, ddt, rank, P, local, FACE_DIRS, 1, best["comm"], e2e_mode,
-                                         max(20, K // 5), dist_on)
+        e2e_ms, h2d, d2h, e2e_bd = e2e_zero_copy(torch, ddt, rank, P, local, FACE_DIRS, 1, best["comm"], e2e_mode,
+                                                 max(20, K // 5), dist_on, breakdown=not dist_on)
         e2e_ms = max_over_ranks(torch, e2e_ms, dist_on)
     except Exception as e:  # report the staged flow instead, say why
-        e2e_ms, h2d, d2h = staged_ms, st_h2d, st_d2h
+        e2e_ms, h2d, d2h, e2e_bd = staged_ms, st_h2d, st_d2h, None
         e2e_note = f"zero-copy flow failed ({type(e).__name__}: {e}); staged flow reported"
     clocks = sampler.stop() if sampler else None
 
     alg_bytes = wl.alg_bytes
     step_s = best["mean_ms"] / 1e3
     achieved = alg_bytes / step_s / 1e9
-    kname = "ddt_exchange_*" if (best_mode != "nccl" and dist_on) else "ddt_fused_*"
+    kname = "ddt_exchange_*" if (best_mode.startswith("p2p") and dist_on) else "ddt_fused_*"
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": hbm, "unit": "GB/s",
             "frac": round(achieved / hbm, 4), "peak_source": peak_src,
             "traffic": traffic_from_profiles(kname, "configs[1]"),
@@ -785,9 +801,9 @@ def main():
         try:
             G = 512
             loc = (G // grid[0], G // grid[1], G // grid[2])
-            c4 = ddt.Comm.from_torch(dev, nccl=(best_mode == "nccl")) if dist_on else ddt.Comm.single(dev)
-            wl4 = HaloWorkload(ddt, torch, rank, P, loc, ALL_DIRS, 4, best_mode, c4, 4)
-            ms4, _ = run_steps(torch, wl4, max(20, K // 5), 5, dist_on, None)
+            c4 = ddt.Comm.from_torch(dev, nccl=best_mode.startswith("nccl")) if dist_on else ddt.Comm.single(dev)
+            wl4 = HaloWorkload(ddt, torch, rank, P, loc, ALL_DIRS, 4, best_mode, c4, 4, graph=False)
+            ms4, _ = run_steps(torch, wl4, max(20, K // 5), 5, dist_on, None, capture=True, flush_buf=flush_buf)
             ms4 = max_over_ranks(torch, ms4, dist_on)
             if dist_on:
                 import torch.distributed as dist
@@ -802,7 +818,8 @@ def main():
                                 "remote_bytes_out_per_rank": wl4.S_remote,
                                 "nvlink_bound_us": round(wl4.S_remote / 900e9 * 1e6, 2),
                                 "launches_per_iter": wl4.launches, "mode": best_mode,
-                                "timing": "back-to-back host-issued steps (one step touches > 2x L2)"}
+                                "timing": ("K-step CUDA graph after an L2 read sweep, back to back on the same arrays "
+                                           "(one step touches > 2x L2)")}
             wl4.close()
             c4.close()
         except Exception as e:
@@ -838,7 +855,8 @@ def main():
                            l2_evict=("256 MiB read sweep enqueued before the start event (L2 holds none of the "
                                      "timed steps' data, no dirty lines to write back)")),
             "e2e": {"value": round(e2e_ms * 1e3, 2), "unit": "us/iter", "h2d_bytes_per_step": h2d,
-                    "d2h_bytes_per_step": d2h,
+                    "d2h_bytes_per_step": d2h, "breakdown": e2e_bd,
+                    "device_resident_us": round(best["mean_ms"] * 1e3, 3),
                     "flow": e2e_note or (f"zero-copy ({e2e_mode} plan): ddt_exchange on a plan over pinned HOST "
                                          "arrays; the fused kernels read the send faces from and write the ghosts "
                                          "into host memory over PCIe")},

@@ -79,10 +79,17 @@ enum ddt_xchg_mode {
     DDT_XCHG_NCCL = 0,  /* fused pack -> grouped ncclSend/ncclRecv per peer -> fused unpack */
     DDT_XCHG_P2P = 1,   /* ONE kernel: pack straight into peers' windows over NVLink,
                            release a per-message flag, unpack each message on arrival */
-    DDT_XCHG_P2P_DIRECT = 2  /* ONE kernel, pack-free (DirectIPC): gather the
+    DDT_XCHG_P2P_DIRECT = 2, /* ONE kernel, pack-free (DirectIPC): gather the
                            send layout and scatter straight into the peer's receive layout
                            through a CUDA-IPC mapping of its buffer, after the peer's
                            "ready" flag; needs closed-form (strided) receive types */
+    DDT_XCHG_NCCL_EARLY = 3  /* NCCL mode with per-peer early send (the sender
+                           sends "as soon as any packing request is completed"): the
+                           fused pack kernel counts each message's completion in device
+                           memory (the CTA finishing its last item), and each remote
+                           peer's ncclSend/ncclRecv group waits on its own stream
+                           (stream memory operation on those counters) for that peer's
+                           messages only, not for the whole pack batch */
 };
 
 typedef struct ddt_type_s* ddt_type_t;   /* opaque, library-owned, immutable after commit */
@@ -307,13 +314,13 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* comm, int32_t nsen
                              int32_t nrecv, const ddt_recv_t* recvs, int32_t mode, ddt_halo_t* out);
 /* One exchange iteration, asynchronous on the queue's stream: every send
  * packed, transferred, every receive unpacked.  NCCL mode: fused
- * pack launch -> grouped send/recv -> fused unpack launch.  P2P modes: a
- * single launch.  ddt_halo_set_graph(h, 1) replays a CUDA graph captured on
- * first use -- except for P2P plans with remote messages, whose per-exchange
- * epoch travels as a kernel argument (always one direct launch); for the same
- * reason such a plan returns DDT_ERR_STATE when called while the caller
- * captures the queue's stream (every other plan may be captured).  All ranks
- * must issue the same sequence of ddt_exchange calls.                        */
+ * pack launch -> grouped send/recv -> fused unpack launch (NCCL_EARLY: one
+ * send/recv group per remote peer on its own stream, each started when that
+ * peer's messages are packed, joined before the unpack).  P2P modes: a single
+ * launch whose exchange epoch lives on the device, so every plan can be
+ * captured into a CUDA graph by the caller (a K-step time loop) or replay its
+ * own graph (ddt_halo_set_graph(h, 1)).  All ranks must issue the same
+ * sequence of ddt_exchange calls.                                            */
 ddt_status_t ddt_exchange(ddt_halo_t h);
 ddt_status_t ddt_halo_set_graph(ddt_halo_t h, int32_t use_graph);
 /* Bound of every device-side flag wait of a P2P plan (default 10 s).  A wait

@@ -19,7 +19,7 @@ BASE_CODES = {"byte": 0, "int32": 1, "int64": 2, "float": 3, "double": 4}
 LAYOUT_KINDS = {0: "empty", 1: "strided", 2: "uniform_list", 3: "general_list"}
 STATE_NAMES = {0: "idle", 1: "pending", 2: "busy", 3: "completed"}
 DDT_PENDING, DDT_BUSY, DDT_COMPLETED = 1, 2, 3
-DDT_XCHG_NCCL, DDT_XCHG_P2P, DDT_XCHG_P2P_DIRECT = 0, 1, 2
+DDT_XCHG_NCCL, DDT_XCHG_P2P, DDT_XCHG_P2P_DIRECT, DDT_XCHG_NCCL_EARLY = 0, 1, 2, 3
 
 c_type_p = ctypes.c_void_p
 I64, I32, P = ctypes.c_int64, ctypes.c_int32, ctypes.c_void_p

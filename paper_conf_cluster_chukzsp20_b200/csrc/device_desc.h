@@ -70,7 +70,7 @@ struct alignas(16) ReqDesc {
     uint32_t list_n;        // general: number of segments per instance
     uint32_t uid_lo;        // low bits of the request UID (debug / tracing)
     uint32_t aux;           // source descriptors: index of the destination descriptor in aux[]
-    uint32_t resp_val;      // value written to *resp when the request's last item is done
+    uint32_t resp_val;      // value written to *resp when the request's last item is done (kRespIncrement: +1)
     uint64_t done_ctr;      // device u32 counter of finished items (reset by the finishing CTA)
     uint32_t nitems;        // items of this request in its batch (set at flush)
     uint8_t ph;             // phased 16-B units (kPh*), 0 = plain vectors; see below
@@ -86,6 +86,10 @@ struct alignas(16) ReqDesc {
 // -> segment s = v / vps, unit j = v % vps (vps = units per segment); the
 // body moves as 16-B accesses.  lw is 4, nvec counts units.
 constexpr uint8_t kPhOn = 1, kPhHead = 2, kPhTail = 4;
+// resp_val meaning "increment the device counter *resp" (NCCL_EARLY per-message
+// completion counters, waited on by stream memory operations) instead of
+// "store resp_val into the host-mapped slot *resp".
+constexpr uint32_t kRespIncrement = 0xffffffffu;
 
 // Sparse sides: the L2 fetches 128 B per missed line by default; a side whose
 // contiguous segments are shorter than kSparseSeg bytes loads with the PTX

@@ -802,7 +802,8 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
                     if (atomicAdd(ctr, 1u) + 1u == S->nitems) {
                         *ctr = 0u;
                         __threadfence_system();
-                        *reinterpret_cast<volatile unsigned int*>(S->resp) = S->resp_val;
+                        if (S->resp_val == kRespIncrement) atomicAdd(reinterpret_cast<unsigned int*>(S->resp), 1u);
+                        else *reinterpret_cast<volatile unsigned int*>(S->resp) = S->resp_val;
                     }
                 }
             }

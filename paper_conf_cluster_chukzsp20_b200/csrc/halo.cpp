@@ -30,6 +30,7 @@
 #include <tuple>
 #include <vector>
 
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include "ddt_internal.h"
@@ -131,6 +132,19 @@ struct ddt_halo_s {
     void* recv_stage = nullptr;
     std::vector<Xfer> xfers;
     bool self_nccl = false;       // test hook DDT_SELF_VIA_NCCL: self messages through staging + NCCL
+    // NCCL_EARLY: per remote peer, its stream, its messages' completion counters
+    // (indices into early_ctr) and the event joining it back into the queue stream
+    struct EarlyPeer {
+        size_t xfer;
+        std::vector<int> ctr;
+        cudaStream_t s = nullptr;
+        cudaEvent_t done = nullptr;
+    };
+    bool early = false;
+    std::vector<EarlyPeer> epeers;
+    uint32_t* early_ctr = nullptr;   // device: per remote pack request, completions since the last reset
+    uint32_t* early_done = nullptr;  // device: per remote pack request, finished items (kernel bookkeeping)
+    cudaEvent_t early_start = nullptr;
     Launchable pack_l, unpack_l;  // NCCL mode: pack (+ direct self copies), unpack
     // P2P mode
     Launchable x_l;               // P2P mode: the single fused exchange kernel
@@ -213,6 +227,8 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
         if (spread) ub = sub;
     }
     if (!spread && (many || (ga && ga[0] == '1'))) group_equal_requests(b, ub);
+    for (ReqDesc& d : b.descs)  // response slots: the finishing CTA compares its count with the item count
+        if (d.resp) d.nitems = desc_items(d, ub);
     make_launchable(b, !spread, l, sm_count, ub);
     bool paired = false;
     for (const ReqDesc& d : b.descs) paired |= d.pair != 0;
@@ -394,6 +410,13 @@ Directory parse_dir(const std::vector<int64_t>& v) {
 
 void free_halo(ddt_halo_s* h) {
     if (h->gexec) cudaGraphExecDestroy(h->gexec);
+    for (auto& p : h->epeers) {
+        if (p.s) cudaStreamDestroy(p.s);
+        if (p.done) cudaEventDestroy(p.done);
+    }
+    if (h->early_start) cudaEventDestroy(h->early_start);
+    cudaFree(h->early_ctr);
+    cudaFree(h->early_done);
     cudaFree(h->send_stage);
     cudaFree(h->recv_stage);
     cudaFree(h->pack_l.dev);
@@ -405,6 +428,69 @@ void free_halo(ddt_halo_s* h) {
     for (auto& s : h->sends) type_release(s.type);
     for (auto& r : h->recvs) type_release(r.type);
     delete h;
+}
+
+// Stream memory operations (driver API, bound through the runtime's entry
+// point query: no link-time libcuda dependency).
+typedef CUresult (*WaitValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+typedef CUresult (*WriteValue32Fn)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+struct MemOps {
+    WaitValue32Fn wait = nullptr;
+    WriteValue32Fn write = nullptr;
+};
+const MemOps* memops() {
+    static MemOps m;
+    static bool init = false;
+    if (!init) {
+        init = true;
+        cudaDriverEntryPointQueryResult q1, q2;
+        if (cudaGetDriverEntryPoint("cuStreamWaitValue32", (void**)&m.wait, cudaEnableDefault, &q1) != cudaSuccess ||
+            q1 != cudaDriverEntryPointSuccess)
+            m.wait = nullptr;
+        if (cudaGetDriverEntryPoint("cuStreamWriteValue32", (void**)&m.write, cudaEnableDefault, &q2) != cudaSuccess ||
+            q2 != cudaDriverEntryPointSuccess)
+            m.write = nullptr;
+    }
+    return (m.wait && m.write) ? &m : nullptr;
+}
+
+// NCCL_EARLY transfer: every remote peer's send/recv group on its own stream,
+// started once that peer's pack requests have completed.  Groups
+// are issued in increasing peer order on every rank (a consistent order of
+// rank pairs: no deadlock even when NCCL serialises a communicator's kernels).
+ddt_status_t record_early_transfer(ddt_halo_s* h) {
+    const NcclApi* n = nccl();
+    const MemOps* mo = memops();
+    if (!n || !mo) return DDT_ERR_UNSUPPORTED;
+    for (auto& P : h->epeers) {
+        cudaError_t e = cudaStreamWaitEvent(P.s, h->early_start, 0);  // after the work preceding this exchange
+        if (e != cudaSuccess) return cuda_fail("early send: stream wait", e);
+        for (int k : P.ctr) {  // this peer's messages are packed (counter set by the finishing CTA)
+            CUresult r = mo->wait((CUstream)P.s, (CUdeviceptr)(uintptr_t)(h->early_ctr + k), 1u,
+                                  CU_STREAM_WAIT_VALUE_GEQ);
+            if (r != CUDA_SUCCESS) return cuda_fail("early send: cuStreamWaitValue32", cudaErrorUnknown);
+        }
+        for (int k : P.ctr) {  // re-arm for the next exchange (ordered before its pack by the join below)
+            CUresult r = mo->write((CUstream)P.s, (CUdeviceptr)(uintptr_t)(h->early_ctr + k), 0u, 0);
+            if (r != CUDA_SUCCESS) return cuda_fail("early send: cuStreamWriteValue32", cudaErrorUnknown);
+        }
+        const Xfer& x = h->xfers[P.xfer];
+        int r = n->GroupStart();
+        if (r == 0 && x.send_bytes)
+            r = n->Send((char*)h->send_stage + x.send_off, (size_t)x.send_bytes, kNcclUint8, x.peer, h->comm, P.s);
+        if (r == 0 && x.recv_bytes)
+            r = n->Recv((char*)h->recv_stage + x.recv_off, (size_t)x.recv_bytes, kNcclUint8, x.peer, h->comm, P.s);
+        int r2 = n->GroupEnd();
+        if (r == 0) r = r2;
+        if (r != 0) return nccl_fail("halo send/recv (early)", r);
+        e = cudaEventRecord(P.done, P.s);
+        if (e != cudaSuccess) return cuda_fail("early send: event", e);
+    }
+    for (auto& P : h->epeers) {
+        cudaError_t e = cudaStreamWaitEvent(h->stream, P.done, 0);
+        if (e != cudaSuccess) return cuda_fail("early send: join", e);
+    }
+    return DDT_OK;
 }
 
 ddt_status_t record_exchange(ddt_halo_s* h) {
@@ -424,13 +510,20 @@ ddt_status_t record_exchange(ddt_halo_s* h) {
         if (e) return cuda_fail("exchange kernel launch", e);
         return DDT_OK;
     }
+    if (h->early) {
+        cudaError_t e = cudaEventRecord(h->early_start, h->stream);
+        if (e != cudaSuccess) return cuda_fail("early send: event", e);
+    }
     if (h->pack_l.total_items) {
         int e = launch_fused(h->pack_l, h->stream, 0);
         if (e) return cuda_fail("pack launch", e);
     }
     bool remote = false;
     for (auto& x : h->xfers) remote |= x.peer != h->rank || h->self_nccl;
-    if (remote) {
+    if (remote && h->early) {
+        ddt_status_t st = record_early_transfer(h);
+        if (st != DDT_OK) return st;
+    } else if (remote) {
         const NcclApi* n = nccl();
         if (!n) return DDT_ERR_UNSUPPORTED;
         int r = n->GroupStart();
@@ -469,7 +562,10 @@ ddt_status_t ddt_halo_window_bytes(int32_t nrecv, const ddt_recv_t* recvs, int64
 ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, const ddt_send_t* sends, int32_t nrecv,
                              const ddt_recv_t* recvs, int32_t mode, ddt_halo_t* out) {
     if (!q || !c || !out || nsend < 0 || nrecv < 0 || (nsend && !sends) || (nrecv && !recvs)) return DDT_ERR_ARG;
-    if (mode != DDT_XCHG_NCCL && mode != DDT_XCHG_P2P && mode != DDT_XCHG_P2P_DIRECT) return DDT_ERR_ARG;
+    if (mode != DDT_XCHG_NCCL && mode != DDT_XCHG_P2P && mode != DDT_XCHG_P2P_DIRECT && mode != DDT_XCHG_NCCL_EARLY)
+        return DDT_ERR_ARG;
+    const bool early = mode == DDT_XCHG_NCCL_EARLY;
+    if (early) mode = DDT_XCHG_NCCL;  // the NCCL-mode plan, with per-peer early send
     const bool p2p = mode != DDT_XCHG_NCCL;
     const bool direct = mode == DDT_XCHG_P2P_DIRECT;
     if (c->nranks < 1 || c->rank < 0 || c->rank >= c->nranks) return DDT_ERR_ARG;
@@ -485,6 +581,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     h->rank = c->rank;
     h->nranks = c->nranks;
     h->mode = mode;
+    h->early = early;
     h->comm = c->nccl_comm;
     h->ag = c->host_allgather;
     h->ag_ctx = c->host_ctx;
@@ -786,7 +883,19 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         }
         for (auto& kv : xf) h->xfers.push_back(kv.second);
         HostBatch packb, unpackb;
-        for (int i = 0; i < nsend && st == DDT_OK; i++) {
+        // remote packs first, peer by peer (early send: the first peers' data is
+        // ready first), then the self messages
+        std::vector<int> sorder((size_t)nsend);
+        for (int i = 0; i < nsend; i++) sorder[(size_t)i] = i;
+        std::stable_sort(sorder.begin(), sorder.end(), [&](int a, int b) {
+            const bool ra = remote_n(sends[a].peer), rb = remote_n(sends[b].peer);
+            if (ra != rb) return ra;
+            return ra && sends[a].peer < sends[b].peer;
+        });
+        std::map<int, std::vector<int>> peer_ctr;  // early send: remote peer -> its counters
+        int nctr = 0;
+        for (int i : sorder) {
+            if (st != DDT_OK) break;
             const auto& s = sends[i];
             if (s.count * s.type->size == 0) continue;
             if (!remote_n(s.peer)) {
@@ -795,6 +904,47 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             }
             char* dst = (char*)h->send_stage + region[s.peer] + (match[(size_t)i]->data_off - span[s.peer].first);
             st = add_req(packb, s.type, OP_PACK, s.buf, dst, s.count, nullptr);
+            if (st == DDT_OK && early) peer_ctr[s.peer].push_back(nctr++);
+        }
+        if (st == DDT_OK && early) {
+            // completion counters (device): the CTA finishing a remote pack
+            // request's last item increments its counter (fused_kernel.cu)
+            if (!memops()) {
+                set_error("NCCL_EARLY needs stream memory operations (cuStreamWaitValue32)");
+                st = DDT_ERR_UNSUPPORTED;
+            }
+            const size_t nb = sizeof(uint32_t) * (size_t)std::max(nctr, 1);
+            cudaError_t e = st == DDT_OK ? cudaMalloc((void**)&h->early_ctr, nb) : cudaSuccess;
+            if (e == cudaSuccess && st == DDT_OK) e = cudaMalloc((void**)&h->early_done, nb);
+            if (e == cudaSuccess && st == DDT_OK) e = cudaMemset(h->early_ctr, 0, nb);
+            if (e == cudaSuccess && st == DDT_OK) e = cudaMemset(h->early_done, 0, nb);
+            if (e == cudaSuccess && st == DDT_OK) e = cudaEventCreateWithFlags(&h->early_start, cudaEventDisableTiming);
+            if (e != cudaSuccess) st = cuda_fail("early send setup", e);
+            int k = 0;
+            for (size_t r = 0; r < packb.descs.size() && st == DDT_OK; r++) {
+                ReqDesc& d = packb.descs[r];
+                if (d.op != OP_PACK) continue;  // remote packs come first, in counter order
+                d.resp = (uint64_t)(uintptr_t)(h->early_ctr + k);
+                d.resp_val = kRespIncrement;
+                d.done_ctr = (uint64_t)(uintptr_t)(h->early_done + k);
+                k++;
+            }
+            for (size_t xi = 0; xi < h->xfers.size() && st == DDT_OK; xi++) {
+                const Xfer& x = h->xfers[xi];
+                if (!remote_n(x.peer)) continue;
+                ddt_halo_s::EarlyPeer P;
+                P.xfer = xi;
+                auto it = peer_ctr.find(x.peer);
+                if (it != peer_ctr.end()) P.ctr = it->second;
+                e = cudaStreamCreateWithFlags(&P.s, cudaStreamNonBlocking);
+                if (e == cudaSuccess) e = cudaEventCreateWithFlags(&P.done, cudaEventDisableTiming);
+                h->epeers.push_back(P);
+                if (e != cudaSuccess) st = cuda_fail("early send streams", e);
+            }
+            std::sort(h->epeers.begin(), h->epeers.end(), [&](const ddt_halo_s::EarlyPeer& a,
+                                                              const ddt_halo_s::EarlyPeer& b) {
+                return h->xfers[a.xfer].peer < h->xfers[b.xfer].peer;
+            });
         }
         for (int i = 0; i < nrecv && st == DDT_OK; i++) {
             const auto& r = recvs[i];

@@ -8,7 +8,7 @@ from __future__ import annotations
 import ctypes
 
 from ._abi import (lib, check, P, ddt_send_t, ddt_recv_t, ddt_comm_t, ALLGATHER_FN, DDT_XCHG_NCCL,
-                   DDT_XCHG_P2P, DDT_XCHG_P2P_DIRECT)
+                   DDT_XCHG_P2P, DDT_XCHG_P2P_DIRECT, DDT_XCHG_NCCL_EARLY)
 from .queue import ptr_of
 
 
@@ -155,17 +155,20 @@ class Halo:
     """A persistent exchange plan.  sends / recvs: lists of
     (peer, tag, Type, buffer, count); a send to (peer, tag) matches the peer's
     receive from (this rank, tag).  mode: "nccl" (fused pack -> NCCL send/recv
-    -> fused unpack), "p2p" (one kernel through peers' windows) or
-    "p2p_direct" (one pack-free kernel writing peers' receive buffers)."""
+    -> fused unpack), "nccl_early" (the same, each peer's send/recv started as
+    soon as that peer's messages are packed), "p2p" (one kernel through peers'
+    windows) or "p2p_direct" (one pack-free kernel writing peers' receive
+    buffers)."""
 
     def __init__(self, queue, comm: Comm, sends, recvs, mode: str = "nccl", graph: bool = True):
         self.queue, self.comm = queue, comm
         self._keep = [m[2] for m in sends] + [m[2] for m in recvs]
         s_arr = _msgs(sends, ddt_send_t)
         r_arr = _msgs(recvs, ddt_recv_t)
-        self.mode = {"nccl": DDT_XCHG_NCCL, "p2p": DDT_XCHG_P2P, "p2p_direct": DDT_XCHG_P2P_DIRECT}[mode]
+        self.mode = {"nccl": DDT_XCHG_NCCL, "p2p": DDT_XCHG_P2P, "p2p_direct": DDT_XCHG_P2P_DIRECT,
+                     "nccl_early": DDT_XCHG_NCCL_EARLY}[mode]
         self.windows = None
-        if self.mode != DDT_XCHG_NCCL:
+        if self.mode in (DDT_XCHG_P2P, DDT_XCHG_P2P_DIRECT):
             nb = ctypes.c_int64()
             check(lib().ddt_halo_window_bytes(len(recvs), r_arr, ctypes.byref(nb)), "ddt_halo_window_bytes")
             self.windows = Windows(comm, nb.value)

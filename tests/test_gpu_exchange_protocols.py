@@ -210,16 +210,21 @@ def test_window_protocol_large_faces_graph(ddt, monkeypatch):
 
 @pytest.mark.parametrize("local,dirs,nvars", [((128, 128, 128), FACE_DIRS, 1), ((10, 12, 14), ALL_DIRS, 2)])
 @pytest.mark.parametrize("graph", [False, True])
-def test_nccl_mode_staging_and_sendrecv(ddt, monkeypatch, local, dirs, nvars, graph):
+@pytest.mark.parametrize("mode", ["nccl", "nccl_early"])
+def test_nccl_mode_staging_and_sendrecv(ddt, monkeypatch, local, dirs, nvars, graph, mode):
     """NCCL mode with every message through the remote path: fused pack into
     per-peer staging, grouped ncclSend/ncclRecv (here: to self, over a 1-rank
-    NCCL communicator), fused unpack from the receive staging."""
+    NCCL communicator), fused unpack from the receive staging.  nccl_early:
+    the peer's send/recv group runs on its own stream once the pack kernel's
+    per-message completion counters (device memory, stream-waited) show its
+    messages packed; the counters are re-armed each exchange (4 iterations,
+    direct and graph-replayed)."""
     import torch
     _env(monkeypatch, DDT_SELF_VIA_NCCL="1")
     comm = ddt.Comm.single(torch.cuda.current_device(), nccl=True)
-    p = Plan(ddt, local, dirs, nvars, "nccl", graph=graph, comm=comm)
+    p = Plan(ddt, local, dirs, nvars, mode, graph=graph, comm=comm)
     assert p.h.launches_per_exchange == 2  # pack batch + unpack batch (NCCL between them)
-    _run(p, 3, f"nccl self {local}")
+    _run(p, 4, f"{mode} self {local}")
     p.close()
 
 
