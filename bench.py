@@ -404,7 +404,7 @@ def pack_roofline(ddt, torch, hbm_peak, reps=20):
             q.pack(t, src[b], 1, dst[b])
         plan = ddt.Plan(q)
         stream = torch.cuda.current_stream()
-        for _ in range(3):
+        for _ in range(5):
             plan.launch()
         torch.cuda.synchronize()
         times = []
@@ -709,6 +709,14 @@ def main():
     # a mode whose capture fails falls back to host-issued steps (reported)
     R = int(os.environ.get("DDT_BENCH_REPLICAS", "96"))
 
+    # bring the GPU to its steady clocks before the first timed mode (the first
+    # mode measured otherwise pays the ramp: nccl 2.76 vs p2p 2.35 us/iter at
+    # N = 1 with the identical DirectIPC kernel)
+    t_w = time.time()
+    while time.time() - t_w < 0.5:
+        for _ in range(20):
+            l2_evict(torch, flush_buf)
+        torch.cuda.synchronize()
     results = {}
     # N = 1: every message is a self message (one DirectIPC launch in every mode);
     # N > 1: the three data paths differ -- measure all, report the fastest
@@ -753,6 +761,17 @@ def main():
     best = ok[best_mode]
     wl = best["wl"]
     K = args.steps
+    # free the other modes' replicas (GBs of arrays) before the e2e and extra measurements
+    for m in list(ok):
+        if m != best_mode:
+            if dist_on:
+                import torch.distributed as dist
+                torch.cuda.synchronize()
+                dist.barrier()  # no peer may still be writing into a window we are about to free
+            ok[m]["wl"].close()
+            ok[m]["comm"].close()
+            del ok[m]
+    torch.cuda.empty_cache()
     staged_ms, st_h2d, st_d2h = e2e_steps(torch, wl, max(10, K // 10), dist_on)
     staged_ms = max_over_ranks(torch, staged_ms, dist_on)
     # zero-copy e2e: NCCL or P2P-window plan (P2P_DIRECT opens the receive
@@ -783,9 +802,13 @@ def main():
     if rank == 0 and not dist_on:
         try:
             fl = latency_floor(ddt, torch, K, flush_buf)
+            fl500 = latency_floor(ddt, torch, 500, flush_buf) if K != 500 else fl
             roof["latency_floor"] = {"us": round(fl, 3), "value_over_floor": round(best["mean_ms"] * 1e3 / fl, 2),
+                                     "us_at_K500": round(fl500, 3),
                                      "what": "same K-step graph harness, one fused launch moving 512 B (configs[0] "
-                                             "vector pack) from cold buffers: launch + one dependent DRAM round trip"}
+                                             "vector pack) from cold buffers: launch + one dependent DRAM round trip; "
+                                             "us_at_K500: the same with K = 500 (the fixed cost of a graph's first, "
+                                             "cold-code launch weighs 25x less)"}
         except Exception as e:
             roof["latency_floor"] = {"error": f"{type(e).__name__}: {e}"}
 
