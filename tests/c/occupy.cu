@@ -8,9 +8,10 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
-__global__ void occupy_kernel(volatile int* stop, unsigned int* started, unsigned long long max_ns) {
+__global__ void occupy_kernel(volatile int* stop, volatile unsigned int* started, unsigned long long max_ns) {
     if (threadIdx.x == 0) {
-        atomicAdd_system(started, 1u);
+        started[blockIdx.x] = 1u;  // host-mapped, one slot per CTA (no system-scope atomics on host memory)
+        __threadfence_system();
         unsigned long long t0, t;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
         for (;;) {
@@ -24,7 +25,7 @@ __global__ void occupy_kernel(volatile int* stop, unsigned int* started, unsigne
 }
 
 extern "C" int occupy_launch(void* stream, int ctas, int threads, void* stop, void* started, long long max_ns) {
-    occupy_kernel<<<ctas, threads, 0, (cudaStream_t)stream>>>((volatile int*)stop, (unsigned int*)started,
+    occupy_kernel<<<ctas, threads, 0, (cudaStream_t)stream>>>((volatile int*)stop, (volatile unsigned int*)started,
                                                               (unsigned long long)max_ns);
     return (int)cudaGetLastError();
 }

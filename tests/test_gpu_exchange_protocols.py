@@ -245,16 +245,16 @@ def test_exchange_completes_while_another_kernel_holds_the_sms(ddt, monkeypatch)
     p.fill(0)
     torch.cuda.synchronize()
     stop = torch.zeros(1, dtype=torch.int32).pin_memory()
-    started = torch.zeros(1, dtype=torch.int32).pin_memory()
     s_occ = torch.cuda.Stream()
     ctas = 2 * nsm - 1
+    started = torch.zeros(ctas, dtype=torch.int32).pin_memory()  # one slot per occupier CTA
     rc = occ.occupy_launch(ctypes.c_void_p(s_occ.cuda_stream), ctas, 1024, ctypes.c_void_p(stop.data_ptr()),
                            ctypes.c_void_p(started.data_ptr()), int(20e9))
     assert rc == 0
     t0 = time.time()
-    while int(started[0]) < ctas and time.time() - t0 < 10:
+    while int(started.sum()) < ctas and time.time() - t0 < 10:
         time.sleep(0.001)
-    assert int(started[0]) == ctas, "occupier did not become resident"
+    assert int(started.sum()) == ctas, "occupier did not become resident"
     p.h.exchange()  # on the queue's stream (the current stream at Plan creation)
     done_stream = torch.cuda.current_stream()
     t0 = time.time()
