@@ -690,8 +690,20 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         const uint64_t nch = xclaim ? ((uint64_t)tv.total + xclaim - 1) / xclaim : (uint64_t)tv.total;
         xspan = xclaim ? (uint64_t)xclaim * (nch + gridDim.x) : (uint64_t)tv.total;
         xend = xclaim ? (uint64_t)xclaim * nch : (uint64_t)tv.total;
+        // programmatic dependent launch: with one item per CTA (claim 0) the
+        // CTA claims its ticket BEFORE waiting for the preceding grid and only
+        // then lets the next grid launch -- the claim's atomic round trip hides
+        // under the predecessor's tail, and a successor (of this plan or any
+        // other kernel) can only start once every CTA of this grid has claimed,
+        // so launches of one plan never interleave their tickets (the span
+        // arithmetic holds).  Looping grids trigger and wait first.
+        if (xclaim) {
+            pdl_trigger();
+            pdl_wait();
+        }
         if (threadIdx.x == 0) s_xt[0] = atomicAdd(xtick, xclaim ? (unsigned long long)xclaim : 1ull);
         __syncthreads();
+        if (!xclaim) pdl_trigger();  // the wait follows the first item's descriptor staging (static data)
         const uint64_t t = s_xt[0];
         epoch = t / xspan + 1ull;
         const uint64_t loc = t % xspan;
@@ -751,6 +763,9 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             cur = r;
         }
         // exchange requests and the dense requests of spread plans carry their own item size
+        if constexpr (XCHG) {
+            if (!xclaim && item == first) pdl_wait();  // before any flag or data access
+        }
         const int ubr = S->xub ? (int)S->xub : (int)tv.ub;
         const uint32_t v0 = local * (uint32_t)(kThreads * ubr);
         bool run = true;
@@ -933,16 +948,14 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const
 template <int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_dev(const uint8_t* __restrict__ table, const XArgs xa) {
-    pdl_trigger();
-    pdl_wait();  // before any table read, flag or data access
+    // the table is written once at plan creation (never by a kernel): read
+    // before the PDL wait; fused_body claims, triggers and waits (see there)
     fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::XUNR>(view_of(table), &xa);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, const XArgs xa) {
-    pdl_trigger();
-    pdl_wait();
     fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::XUNR>(view_of(pb), &xa);
 }
 
