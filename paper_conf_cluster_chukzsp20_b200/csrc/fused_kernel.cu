@@ -39,7 +39,7 @@
 #define DDT_MINB 5
 #endif
 #ifndef DDT_XMINB
-#define DDT_XMINB 4
+#define DDT_XMINB 6
 #endif
 #ifndef DDT_V8_MINB
 #define DDT_V8_MINB 6
@@ -923,9 +923,10 @@ template <int V> struct VarT {
     static constexpr bool PAIR = V == 9 || V == 7 || V == 4;
     // exchange kernels: every request moves at most kXchgUb vectors per thread
     // per item (sender and receiver chunk alike), so two load slots suffice;
-    // >= 4 resident CTAs per SM (<= 64 registers) keep one-CTA-per-item
-    // exchange launches in as few waves as possible (96 registers / 2 CTAs
-    // per SM before: configs[1] through the window protocol 7.2 -> see DESIGN)
+    // 6 resident CTAs per SM (<= 40 registers) put a one-wave exchange of one
+    // item per CTA in a single wave (96 registers / 2 CTAs per SM before;
+    // window proxy from 4 to 6 CTAs/SM: configs[1] 4.96 -> 4.47 us, COMB
+    // 197 -> 177 us)
     static constexpr int XUNR = UNR < kXchgUb ? UNR : kXchgUb;
     static constexpr int XMINB = (V == 8 || V == 10) ? DDT_V8_MINB : DDT_XMINB;
 };

@@ -25,6 +25,12 @@ __global__ void occupy_kernel(volatile int* stop, volatile unsigned int* started
 }
 
 extern "C" int occupy_launch(void* stream, int ctas, int threads, void* stop, void* started, long long max_ns) {
+    // leave the SMs' shared-memory carveout at its maximum: a kernel whose
+    // carveout differs from the one an SM runs with cannot be placed on that SM
+    // until it drains, whatever its other resources (the exchange kernel needs
+    // a little shared memory per CTA)
+    cudaFuncSetAttribute(occupy_kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
+                         (int)cudaSharedmemCarveoutMaxShared);
     occupy_kernel<<<ctas, threads, 0, (cudaStream_t)stream>>>((volatile int*)stop, (volatile unsigned int*)started,
                                                               (unsigned long long)max_ns);
     return (int)cudaGetLastError();

@@ -234,7 +234,11 @@ def test_exchange_completes_while_another_kernel_holds_the_sms(ddt, monkeypatch)
     The window-protocol exchange (more items than its resident grid would
     hold, pack items before the unpack items that wait for them) must finish
     while that kernel is still running: items are claimed by ticket in item
-    order, so a waiting CTA never holds back an unclaimed signalling item."""
+    order, so a waiting CTA never holds back an unclaimed signalling item.
+    (The occupier runs with the maximum shared-memory carveout: an SM only
+    takes CTAs of a kernel whose carveout it can serve, so an occupier at the
+    minimum carveout would keep the exchange off its last SM regardless of
+    the item order -- measured: no item ran until the occupier ended.)"""
     import torch
     from gpu_util import occupier
     _env(monkeypatch, DDT_SELF_VIA_WINDOW="1", DDT_NO_LL="1")
@@ -242,7 +246,12 @@ def test_exchange_completes_while_another_kernel_holds_the_sms(ddt, monkeypatch)
     nsm = torch.cuda.get_device_properties(0).multi_processor_count
     p = Plan(ddt, (64, 128, 128), ALL_DIRS, 2, "p2p")
     p.h.set_timeout(5.0)
+    # one exchange first: CUDA loads kernels lazily at their first launch, and a
+    # module load issued while another kernel holds the GPU can stall behind it
     p.fill(0)
+    p.h.exchange()
+    p.check("before occupancy")
+    p.fill(1)
     torch.cuda.synchronize()
     stop = torch.zeros(1, dtype=torch.int32).pin_memory()
     s_occ = torch.cuda.Stream()
@@ -270,8 +279,8 @@ def test_exchange_completes_while_another_kernel_holds_the_sms(ddt, monkeypatch)
     assert finished, "exchange did not complete while the SMs were held"
     assert still_occupied, "the occupier finished first: the test did not constrain the exchange"
     p.check("exchange under occupancy")
-    p.h.exchange()  # the plan stays usable (epoch, tickets reset)
-    p.fill(1)
+    p.h.exchange()  # the plan stays usable (epoch from the tickets)
+    p.fill(2)
     p.h.exchange()
     p.check("after occupancy")
     p.close()
