@@ -41,6 +41,9 @@
 #ifndef DDT_XMINB
 #define DDT_XMINB 6
 #endif
+#ifndef DDT_LL_SLEEP
+#define DDT_LL_SLEEP 16
+#endif
 #ifndef DDT_V8_MINB
 #define DDT_V8_MINB 6
 #endif
@@ -194,7 +197,7 @@ __device__ __forceinline__ uint4 ll_load(const uint8_t* p, uint32_t epoch, const
                 break;
             }
         }
-        __nanosleep(64);
+        __nanosleep(DDT_LL_SLEEP);
     }
     return make_uint4(r.x, r.z, 0u, 0u);
 }
@@ -762,10 +765,10 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             }
             cur = r;
         }
-        // exchange requests and the dense requests of spread plans carry their own item size
         if constexpr (XCHG) {
             if (!xclaim && item == first) pdl_wait();  // before any flag or data access
         }
+        // exchange requests and the dense requests of spread plans carry their own item size
         const int ubr = S->xub ? (int)S->xub : (int)tv.ub;
         const uint32_t v0 = local * (uint32_t)(kThreads * ubr);
         bool run = true;
