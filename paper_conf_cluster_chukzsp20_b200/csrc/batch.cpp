@@ -24,7 +24,11 @@ static uint32_t fill_prefix(uint32_t* prefix, const HostBatch& b, int ub) {
     for (size_t i = 0; i < d.size();) {
         const size_t m = b.gm.empty() ? 1 : std::max<uint32_t>(1, b.gm[i]);
         for (size_t j = 0; j < m; j++) prefix[i + j] = (uint32_t)acc;
-        acc += (uint64_t)m * desc_items(d[i], ub);
+        // the second member of an exchange pair runs inside its partner's items
+        // (zero items: the kernel's "largest r with prefix[r] <= item" search
+        // never lands on it)
+        const bool partner = b.order.empty() && i > 0 && d[i - 1].pair;
+        acc += partner ? 0u : (uint64_t)m * desc_items(d[i], ub);
         i += m;
     }
     prefix[d.size()] = (uint32_t)acc;
@@ -200,6 +204,61 @@ static void pair_requests(HostBatch& b) {
         }
     }
     b = std::move(out);
+}
+
+// Exchange pairs (fused_kernel.cu run_pair_x): two requests of an exchange
+// batch, both non-waiting or both waiting, neither a remote direct nor a
+// signal-only item, with equal vector counts and item sizes, whose typed sides
+// walk the same short-segment lattice and whose packed sides are both windows
+// of one kind (K_CONTIG or K_LL).  Partners become adjacent (relative order of
+// the waiting / non-waiting partition kept).  DDT_NO_XPAIR=1: off.
+bool pair_exchange_requests(HostBatch& b) {
+    const char* off = DDT_KNOB("DDT_NO_XPAIR");
+    if ((off && off[0] == '1') || !b.gm.empty() || b.xinfo.size() != b.descs.size()) return false;
+    const size_t n = b.descs.size();
+    auto waits = [&](size_t i) { return b.xinfo[i].wait != 0 || b.descs[i].kind == K_LL; };
+    auto typed = [&](size_t i) -> const ReqDesc& {
+        return b.descs[i].op == OP_PACK ? b.descs[i] : b.aux[b.descs[i].aux];
+    };
+    auto packed = [&](size_t i) -> const ReqDesc& {
+        return b.descs[i].op == OP_PACK ? b.aux[b.descs[i].aux] : b.descs[i];
+    };
+    std::vector<int> partner(n, -1);
+    bool any = false;
+    for (size_t i = 0; i < n; i++) {
+        const ReqDesc& A = b.descs[i];
+        if (partner[i] >= 0 || A.resp || A.nvec == 0 || (A.op != OP_PACK && A.op != OP_UNPACK)) continue;
+        if (b.xinfo[i].wait && b.xinfo[i].signal) continue;  // remote directs
+        if (!typed(i).l2_64) continue;                        // short segments only (x faces)
+        for (size_t j = i + 1; j < n; j++) {
+            const ReqDesc& B = b.descs[j];
+            if (partner[j] >= 0 || B.resp || B.nvec != A.nvec || B.op != A.op || B.xub != A.xub) continue;
+            if (waits(i) != waits(j) || (b.xinfo[j].wait && b.xinfo[j].signal)) continue;
+            const ReqDesc &pa = packed(i), &pb = packed(j);
+            if (pa.kind != pb.kind || (pa.kind != K_CONTIG && pa.kind != K_LL) || pa.lw != pb.lw) continue;
+            if (!same_lattice(typed(i), typed(j))) continue;
+            partner[i] = (int)j;
+            partner[j] = (int)i;
+            any = true;
+            break;
+        }
+    }
+    if (!any) return false;
+    HostBatch out;
+    out.ticket = b.ticket;
+    for (size_t i = 0; i < n; i++) {
+        if (partner[i] >= 0 && (size_t)partner[i] < i) continue;  // placed with its partner
+        ReqDesc d = b.descs[i];
+        d.pair = partner[i] >= 0 ? 1 : 0;
+        out.add(d, b.aux[b.descs[i].aux]);
+        out.xinfo.push_back(b.xinfo[i]);
+        if (partner[i] >= 0) {
+            out.add(b.descs[(size_t)partner[i]], b.aux[b.descs[(size_t)partner[i]].aux]);
+            out.xinfo.push_back(b.xinfo[(size_t)partner[i]]);
+        }
+    }
+    b = std::move(out);
+    return true;
 }
 
 bool spread_items(HostBatch& b, int ub, bool allow_pair) {
@@ -449,6 +508,11 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
     bool multi = false;  // a request with its own item size > 1 needs the multi-slot kernel
     for (const ReqDesc& d : b.descs) multi |= d.xub > 1;
     if (out.variant == 7 && out.ub == 1 && !multi && !(v9 && v9[0] == '1')) out.variant = 9;
+    if (is_exchange_batch(b) && (out.variant == 3 || out.variant == 4)) {  // exchange pairs: their own instance
+        bool paired = false;
+        for (const ReqDesc& d : b.descs) paired |= d.pair != 0;
+        if (paired) out.variant += 8;
+    }
     out.grid_mode = grid_mode_for(b, out.ub, sm_count);
     out.ticket = out.grid_mode == 1 ? b.ticket : 0;
     out.claim = 0;

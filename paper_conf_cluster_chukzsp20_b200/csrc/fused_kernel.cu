@@ -202,6 +202,31 @@ __device__ __forceinline__ uint4 ll_load(const uint8_t* p, uint32_t epoch, const
     return make_uint4(r.x, r.z, 0u, 0u);
 }
 
+// Two LL words polled in one loop (exchange pairs).
+__device__ __forceinline__ void ll_load2(const uint8_t* p, const uint8_t* q, uint32_t epoch, const XArgs* xa,
+                                         uint4& a, uint4& b) {
+    uint4 r, t;
+    uint64_t t0 = 0;
+    for (uint32_t n = 0;; n++) {
+        asm volatile("ld.volatile.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+                     : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p) : "memory");
+        asm volatile("ld.volatile.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+                     : "=r"(t.x), "=r"(t.y), "=r"(t.z), "=r"(t.w) : "l"(q) : "memory");
+        if (r.y == epoch && r.w == epoch && t.y == epoch && t.w == epoch) break;
+        if ((n & 63) == 0) {
+            const uint64_t tn = globaltimer_ns();
+            if (n == 0) t0 = tn;
+            else if (tn - t0 > xa->timeout_ns) {
+                *reinterpret_cast<volatile int*>(xa->err_flag) = 1;
+                break;
+            }
+        }
+        __nanosleep(DDT_LL_SLEEP);
+    }
+    a = make_uint4(r.x, r.z, 0u, 0u);
+    b = make_uint4(t.x, t.z, 0u, 0u);
+}
+
 __device__ __forceinline__ void ll_store(uint8_t* p, const uint4& d, uint32_t epoch) {
     asm volatile("st.volatile.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(d.x), "r"(epoch), "r"(d.y),
                  "r"(epoch) : "memory");
@@ -526,6 +551,46 @@ __device__ __forceinline__ void run_pair(const ReqDesc& SA, const ReqDesc& DA, c
     if (pdlw) pdl_wait();
 }
 
+// Exchange pairs: like run_pair, for two requests of an exchange batch whose
+// typed sides walk the same lattice and whose other sides are both packed
+// (window / LL window): the +x and -x packs read both ends of each row in one
+// thread, the +x and -x unpacks write both ghost ends of each row.  One slot
+// at a time; window sources are loaded coherently (another GPU writes them),
+// LL sides validate / carry the epoch per word.
+template <int LW, bool SONLY>
+__device__ __forceinline__ void run_pair_x(const ReqDesc& SA, const ReqDesc& DA, const ReqDesc& SB,
+                                           const ReqDesc& DB, uint32_t v0, int ub, const XArgs* xa,
+                                           uint32_t epoch) {
+    const int lw = LW >= 0 ? LW : SA.lw;
+    const uint32_t nvec = SA.nvec;
+    const bool coh = SA.op == OP_UNPACK;
+    for (int u = 0; u < ub; u++) {
+        const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+        if (v >= nvec) break;
+        const uint8_t* pa = reinterpret_cast<const uint8_t*>(SA.ptr) + vec_offset<LW, SONLY>(SA, v);
+        const uint8_t* pb = reinterpret_cast<const uint8_t*>(SB.ptr) + vec_offset<LW, SONLY>(SB, v);
+        uint4 a, b;
+        if (SA.kind == K_LL) {
+            ll_load2(pa, pb, epoch, xa, a, b);  // one polling loop for both words
+        } else if (coh) {
+            a = ld_vec<false, LW>(pa, lw);
+            b = ld_vec<false, LW>(pb, lw);
+        } else {
+            a = ld_vec<true, LW>(pa, lw, SA.l2_64 != 0);
+            b = ld_vec<true, LW>(pb, lw, SB.l2_64 != 0);
+        }
+        uint8_t* qa = reinterpret_cast<uint8_t*>(DA.ptr) + vec_offset<LW, SONLY>(DA, v);
+        uint8_t* qb = reinterpret_cast<uint8_t*>(DB.ptr) + vec_offset<LW, SONLY>(DB, v);
+        if (DA.kind == K_LL) {
+            ll_store(qa, a, epoch);
+            ll_store(qb, b, epoch);
+        } else {
+            st_vec<LW>(qa, lw, a);
+            st_vec<LW>(qb, lw, b);
+        }
+    }
+}
+
 // Largest r with prefix[r] <= item (prefix strictly increasing, prefix[0] = 0).
 __device__ __forceinline__ uint32_t find_request(const uint32_t* prefix, uint32_t nreq, uint32_t item) {
     uint32_t lo = 0, hi = nreq;
@@ -640,8 +705,8 @@ template <bool XCHG, int LW, bool SONLY, bool GW, bool PH, bool INPLACE = false,
 __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa) {
     __shared__ ReqDesc sd;
     __shared__ ReqDesc sa;
-    __shared__ ReqDesc sd2, sa2;  // the partner of a paired request (plain device-table batches)
-    __shared__ XInfo sx;
+    __shared__ ReqDesc sd2, sa2;  // the partner of a paired request
+    __shared__ XInfo sx, sx2;
     __shared__ int s_ok;
     uint64_t epoch = 0;
     XCtrl* ctrl = nullptr;
@@ -752,13 +817,26 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
                     copy_words(&sa2, tv.aux + r + 1, kWords, 192);
                 }
             }
+            if constexpr (XCHG && PAIR) {
+                if (tv.descs[r].pair) {  // exchange pair: the partner's descriptors and exchange info
+                    copy_words(&sd2, tv.descs + r + 1, kWords, 128);
+                    copy_words(&sa2, tv.aux + r + 1, kWords, 160);
+                    copy_words(&sx2, tv.xinfo + r + 1, kXWords, 192);
+                }
+            }
             __syncthreads();
             if constexpr (XCHG) {
-                if (sx.parity_stride) {  // double-buffered window: pack writes it, unpack reads it
+                const bool pr = PAIR && sd.pair;
+                if (sx.parity_stride || (pr && sx2.parity_stride)) {  // double-buffered window halves
                     if (threadIdx.x == 0) {
                         const uint64_t off = (epoch & 1ull) * (uint64_t)sx.parity_stride;
                         if (sd.op == OP_PACK) sa.ptr += off;
                         else sd.ptr += off;
+                        if (pr) {
+                            const uint64_t off2 = (epoch & 1ull) * (uint64_t)sx2.parity_stride;
+                            if (sd2.op == OP_PACK) sa2.ptr += off2;
+                            else sd2.ptr += off2;
+                        }
                     }
                     __syncthreads();
                 }
@@ -777,22 +855,26 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             if (trace && threadIdx.x == 0) tr0 = globaltimer();
         }
         if constexpr (XCHG) {
-            if (sx.wait) {  // acquire: the peer's data / ready signal has arrived
+            const bool pr = PAIR && S->pair;
+            if (sx.wait || (pr && sx2.wait)) {  // acquire: the peer's data / ready signal has arrived
                 if (threadIdx.x == 0) {
-                    const uint64_t* flag = reinterpret_cast<const uint64_t*>(sx.wait) +
-                                           (sx.per_item ? local : 0u);
                     int ok = 1;
-                    const bool g = sx.gpu_scope != 0;  // the writer runs on this GPU
-                    if ((g ? ld_acquire_gpu(flag) : ld_acquire_sys(flag)) < epoch) {
-                        const uint64_t t0 = globaltimer();
-                        while ((g ? ld_acquire_gpu(flag) : ld_acquire_sys(flag)) < epoch) {
-                            if (globaltimer() - t0 > xa->timeout_ns) {
-                                ok = 0;
-                                *reinterpret_cast<volatile int*>(xa->err_flag) = 1;
-                                __threadfence_system();
-                                break;
+                    for (int m = 0; m < (pr ? 2 : 1); m++) {
+                        const XInfo& X = m ? sx2 : sx;
+                        if (!X.wait) continue;
+                        const uint64_t* flag = reinterpret_cast<const uint64_t*>(X.wait) + (X.per_item ? local : 0u);
+                        const bool g = X.gpu_scope != 0;  // the writer runs on this GPU
+                        if ((g ? ld_acquire_gpu(flag) : ld_acquire_sys(flag)) < epoch) {
+                            const uint64_t t0 = globaltimer();
+                            while ((g ? ld_acquire_gpu(flag) : ld_acquire_sys(flag)) < epoch) {
+                                if (globaltimer() - t0 > xa->timeout_ns) {
+                                    ok = 0;
+                                    *reinterpret_cast<volatile int*>(xa->err_flag) = 1;
+                                    __threadfence_system();
+                                    break;
+                                }
+                                __nanosleep(32);
                             }
-                            __nanosleep(32);
                         }
                     }
                     s_ok = ok;
@@ -806,6 +888,8 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             run_seg<kSegUnroll>(*S, *D, v0, (int)tv.ub, !waited);
         } else if (!XCHG && PAIR && S->pair) {
             run_pair<LW, SONLY>(sd, sa, sd2, sa2, v0, ubr, !waited);
+        } else if (XCHG && PAIR && S->pair) {
+            if (run) run_pair_x<LW, SONLY>(sd, sa, sd2, sa2, v0, ubr, xa, (uint32_t)epoch);
         } else {
             if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, ubr, xa,
                                                               (uint32_t)epoch, !waited);
@@ -831,22 +915,27 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
                 __syncthreads();
                 if (threadIdx.x == 0) tr2 = globaltimer();
             }
-            if (sx.signal) {  // release: this chunk (per_item) or the whole message has moved
+            const bool pr = PAIR && S->pair;
+            if (sx.signal || (pr && sx2.signal)) {  // release: this chunk (per_item) or the whole message has moved
                 __syncthreads();  // the CTA's (peer) stores precede thread 0's release (cumulativity)
                 if (threadIdx.x == 0) {
-                    uint64_t* flag = reinterpret_cast<uint64_t*>(sx.signal);
-                    if (sx.per_item) {
-                        if (sx.gpu_scope) st_release_gpu(flag + local, epoch);
-                        else st_release_sys(flag + local, epoch);
-                    } else if (sx.nitems <= 1) {
-                        __threadfence_system();
-                        for (uint32_t k = 0; k < sx.fanout; k++) st_relaxed_sys(flag + k, epoch);
-                    } else {
-                        __threadfence_system();
-                        unsigned long long old = atomicAdd_system(&ctrl->counters[sx.counter], 1ull);
-                        if (old + 1ull == epoch * (unsigned long long)sx.nitems) {
-                            __threadfence_system();  // one release for all of the message's flags
-                            for (uint32_t k = 0; k < sx.fanout; k++) st_relaxed_sys(flag + k, epoch);
+                    for (int m = 0; m < (pr ? 2 : 1); m++) {
+                        const XInfo& X = m ? sx2 : sx;
+                        if (!X.signal) continue;
+                        uint64_t* flag = reinterpret_cast<uint64_t*>(X.signal);
+                        if (X.per_item) {
+                            if (X.gpu_scope) st_release_gpu(flag + local, epoch);
+                            else st_release_sys(flag + local, epoch);
+                        } else if (X.nitems <= 1) {
+                            __threadfence_system();
+                            for (uint32_t k = 0; k < X.fanout; k++) st_relaxed_sys(flag + k, epoch);
+                        } else {
+                            __threadfence_system();
+                            unsigned long long old = atomicAdd_system(&ctrl->counters[X.counter], 1ull);
+                            if (old + 1ull == epoch * (unsigned long long)X.nitems) {
+                                __threadfence_system();  // one release for all of the message's flags
+                                for (uint32_t k = 0; k < X.fanout; k++) st_relaxed_sys(flag + k, epoch);
+                            }
                         }
                     }
                 }
@@ -908,7 +997,10 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
 // halo steps such as configs[1]): no unrolled load slots, a short hot path.
 // 10 = segment per thread (run_seg): uniform-list <-> packed batches of <= 16-B
 // segments moved as 4-B words (batch.cpp segment_batch_vps).
-template <int V> struct VarT {
+// 11 / 12 = exchange kernels of variants 3 / 4 that also run exchange pairs
+// (run_pair_x): a separate instance, so unpaired plans keep the lean one.
+template <int V0> struct VarT {
+    static constexpr int V = V0 == 11 ? 3 : (V0 == 12 ? 4 : V0);
     static constexpr bool SEG = V == 10;
     static constexpr int LW = (V == 0 || V == 6 || V == 7 || V == 9) ? -1 : ((V == 8 || V == 10) ? 2 : V - 1);
     static constexpr int UNR = V == 8 ? kUnrollNarrow : (V == 9 ? 1 : kUnroll);
@@ -924,6 +1016,7 @@ template <int V> struct VarT {
     // paired requests (device-table spread plans): the one-slot variants only
     // (batch.cpp kPairVariants), so the register budget of the others is untouched
     static constexpr bool PAIR = V == 9 || V == 7 || V == 4;
+    static constexpr bool XPAIR = V0 == 11 || V0 == 12;  // exchange pairs (ddt_internal.h xpair_variant)
     // exchange kernels: every request moves at most kXchgUb vectors per thread
     // per item (sender and receiver chunk alike), so two load slots suffice;
     // 6 resident CTAs per SM (<= 40 registers) put a one-wave exchange of one
@@ -954,13 +1047,15 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_dev(const uint8_t* __restrict__ table, const XArgs xa) {
     // the table is written once at plan creation (never by a kernel): read
     // before the PDL wait; fused_body claims, triggers and waits (see there)
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::XUNR>(view_of(table), &xa);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::XUNR, false, false,
+               VarT<V>::XPAIR>(view_of(table), &xa);
 }
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_param(const __grid_constant__ ParamBatch<CAP> pb, const XArgs xa) {
-    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::XUNR>(view_of(pb), &xa);
+    fused_body<true, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, false, VarT<V>::XUNR, false, false,
+               VarT<V>::XPAIR>(view_of(pb), &xa);
 }
 
 // ------------------------------------------------------------------ host side
@@ -1088,6 +1183,8 @@ int launch_exchange_form(int form, int variant, const void* src, uint32_t total_
     case 7: launch_exchange_v<7>(form, src, total_items, xa, s, grid_cap); break;
     case 8: launch_exchange_v<8>(form, src, total_items, xa, s, grid_cap); break;
     case 9: launch_exchange_v<9>(form, src, total_items, xa, s, grid_cap); break;
+    case 11: launch_exchange_v<11>(form, src, total_items, xa, s, grid_cap); break;
+    case 12: launch_exchange_v<12>(form, src, total_items, xa, s, grid_cap); break;
     default: launch_exchange_v<0>(form, src, total_items, xa, s, grid_cap); break;
     }
     return (int)cudaGetLastError();

@@ -226,13 +226,23 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
             for (ReqDesc& d : b.descs) d.xub = 0;
         if (spread) ub = sub;
     }
-    if (!spread && (many || (ga && ga[0] == '1'))) group_equal_requests(b, ub);
+    // multi-wave exchange plans: pair +x / -x style packs and unpacks
+    // (fused_kernel.cu run_pair_x; COMB window proxy 178 -> 144 us); one-wave
+    // (latency-bound) plans keep one request per item (configs[1] window
+    // proxy: 4.35 us unpaired, 6.35 us paired)
+    const char* xpa = DDT_KNOB("DDT_XPAIR_ALWAYS");  // tests: pair one-wave exchange plans too
+    const bool xpaired = force_ub > 0 && (many || (xpa && xpa[0] == '1')) && pair_exchange_requests(b);
+    if (!spread && !xpaired && (many || (ga && ga[0] == '1'))) group_equal_requests(b, ub);
     for (ReqDesc& d : b.descs)  // response slots: the finishing CTA compares its count with the item count
         if (d.resp) d.nitems = desc_items(d, ub);
     make_launchable(b, !spread, l, sm_count, ub);
     bool paired = false;
     for (const ReqDesc& d : b.descs) paired |= d.pair != 0;
-    if (paired && !pair_variant(l.variant)) {  // the chosen instance cannot run pairs: undo them
+    if (paired && xpaired && !xpair_variant(l.variant)) {  // the exchange instance cannot run pairs: undo them
+        for (ReqDesc& d : b.descs) d.pair = 0;
+        if (many || (ga && ga[0] == '1')) group_equal_requests(b, ub);
+        make_launchable(b, true, l, sm_count, ub);
+    } else if (paired && !xpaired && !pair_variant(l.variant)) {  // the chosen instance cannot run pairs: undo them
         for (ReqDesc& d : b.descs) d.pair = 0;
         spread_items(b, ub, false);
         make_launchable(b, false, l, sm_count, ub);

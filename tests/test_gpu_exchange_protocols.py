@@ -199,6 +199,31 @@ def test_window_protocol_mismatched_widths_fan_out(ddt, monkeypatch, no_ll):
     p.close()
 
 
+@pytest.mark.parametrize("base,no_ll", [("double", False), ("double", True), ("float", False)])
+def test_window_protocol_exchange_pairs(ddt, monkeypatch, base, no_ll):
+    """Exchange pairs (+x / -x packs in one item, both ghost ends unpacked in
+    one item: two flags waited, two signalled, or two LL words polled
+    together), forced on a small 26-direction plan (multi-wave plans pair by
+    default), direct and captured in a graph."""
+    import torch
+    env = {"DDT_SELF_VIA_WINDOW": "1", "DDT_XPAIR_ALWAYS": "1"}
+    if no_ll:
+        env["DDT_NO_LL"] = "1"
+    _env(monkeypatch, **env)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):  # the plan's queue (and the capture) on a side stream
+        p = Plan(ddt, (10, 14, 18), ALL_DIRS, 2, "p2p", base=base)
+        _run(p, 3, f"exchange pairs {base} no_ll={no_ll}")
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(3):
+                p.h.exchange()
+        p.fill(7)
+        g.replay()
+        p.check("exchange pairs graph")
+    p.close()
+
+
 def test_window_protocol_large_faces_graph(ddt, monkeypatch):
     """(4, 260, 260) doubles: 528 KiB z faces (> the LL limit) -> per-chunk
     flags at 2 vectors per thread per item, replayed from a captured graph."""

@@ -220,6 +220,9 @@ def _spawn(target, world, extra, timeout=400):
     (2, dict(dirs="faces", local=(128, 128, 128), nvars=1, iters=2, mode="p2p_direct")),
     # one CTA per item forced for the exchange kernel (ticket-claimed)
     (2, dict(dirs="all", local=(12, 20, 24), iters=3, env={"DDT_XGRID_MODE": "2"})),
+    # exchange pairs (+x / -x packs and unpacks in one item) between real processes
+    (2, dict(dirs="all", local=(12, 20, 24), iters=3, env={"DDT_XPAIR_ALWAYS": "1"})),
+    (8, dict(dirs="all", local=(6, 10, 12), iters=2, env={"DDT_XPAIR_ALWAYS": "1", "DDT_NO_LL": "1"})),
 ])
 def test_exchange_protocols_multiprocess(world, opts):
     res = _spawn(_worker_bytes, world, (opts,))
