@@ -444,8 +444,8 @@ static int batch_variant(const HostBatch& b) {
 }
 
 // Work distribution of a multi-wave plain batch (>= kTicketMinItemsPerSM
-// items per SM, no exchange flags; exchange batches keep the static order their
-// flag protocol is proven for).  Measured on one B200:
+// items per SM, no exchange flags; exchange batches: see below).  Measured on
+// one B200:
 //   * spread halo plans (COMB) and sparse batches: one CTA per item (grid_mode 2)
 //     -- COMB 128 -> 116 us, configs[2] 32 x 10^5 x 12 B 55 -> 52 us;
 //   * <= kTicketMaxReqs large requests: dynamic tickets (grid_mode 1) --

@@ -9,9 +9,11 @@
 //
 // B200 design: pure HBM-bound byte movement, no tensor
 // cores.  The host builds a work table (exclusive prefix sum of per-request
-// item counts); CTA b walks items b, b + grid, ... in
-// increasing order (grid <= resident CTAs on the 148 SMs), finds its request
-// with a binary search of the prefix, caches the descriptors in shared memory
+// item counts); CTAs take items in a static cyclic order
+// (CTA b: b, b + grid, ...), from a dynamic ticket, from an explicit spread
+// table or one item per CTA (batch.cpp grid_mode_for; exchange kernels always
+// claim by ticket), find the request with a binary search of the prefix,
+// cache the descriptors in shared memory
 // and moves kItemVecs vectors of the request's packed stream.  Thread i of the
 // CTA takes vectors v0 + i + u*kThreads, so the packed side is perfectly
 // coalesced and the strided side is coalesced within each segment.  The vector
