@@ -179,7 +179,8 @@ __device__ __forceinline__ int64_t vec_offset(const ReqDesc& d, uint32_t v) {
 // prologue of step k+1 hide under step k.
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 // Source lines of the first item are prefetched into L2 BEFORE griddepcontrol.wait
-// (one-slot latency instances, UNR == 1): a prefetch only moves a line into L2,
+// (latency-bound batches of one vector per thread per item, ub == 1): a
+// prefetch only moves a line into L2,
 // the point of coherence, so a write the preceding grid makes to it later
 // still lands there before the (post-wait) load reads it -- the DRAM latency
 // of the first loads hides under the wait.  configs[1] step 2.40 -> 2.09 us;
@@ -364,7 +365,7 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
                     wd[u] = false;
                     if (u < ub && v < nvec) phased_unit(S, v, s, within, wd[u]);
                     ps[u] = src + seg_offset(S, s) + within;
-                    if (DDT_PDL_PREFETCH && UNR == 1 && u < ub && v < nvec) prefetch_l2(ps[u]);
+                    if (DDT_PDL_PREFETCH && ub == 1 && u < ub && v < nvec) prefetch_l2(ps[u]);
                 }
                 pdl_wait();
 #pragma unroll
@@ -437,7 +438,7 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
             ps[u] = src + ((u < ub && v < nvec) ? (win_s ? gen_offset_win(S, v, *win, pre0, cnt, lw)
                                                          : vec_offset<LW, SONLY>(S, v))
                                                 : 0);
-            if (DDT_PDL_PREFETCH && UNR == 1 && u < ub && v < nvec) prefetch_l2(ps[u]);
+            if (DDT_PDL_PREFETCH && ub == 1 && u < ub && v < nvec) prefetch_l2(ps[u]);
         }
         pdl_wait();
 #pragma unroll
