@@ -266,3 +266,88 @@ def test_halo_create_fails_on_every_rank_together():
     res = _spawn(_bad_args_worker, 2, (), timeout=200)
     assert len(res) == 2, res
     assert all(v.startswith("error:") for v in res.values()), res
+
+
+def _occupied_worker(rank, world, port, q):
+    """2 processes on one GPU: each holds all but one SM of its context with an
+    occupier kernel (max shared carveout) on a side stream, then runs the P2P
+    window exchange (per-chunk flags, DDT_NO_LL) with its peer; both must finish
+    while their occupiers still run (processes time-slice the GPU)."""
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    os.environ["DDT_NO_LL"] = "1"
+    ok = False
+    try:
+        init(rank, world, port)
+        import ctypes
+        import time
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(0)
+        import paper_conf_cluster_chukzsp20_b200 as ddt
+        from gpu_util import occupier
+        from ddt_inputs import halo_messages, proc_grid, global_block, padded_block, ghost_mask, random_bytes, ALL_DIRS
+        P, local = world, (16, 40, 48)
+        G = tuple(n * g for n, g in zip(local, proc_grid(P)))
+        a = torch.zeros(tuple(n + 2 for n in local), dtype=torch.int64, device="cuda")
+        msgs = halo_messages(rank, P, local, dirs=ALL_DIRS)
+        sends = [(m["peer"], m["tag"], ddt.Type.from_spec(m["send_spec"]), a, 1) for m in msgs]
+        recvs = [(m["recv_peer"], m["recv_tag"], ddt.Type.from_spec(m["recv_spec"]), a, 1) for m in msgs]
+        comm = ddt.Comm.from_torch(0, nccl=False)
+        qq = ddt.Queue()
+        h = ddt.Halo(qq, comm, sends, recvs, mode="p2p", graph=False)
+        h.set_timeout(20.0)
+        gm = ghost_mask(local, ALL_DIRS)
+
+        def fill(it):
+            glob = random_bytes(int(np.prod(G)) * 8, 300 + it).view(np.int64).reshape(G)
+            a[1:-1, 1:-1, 1:-1] = torch.from_numpy(np.ascontiguousarray(global_block(glob, rank, P))).cuda()
+            torch.cuda.synchronize()
+            return glob
+
+        glob = fill(0)  # warm-up exchange: kernels loaded before the SMs are held
+        dist.barrier()
+        h.exchange()
+        torch.cuda.synchronize()
+        dist.barrier()
+        ok = bool(np.array_equal(a.cpu().numpy()[gm], padded_block(glob, rank, P)[gm]))
+        glob = fill(1)
+        occ = occupier()
+        nsm = torch.cuda.get_device_properties(0).multi_processor_count
+        ctas = 2 * nsm - 1
+        stop = torch.zeros(1, dtype=torch.int32).pin_memory()
+        started = torch.zeros(ctas, dtype=torch.int32).pin_memory()
+        s_occ = torch.cuda.Stream()
+        assert occ.occupy_launch(ctypes.c_void_p(s_occ.cuda_stream), ctas, 1024, ctypes.c_void_p(stop.data_ptr()),
+                                 ctypes.c_void_p(started.data_ptr()), int(60e9)) == 0
+        t0 = time.time()
+        while int(started.sum()) < ctas and time.time() - t0 < 20:
+            time.sleep(0.001)
+        ok &= int(started.sum()) == ctas
+        dist.barrier()
+        h.exchange()
+        cur = torch.cuda.current_stream()
+        t0 = time.time()
+        while not cur.query() and time.time() - t0 < 40:
+            time.sleep(0.002)
+        finished = cur.query()
+        still = not s_occ.query()
+        stop[0] = 1
+        torch.cuda.synchronize()
+        ok &= finished and still
+        dist.barrier()
+        ok &= bool(np.array_equal(a.cpu().numpy()[gm], padded_block(glob, rank, P)[gm]))
+        h.destroy()
+        dist.barrier()
+        comm.close()
+        qq.destroy()
+        dist.destroy_process_group()
+    except Exception as e:
+        print(f"rank {rank}: {type(e).__name__}: {e}", flush=True)
+        ok = False
+    q.put((rank, ok))
+
+
+@pytest.mark.timeout(600)
+def test_exchange_multiprocess_while_sms_are_held():
+    res = _spawn(_occupied_worker, 2, (), timeout=300)
+    assert len(res) == 2 and all(res.values()), res
