@@ -21,6 +21,9 @@ from ddt_inputs import FACE_DIRS, ALL_DIRS  # noqa: E402
 VARIANTS = {
     "direct": {},
     "direct_nopair": {"DDT_NO_PAIR": "1"},
+    "direct_grid0": {"DDT_GRID_MODE": "0"},
+    "direct_grid1": {"DDT_GRID_MODE": "1"},
+    "direct_nospread": {"DDT_SPREAD": "0"},
     "direct_ub2": {"DDT_SPREAD_UB": "2"},
     "direct_dense4": {"DDT_SPREAD_DENSE_UB": "4"},
     "direct_dense2": {"DDT_SPREAD_DENSE_UB": "2"},
@@ -40,7 +43,7 @@ def build(cfg, names):
     wls = {}
     base_env = dict(os.environ)
     for n in names:
-        for k in ("DDT_SELF_VIA_WINDOW", "DDT_XGRID_MODE", "DDT_XCLAIM", "DDT_NO_LL", "DDT_NO_PAIR", "DDT_SPREAD_UB", "DDT_SPREAD_DENSE_UB", "DDT_XUB_LL", "DDT_NO_XPAIR"):
+        for k in ("DDT_SELF_VIA_WINDOW", "DDT_XGRID_MODE", "DDT_XCLAIM", "DDT_NO_LL", "DDT_NO_PAIR", "DDT_SPREAD_UB", "DDT_SPREAD_DENSE_UB", "DDT_XUB_LL", "DDT_NO_XPAIR", "DDT_GRID_MODE", "DDT_SPREAD"):
             os.environ.pop(k, None)
         os.environ.update(VARIANTS[n])
         ddt.reload_env()
