@@ -797,7 +797,9 @@ def main():
             "kernel": kname, "alg_bytes_per_launch": alg_bytes,
             "note": (f"latency-bound: {alg_bytes / 1e6:.2f} MB of algorithmic bytes per step (self messages: "
                      "DirectIPC 2S, remote: 4S); time = device time per step in the back-to-back K-step run "
-                     "(kernel + inter-kernel gap)")}
+                     "(kernel + inter-kernel gap); traffic = DRAM bytes of ONE launch replayed alone under ncu, where "
+                     "the L2 prefetch issued before the PDL wait races the demand loads of the x-face cells (~1 MB "
+                     "of duplicate sector reads; back to back the prefetch completes first), 1.86 MB without it")}
 
     if rank == 0 and not dist_on:
         try:
