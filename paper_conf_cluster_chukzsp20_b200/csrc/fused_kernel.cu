@@ -46,6 +46,9 @@
 #ifndef DDT_PDL_PREFETCH
 #define DDT_PDL_PREFETCH 1
 #endif
+#ifndef DDT_PREFETCH_MAX_UB
+#define DDT_PREFETCH_MAX_UB 1
+#endif
 #ifndef DDT_LL_SLEEP
 #define DDT_LL_SLEEP 16
 #endif
@@ -365,7 +368,7 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
                     wd[u] = false;
                     if (u < ub && v < nvec) phased_unit(S, v, s, within, wd[u]);
                     ps[u] = src + seg_offset(S, s) + within;
-                    if (DDT_PDL_PREFETCH && ub == 1 && u < ub && v < nvec) prefetch_l2(ps[u]);
+                    if (DDT_PDL_PREFETCH && ub <= DDT_PREFETCH_MAX_UB && u < ub && v < nvec) prefetch_l2(ps[u]);
                 }
                 pdl_wait();
 #pragma unroll
@@ -438,7 +441,7 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
             ps[u] = src + ((u < ub && v < nvec) ? (win_s ? gen_offset_win(S, v, *win, pre0, cnt, lw)
                                                          : vec_offset<LW, SONLY>(S, v))
                                                 : 0);
-            if (DDT_PDL_PREFETCH && ub == 1 && u < ub && v < nvec) prefetch_l2(ps[u]);
+            if (DDT_PDL_PREFETCH && ub <= DDT_PREFETCH_MAX_UB && u < ub && v < nvec) prefetch_l2(ps[u]);
         }
         pdl_wait();
 #pragma unroll
