@@ -1,7 +1,7 @@
 """Measurement sweep over BASELINE.json configs 1, 3 and 5 on one B200 (the
 bench line carries configs[1]; this tool produces the per-config tables in
-profiles/).  Device times from CUDA events on the queue's stream; L2 flushed
-(256 MiB write) before every timed repetition unless the working set exceeds
+profiles/).  Device times from CUDA events on the queue's stream; L2 evicted
+(256 MiB read sweep) before every timed repetition unless the working set exceeds
 L2 by itself.  Prints one JSON document.
 
 configs[0]  vector(16,4,64) of double: pack+unpack per iteration (2 flushes or
@@ -33,7 +33,7 @@ FLUSH = None
 
 
 def flush_l2():
-    FLUSH.fill_(1)
+    FLUSH.max()  # read sweep: evicts L2 without leaving dirty lines to write back in the timed region
 
 
 def timed(fn, reps, flush=True, setup=None):
