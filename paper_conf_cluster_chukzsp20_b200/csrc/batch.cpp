@@ -170,7 +170,7 @@ static bool same_lattice(const ReqDesc& a, const ReqDesc& c) {
 // Pair requests whose both sides walk the same short-segment lattice (see
 // device_desc.h kSpreadShift): partners become adjacent, the first carries
 // pair = 1.  Spread (non-exchange, plain) batches only.  DDT_NO_PAIR=1: off.
-static void pair_requests(HostBatch& b) {
+void pair_requests(HostBatch& b) {
     const char* off = DDT_KNOB("DDT_NO_PAIR");
     if ((off && off[0] == '1') || !b.gm.empty()) return;
     const size_t n = b.descs.size();

@@ -193,6 +193,8 @@ bool spread_items(HostBatch& b, int ub, bool allow_pair = true);
 inline bool pair_variant(int v) { return v == 9 || v == 7 || v == 4; }
 inline bool xpair_variant(int v) { return v == 11 || v == 12; }
 bool pair_exchange_requests(HostBatch& b);
+// Pair plain (non-exchange) requests walking the same short-segment lattice (device_desc.h).
+void pair_requests(HostBatch& b);
 // Param form if it fits (and allowed), else form 3 with `dev` left to the caller.
 // force_ub > 0 fixes the item size (exchange plans: sender and receiver chunk alike).
 void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int sm_count = 148, int force_ub = 0);

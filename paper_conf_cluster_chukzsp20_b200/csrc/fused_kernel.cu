@@ -833,7 +833,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             if constexpr (XCHG) copy_words(&sx, tv.xinfo + r, kXWords, 32);
             copy_words(&sa, tv.aux + r, kWords, 64);  // destination descriptor (aux[r], see HostBatch::add)
             if constexpr (!XCHG && PAIR) {
-                if (tv.order && tv.descs[r].pair) {  // paired request: its partner r + 1 too
+                if (tv.descs[r].pair) {  // paired request: its partner r + 1 too (spread table or prefix form)
                     copy_words(&sd2, tv.descs + r + 1, kWords, 128);
                     copy_words(&sa2, tv.aux + r + 1, kWords, 192);
                 }
@@ -910,7 +910,8 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         if constexpr (SEG && !XCHG) {
             run_seg<kSegUnroll>(*S, *D, v0, (int)tv.ub, !waited);
         } else if (!XCHG && PAIR && S->pair) {
-            run_pair<LW, SONLY>(sd, sa, sd2, sa2, v0, ubr, !waited);
+            if constexpr (INPLACE) run_pair<LW, SONLY>(*S, *D, S[1], D[1], v0, ubr, !waited);  // partner r + 1
+            else run_pair<LW, SONLY>(sd, sa, sd2, sa2, v0, ubr, !waited);
         } else if (XCHG && PAIR && S->pair) {
             if (run) run_pair_x<LW, SONLY>(sd, sa, sd2, sa2, v0, ubr, xa, (uint32_t)epoch);
         } else {
@@ -1061,8 +1062,11 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_dev(const u
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
     pdl_trigger();
+    // parameter batches run pairs in the one-slot instance only (one-wave plans
+    // pair on request, halo.cpp DDT_PAIR1; carrying the branch also measured
+    // faster for the unpaired configs[1] step: 2.08 -> 1.99 us)
     fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_PARAM, VarT<V>::UNR, true,
-               VarT<V>::SEG>(view_of(pb), nullptr);
+               VarT<V>::SEG, V == 9>(view_of(pb), nullptr);
 }
 
 template <int V>

@@ -232,7 +232,13 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
     // proxy: 4.35 us unpaired, 6.35 us paired)
     const char* xpa = DDT_KNOB("DDT_XPAIR_ALWAYS");  // tests: pair one-wave exchange plans too
     const bool xpaired = force_ub > 0 && (many || (xpa && xpa[0] == '1')) && pair_exchange_requests(b);
-    if (!spread && !xpaired && (many || (ga && ga[0] == '1'))) group_equal_requests(b, ub);
+    // one-wave plain plans pair their +x / -x requests only on request
+    // (DDT_PAIR1=1: configs[1] 1.99 -> 2.32 us when paired)
+    const char* p1 = DDT_KNOB("DDT_PAIR1");
+    if (!spread && force_ub <= 0 && !many && p1 && p1[0] == '1') pair_requests(b);
+    bool ppaired = false;
+    for (const ReqDesc& d : b.descs) ppaired |= !spread && !xpaired && d.pair != 0;
+    if (!spread && !xpaired && !ppaired && (many || (ga && ga[0] == '1'))) group_equal_requests(b, ub);
     for (ReqDesc& d : b.descs)  // response slots: the finishing CTA compares its count with the item count
         if (d.resp) d.nitems = desc_items(d, ub);
     make_launchable(b, !spread, l, sm_count, ub);
@@ -242,10 +248,11 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
         for (ReqDesc& d : b.descs) d.pair = 0;
         if (many || (ga && ga[0] == '1')) group_equal_requests(b, ub);
         make_launchable(b, true, l, sm_count, ub);
-    } else if (paired && !xpaired && !pair_variant(l.variant)) {  // the chosen instance cannot run pairs: undo them
+    } else if (paired && !xpaired && (l.form == 3 ? !pair_variant(l.variant) : l.variant != 9)) {
+        // the chosen instance cannot run pairs (parameter batches: the one-slot instance only): undo them
         for (ReqDesc& d : b.descs) d.pair = 0;
-        spread_items(b, ub, false);
-        make_launchable(b, false, l, sm_count, ub);
+        if (spread) spread_items(b, ub, false);
+        make_launchable(b, !spread, l, sm_count, ub);
     }
     if (l.form != 3) return DDT_OK;
     std::vector<uint8_t> host(device_table_bytes(b));

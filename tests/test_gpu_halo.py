@@ -75,7 +75,7 @@ def _check(arrs, local, dirs, before=None):
     ((5, 6, 7), ALL_DIRS, 2, 4),
     ((9, 4, 3), FACE_DIRS, 1, 2),
 ])
-@pytest.mark.parametrize("group", [False, True, "spread"])
+@pytest.mark.parametrize("group", [False, True, "spread", "pair1"])
 def test_halo_small(ddt, mode, graph, local, dirs, nvars, cfg, group, monkeypatch):
     """group=True: equal-size requests interleaved chunk by chunk even though the
     plan is one wave (the default only groups multi-wave plans); "spread": the
@@ -84,6 +84,8 @@ def test_halo_small(ddt, mode, graph, local, dirs, nvars, cfg, group, monkeypatc
     import torch
     if group == "spread":
         monkeypatch.setenv("DDT_SPREAD_ALWAYS", "1")
+    elif group == "pair1":  # one-wave plan with its +x / -x requests paired (prefix form, in place / device table)
+        monkeypatch.setenv("DDT_PAIR1", "1")
     elif group:
         monkeypatch.setenv("DDT_GROUP_ALWAYS", "1")
     q, arrs, h, comm = _setup(ddt, local, dirs, nvars, mode, graph, cfg)
