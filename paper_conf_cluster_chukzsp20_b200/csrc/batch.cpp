@@ -522,7 +522,9 @@ void make_launchable(const HostBatch& b, bool allow_param, Launchable& out, int 
         // (default kXClaim) consecutive items over a resident grid (grid_mode 1)
         out.ticket = b.ticket;
         const char* xc = DDT_KNOB("DDT_XCLAIM");
-        out.claim = out.grid_mode == 2 ? 0u : (uint32_t)(xc ? std::max(1, atoi(xc)) : kXClaim);
+        const char* xg = DDT_KNOB("DDT_XONCE_G");  // items per CTA of one-wave exchange launches
+        out.claim = out.grid_mode == 2 ? (kXOnce | (uint32_t)(xg ? std::max(1, std::min(64, atoi(xg))) : 1))
+                                       : (uint32_t)(xc ? std::max(1, atoi(xc)) : kXClaim);
     }
     const char* force = DDT_KNOB("DDT_FORCE_TABLE");  // experiments: always use the device-table form
     if (force && force[0] == '1') allow_param = false;
@@ -551,7 +553,10 @@ int launch_fused(const Launchable& l, void* stream, int grid_cap) {
 
 int launch_exchange(const Launchable& l, const XArgs& xa, void* stream, int grid_cap) {
     const void* src = l.form == 3 ? l.dev : (const void*)l.blob.data();
-    if (l.grid_mode == 2 && grid_cap <= 0) grid_cap = -1;  // one CTA per item (ticket-claimed)
+    if (l.grid_mode == 2 && grid_cap <= 0) {  // one claim of G items per CTA: grid = ceil(items / G)
+        const uint32_t G = std::max(1u, l.claim & ~kXOnce);
+        grid_cap = -(int)((l.total_items + G - 1) / G);
+    }
     return launch_exchange_form(l.form, l.variant, src, l.total_items, xa, stream, grid_cap);
 }
 

@@ -160,7 +160,7 @@ struct alignas(16) BatchHeader {
     uint32_t ub;            // vectors per thread per item (1, 2 or 4)
     uint32_t flags;         // bit 0: blocked item order (else cyclic over CTAs); bit 1: grouped (gm[] present)
     uint32_t order_offset;  // 0, or byte offset of the explicit item table (kBatchSpread)
-    uint32_t claim;         // exchange batches: items per claim (0 = one item per CTA, grid == total_items)
+    uint32_t claim;         // exchange batches: items per claim, | kXOnce = one claim per CTA (grid = ceil(items / G))
     uint64_t ticket;        // plain: 0 = static order, else device u32[2] {next, exited}; exchange: XCtrl::tick
 };
 // Dynamic item tickets (multi-wave plain batches): a resident-sized grid takes
@@ -175,6 +175,9 @@ constexpr uint32_t kTicketMaxReqs = 64;
 constexpr uint32_t kBatchBlocked = 1u, kBatchGrouped = 2u;
 // Items per ticket claim of a multi-wave exchange launch (resident grid).
 constexpr uint32_t kXClaim = 4;
+// BatchHeader::claim flag: one claim per CTA (one-wave exchange plans, grid =
+// ceil(items / G) for claim = kXOnce | G).
+constexpr uint32_t kXOnce = 0x80000000u;
 // Spread batches (batch.cpp spread_items): an explicit item table order[item] =
 // (request << kSpreadShift) | chunk, ordered so that every request's chunks are
 // spread evenly over the whole launch (chunk c of a request of n items sits at

@@ -766,33 +766,38 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         first = s_tk[0];
         last = tv.total;
     }
-    // exchange: claim items (chunks of xclaim, or one item per CTA) from the
-    // plan's monotonic tick in item order; the first claim also fixes the
-    // epoch (device_desc.h XCtrl).  Thread 0 prefetches the next chunk's claim.
+    // exchange: claim items from the plan's monotonic tick in item order; the
+    // first claim also fixes the epoch (device_desc.h XCtrl).  Two modes:
+    //   once (one-wave plans, claim = kXOnce | G): grid = ceil(items / G), every
+    //     CTA claims exactly one chunk of G items, span = G * grid;
+    //   loop (multi-wave plans, claim = G): a resident grid claims chunks of G
+    //     until one claim lands past the end (thread 0 prefetches the next).
     __shared__ unsigned long long s_xt[2];
     unsigned long long* xtick = nullptr;
     uint32_t xclaim = 0;
+    bool xonce = false;
     uint64_t xspan = 0, xend = 0;
     if constexpr (XCHG) {
         xtick = reinterpret_cast<unsigned long long*>(tv.ticket);
-        xclaim = tv.claim;
-        const uint64_t nch = xclaim ? ((uint64_t)tv.total + xclaim - 1) / xclaim : (uint64_t)tv.total;
-        xspan = xclaim ? (uint64_t)xclaim * (nch + gridDim.x) : (uint64_t)tv.total;
-        xend = xclaim ? (uint64_t)xclaim * nch : (uint64_t)tv.total;
-        // programmatic dependent launch: with one item per CTA (claim 0) the
-        // CTA claims its ticket BEFORE waiting for the preceding grid and only
-        // then lets the next grid launch -- the claim's atomic round trip hides
-        // under the predecessor's tail, and a successor (of this plan or any
-        // other kernel) can only start once every CTA of this grid has claimed,
-        // so launches of one plan never interleave their tickets (the span
-        // arithmetic holds).  Looping grids trigger and wait first.
-        if (xclaim) {
+        xonce = tv.claim == 0 || (tv.claim & kXOnce);
+        xclaim = xonce ? max(1u, tv.claim & ~kXOnce) : tv.claim;
+        const uint64_t nch = ((uint64_t)tv.total + xclaim - 1) / xclaim;
+        xspan = xonce ? (uint64_t)xclaim * gridDim.x : (uint64_t)xclaim * (nch + gridDim.x);
+        xend = xonce ? (uint64_t)tv.total : (uint64_t)xclaim * nch;
+        // programmatic dependent launch: in once mode the CTA claims its chunk
+        // BEFORE waiting for the preceding grid and only then lets the next grid
+        // launch -- the claim's atomic round trip hides under the predecessor's
+        // tail, and a successor (of this plan or any other kernel) can only start
+        // once every CTA of this grid has claimed, so launches of one plan never
+        // interleave their tickets (the span arithmetic holds).  Looping grids
+        // trigger and wait first.
+        if (!xonce) {
             pdl_trigger();
             pdl_wait();
         }
-        if (threadIdx.x == 0) s_xt[0] = atomicAdd(xtick, xclaim ? (unsigned long long)xclaim : 1ull);
+        if (threadIdx.x == 0) s_xt[0] = atomicAdd(xtick, (unsigned long long)xclaim);
         __syncthreads();
-        if (!xclaim) pdl_trigger();  // the wait follows the first item's descriptor staging (static data)
+        if (xonce) pdl_trigger();  // the wait follows the first item's descriptor staging (static data)
         const uint64_t t = s_xt[0];
         epoch = t / xspan + 1ull;
         const uint64_t loc = t % xspan;
@@ -800,8 +805,8 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             first = last = 0;  // this CTA's one failing claim: nothing to do
         } else {
             first = (uint32_t)loc;
-            last = xclaim ? min(tv.total, (uint32_t)loc + xclaim) : (uint32_t)loc + 1u;
-            if (xclaim && threadIdx.x == 0) s_xt[1] = atomicAdd(xtick, (unsigned long long)xclaim);  // prefetch
+            last = min(tv.total, (uint32_t)loc + xclaim);
+            if (!xonce && threadIdx.x == 0) s_xt[1] = atomicAdd(xtick, (unsigned long long)xclaim);  // prefetch
         }
     }
     for (uint32_t item = first; item < last;) {
@@ -865,7 +870,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             cur = r;
         }
         if constexpr (XCHG) {
-            if (!xclaim && item == first) {
+            if (xonce && item == first) {
                 pdl_wait();  // before any flag or data access
             }
         }
@@ -985,7 +990,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             item = s_tk[par];
         } else if (XCHG) {
             if (++item >= last) {  // chunk done: take the prefetched claim
-                if (!xclaim) break;
+                if (xonce) break;
                 __syncthreads();   // the prefetched claim is visible; every thread is past this item
                 par ^= 1;
                 const uint64_t loc = s_xt[par] % xspan;
@@ -1106,7 +1111,10 @@ static int resident_ctas(K kernel) {
 }
 
 static uint32_t grid_for(uint32_t total, int resident, int grid_cap) {
-    if (grid_cap < 0) return total;  // one CTA per item (Launchable::grid_mode 2, plain batches only)
+    // grid_cap < 0: an explicit grid of -grid_cap CTAs (one CTA per item: -1 = total;
+    // one-wave exchange launches: ceil(items / G)), not limited to the resident CTAs
+    if (grid_cap == -1) return total;
+    if (grid_cap < 0) return (uint32_t)(-grid_cap);
     uint32_t cap = (uint32_t)resident;
     if (grid_cap > 0 && (uint32_t)grid_cap < cap) cap = (uint32_t)grid_cap;
     return total < cap ? total : cap;
