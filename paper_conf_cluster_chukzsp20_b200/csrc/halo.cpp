@@ -27,6 +27,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <map>
+#include <mutex>
 #include <tuple>
 #include <vector>
 
@@ -457,9 +458,8 @@ struct MemOps {
 };
 const MemOps* memops() {
     static MemOps m;
-    static bool init = false;
-    if (!init) {
-        init = true;
+    static std::once_flag once;
+    std::call_once(once, [] {
         cudaDriverEntryPointQueryResult q1, q2;
         if (cudaGetDriverEntryPoint("cuStreamWaitValue32", (void**)&m.wait, cudaEnableDefault, &q1) != cudaSuccess ||
             q1 != cudaDriverEntryPointSuccess)
@@ -467,7 +467,7 @@ const MemOps* memops() {
         if (cudaGetDriverEntryPoint("cuStreamWriteValue32", (void**)&m.write, cudaEnableDefault, &q2) != cudaSuccess ||
             q2 != cudaDriverEntryPointSuccess)
             m.write = nullptr;
-    }
+    });
     return (m.wait && m.write) ? &m : nullptr;
 }
 
