@@ -57,6 +57,16 @@ struct RecvLayout {
     int64_t flags_bytes = 0, parity_stride = 0, window_bytes = 0;
 };
 
+// Item size (vectors per thread) of a flagged / LL exchange message: a
+// function of its byte size (and of one run-wide knob), so the sender and the
+// receiver -- whose plans differ -- chunk it identically (device_desc.h
+// xchg_ub_for).  DDT_XUB_SMALL: experiments (messages <= kLLMaxBytes).
+int xub_for(int64_t bytes) {
+    const char* e = DDT_KNOB("DDT_XUB_SMALL");
+    if (bytes <= kLLMaxBytes && e && (e[0] == '1' || e[0] == '2')) return e[0] - '0';
+    return xchg_ub_for(bytes);
+}
+
 // reserve_ll: window space for the LL format (P2P window mode only; the NCCL
 // staging must not carry the gaps -- they would be transferred).
 RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs, bool reserve_ll = true) {
@@ -75,7 +85,7 @@ RecvLayout layout_recvs(int32_t nrecv, const ddt_recv_t* recvs, bool reserve_ll 
     for (size_t k = 0; k < L.order.size(); k++) {
         int i = L.order[k];
         int64_t bytes = recvs[i].count * recvs[i].type->size;
-        const int64_t chunk = (int64_t)kThreads * xchg_ub_for(bytes);  // vectors per exchange item
+        const int64_t chunk = (int64_t)kThreads * xub_for(bytes);  // vectors per exchange item
         off = round_up(off, kAlign);
         L.data_off[(size_t)i] = off;
         int lw = recvs[i].type->committed ? std::min(4, side_lw(recvs[i].type, recvs[i].buf, recvs[i].count)) : 0;
@@ -1013,7 +1023,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                     st = build_ll(OP_PACK, s.type, dl, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count,
                                   &sd, &dd);
                 if (st != DDT_OK) break;
-                sd.xub = (uint8_t)xchg_ub_for(s.count * s.type->size);  // no flags: free to pick the item size
+                sd.xub = (uint8_t)xub_for(s.count * s.type->size);  // no flags: free to pick the item size
                 xb.add(sd, dd);
                 XInfo x{};
                 x.parity_stride = d.parity_stride;
@@ -1022,7 +1032,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             }
             int lw = 0;
             st = add_req(xb, s.type, OP_PACK, s.buf, win + d.data_base + match[(size_t)i]->data_off, s.count, &lw);
-            if (st == DDT_OK) xb.descs.back().xub = (uint8_t)xchg_ub_for(s.count * s.type->size);
+            if (st == DDT_OK) xb.descs.back().xub = (uint8_t)xub_for(s.count * s.type->size);
             XInfo x{};
             x.signal = (uint64_t)(uintptr_t)(win + 8 * match[(size_t)i]->flag_idx);
             x.counter = npack++;
@@ -1066,7 +1076,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             if (st == DDT_OK && sd.nvec != dd.nvec) st = DDT_ERR_SIZE_MISMATCH;
             if (st != DDT_OK) break;
             sd.op = dd.op = OP_DIRECT;
-            sd.xub = (uint8_t)xchg_ub_for(s.count * s.type->size);  // one done flag per message: any chunking
+            sd.xub = (uint8_t)xub_for(s.count * s.type->size);  // one done flag per message: any chunking
             xb.add(sd, dd);
             XInfo x{};
             x.signal = (uint64_t)(uintptr_t)((char*)c->peer_windows[s.peer] + 8 * e.flag_idx);
@@ -1090,14 +1100,14 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                     st = build_ll(OP_UNPACK, r.type, dl, r.buf, mywin + RL.flags_bytes + RL.data_off[(size_t)i],
                                   r.count, &sd, &dd);
                 if (st != DDT_OK) break;
-                sd.xub = (uint8_t)xchg_ub_for(r.count * r.type->size);
+                sd.xub = (uint8_t)xub_for(r.count * r.type->size);
                 xb.add(sd, dd);
                 x.wait = 0;
                 x.parity_stride = RL.parity_stride;
             } else {  // unpack chunk k as soon as the sender's chunk k has landed
                 st = add_req(xb, r.type, OP_UNPACK, mywin + RL.flags_bytes + RL.data_off[(size_t)i], r.buf, r.count,
                              nullptr);
-                if (st == DDT_OK) xb.descs.back().xub = (uint8_t)xchg_ub_for(r.count * r.type->size);
+                if (st == DDT_OK) xb.descs.back().xub = (uint8_t)xub_for(r.count * r.type->size);
                 x.parity_stride = RL.parity_stride;
                 x.per_item = 1;
             }

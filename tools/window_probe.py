@@ -34,6 +34,7 @@ VARIANTS = {
     "window_claim16": {"DDT_SELF_VIA_WINDOW": "1", "DDT_XGRID_MODE": "1", "DDT_XCLAIM": "16"},
     "window_noll": {"DDT_SELF_VIA_WINDOW": "1", "DDT_NO_LL": "1"},
     "window_g2": {"DDT_SELF_VIA_WINDOW": "1", "DDT_XONCE_G": "2"},
+    "window_xub2": {"DDT_SELF_VIA_WINDOW": "1", "DDT_XUB_SMALL": "2"},
     "window_g4": {"DDT_SELF_VIA_WINDOW": "1", "DDT_XONCE_G": "4"},
     "window_noxpair": {"DDT_SELF_VIA_WINDOW": "1", "DDT_NO_XPAIR": "1"},
     "window_llub2": {"DDT_SELF_VIA_WINDOW": "1", "DDT_XUB_LL": "2"},
@@ -45,7 +46,7 @@ def build(cfg, names):
     wls = {}
     base_env = dict(os.environ)
     for n in names:
-        for k in ("DDT_SELF_VIA_WINDOW", "DDT_XGRID_MODE", "DDT_XCLAIM", "DDT_NO_LL", "DDT_NO_PAIR", "DDT_SPREAD_UB", "DDT_SPREAD_DENSE_UB", "DDT_XUB_LL", "DDT_NO_XPAIR", "DDT_GRID_MODE", "DDT_SPREAD", "DDT_XONCE_G"):
+        for k in ("DDT_SELF_VIA_WINDOW", "DDT_XGRID_MODE", "DDT_XCLAIM", "DDT_NO_LL", "DDT_NO_PAIR", "DDT_SPREAD_UB", "DDT_SPREAD_DENSE_UB", "DDT_XUB_LL", "DDT_NO_XPAIR", "DDT_GRID_MODE", "DDT_SPREAD", "DDT_XONCE_G", "DDT_XUB_SMALL"):
             os.environ.pop(k, None)
         os.environ.update(VARIANTS[n])
         ddt.reload_env()
