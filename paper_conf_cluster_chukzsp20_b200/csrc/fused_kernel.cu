@@ -956,13 +956,27 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
                             if (X.gpu_scope) st_release_gpu(flag + local, epoch);
                             else st_release_sys(flag + local, epoch);
                         } else if (X.nitems <= 1) {
-                            __threadfence_system();
+                            // a data-free signal (the pack-free "ready" item) orders no
+                            // stores of its own: the reads it vouches for belong to the
+                            // preceding grid, complete at the grid dependency
+                            if (sd.op != OP_SIGNAL) {
+                                if (X.gpu_scope) __threadfence();
+                                else __threadfence_system();
+                            }
                             for (uint32_t k = 0; k < X.fanout; k++) st_relaxed_sys(flag + k, epoch);
                         } else {
-                            __threadfence_system();
-                            unsigned long long old = atomicAdd_system(&ctrl->counters[X.counter], 1ull);
+                            // fan-in over this GPU's CTAs: the counter is only touched by
+                            // them, so a gpu-scope release / atomic synchronises each CTA
+                            // with the last one, and the last one's fence at the flag
+                            // reader's scope (a peer GPU: sys) releases every CTA's stores
+                            // (causality order is transitive, PTX ISA memory model) --
+                            // configs[1] pack-free proxy at sys scope 16.5 -> see DESIGN.md
+                            __threadfence();
+                            unsigned long long old = atomicAdd(&ctrl->counters[X.counter], 1ull);
                             if (old + 1ull == epoch * (unsigned long long)X.nitems) {
-                                __threadfence_system();  // one release for all of the message's flags
+                                // one release for all of the message's flags
+                                if (X.gpu_scope) __threadfence();
+                                else __threadfence_system();
                                 for (uint32_t k = 0; k < X.fanout; k++) st_relaxed_sys(flag + k, epoch);
                             }
                         }

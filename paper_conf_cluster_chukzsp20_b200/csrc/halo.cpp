@@ -233,7 +233,10 @@ ddt_status_t make_table(HostBatch& b, Launchable& l, int sm_count, int force_ub 
             for (ReqDesc& d : b.descs)
                 if (!d.l2_64 && !b.aux[d.aux].l2_64 && d.op != OP_SIGNAL) d.xub = (uint8_t)dub;
         spread = spread_items(b, sub);
-        if (!spread)
+        // undo the dense item sizes set above (only those: an exchange plan's
+        // xub is part of its protocol -- the receiver's chunk flags and the
+        // message counters assume xub_for's chunking)
+        if (!spread && force_ub <= 0)
             for (ReqDesc& d : b.descs) d.xub = 0;
         if (spread) ub = sub;
     }
@@ -687,6 +690,13 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     for (auto& s : h->sends) type_retain(s.type);
     for (auto& r : h->recvs) type_retain(r.type);
 
+    // test hook (never set in production): in P2P_DIRECT mode, route self
+    // messages through the pack-free remote protocol (ready flag -> gather ->
+    // scatter into the "peer's" receive buffer -> done flag), so one GPU
+    // exercises and times it
+    const char* svd = DDT_KNOB("DDT_SELF_VIA_DIRECT");
+    const bool self_direct = direct && svd && svd[0] == '1';
+
     // ---- receive layout (above) and directories (receiver -> each sender)
     const int P = c->nranks;
     std::vector<std::vector<int64_t>> dir_out((size_t)P), dir_in;
@@ -695,7 +705,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         for (int k : RL.order)
             if (recvs[k].peer == p) mine.push_back(k);
         auto& v = dir_out[(size_t)p];
-        const bool dmsg = direct && p != c->rank;
+        const bool dmsg = direct && (p != c->rank || self_direct);
         v = {(int64_t)mine.size(), RL.parity_stride, RL.flags_bytes, RL.ready_off, dmsg ? 1 : 0};
         for (int k : mine) {
             v.push_back(recvs[k].tag);
@@ -784,7 +794,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
     // exercise and time the multi-GPU protocols
     const char* svw = DDT_KNOB("DDT_SELF_VIA_WINDOW");
     const bool self_window = p2p && !direct && svw && svw[0] == '1';
-    auto remote = [&](int peer) { return peer != c->rank || self_window; };
+    auto remote = [&](int peer) { return peer != c->rank || self_window || self_direct; };
     // the same for NCCL mode (needs an NCCL communicator, e.g. a 1-rank one):
     // self messages go pack -> staging -> ncclSend/ncclRecv to self -> unpack
     const char* svn = DDT_KNOB("DDT_SELF_VIA_NCCL");
@@ -997,7 +1007,7 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         none.op = OP_SIGNAL;
         std::vector<int> rpeers;  // remote peers we receive from (== send to: symmetric)
         for (int i = 0; i < nrecv; i++)
-            if (recvs[i].peer != c->rank && recvs[i].count * recvs[i].type->size > 0) rpeers.push_back(recvs[i].peer);
+            if (remote(recvs[i].peer) && recvs[i].count * recvs[i].type->size > 0) rpeers.push_back(recvs[i].peer);
         std::sort(rpeers.begin(), rpeers.end());
         rpeers.erase(std::unique(rpeers.begin(), rpeers.end()), rpeers.end());
         if (direct) {  // "ready": this rank entered the exchange, its ghosts may be overwritten
@@ -1006,6 +1016,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
                 x.signal = (uint64_t)(uintptr_t)((char*)c->peer_windows[p] + dirs[(size_t)p].ready_base + 8 * c->rank);
                 x.nitems = 1;
                 x.fanout = 1;
+                const char* fs0 = DDT_KNOB("DDT_FORCE_SYS_SCOPE");  // experiments: emulate a peer GPU's flags
+                x.gpu_scope = (p == c->rank && !(fs0 && fs0[0] == '1')) ? 1u : 0u;  // self (test hook)
                 xb.add(none, none);
                 xb.xinfo.push_back(x);
             }
@@ -1054,19 +1066,23 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
         }
         for (int i = 0; i < nsend && st == DDT_OK && direct; i++) {
             const auto& s = sends[i];
-            if (s.count * s.type->size == 0 || s.peer == c->rank) continue;
+            if (s.count * s.type->size == 0 || !remote(s.peer)) continue;
             const DirEntry& e = *match[(size_t)i];
-            cudaIpcMemHandle_t ih;
-            std::memcpy(&ih, e.ipc, 64);
-            void* mapped = nullptr;
-            cudaError_t ce = cudaIpcOpenMemHandle(&mapped, ih, cudaIpcMemLazyEnablePeerAccess);
-            if (ce != cudaSuccess) {
-                st = cuda_fail("cudaIpcOpenMemHandle(peer recv buffer)", ce);
-                break;
-            }
-            h->ipc_opened.push_back(mapped);
             ReqDesc sd, dd = e.desc;
-            dd.ptr = (uint64_t)(uintptr_t)((char*)mapped + e.alloc_off);
+            if (s.peer == c->rank) {  // self through the remote protocol (test hook): no IPC mapping needed
+                dd.ptr = (uint64_t)(uintptr_t)recvs[self_recv(s.tag)].buf;
+            } else {
+                cudaIpcMemHandle_t ih;
+                std::memcpy(&ih, e.ipc, 64);
+                void* mapped = nullptr;
+                cudaError_t ce = cudaIpcOpenMemHandle(&mapped, ih, cudaIpcMemLazyEnablePeerAccess);
+                if (ce != cudaSuccess) {
+                    st = cuda_fail("cudaIpcOpenMemHandle(peer recv buffer)", ce);
+                    break;
+                }
+                h->ipc_opened.push_back(mapped);
+                dd.ptr = (uint64_t)(uintptr_t)((char*)mapped + e.alloc_off);
+            }
             DeviceLayout* dl = nullptr;
             st = type_device_layout(s.type, h->device, &dl);
             if (st == DDT_OK) st = build_typed(s.type, dl, s.buf, s.count, &sd);
@@ -1083,6 +1099,8 @@ ddt_status_t ddt_halo_create(ddt_queue_t q, const ddt_comm_t* c, int32_t nsend, 
             x.wait = (uint64_t)(uintptr_t)(mywin + RL.ready_off + 8 * s.peer);
             x.counter = npack++;
             x.fanout = 1;
+            const char* fs1 = DDT_KNOB("DDT_FORCE_SYS_SCOPE");
+            x.gpu_scope = (s.peer == c->rank && !(fs1 && fs1[0] == '1')) ? 1u : 0u;  // self (test hook)
             xb.xinfo.push_back(x);
         }
         for (int i = 0; i < nrecv && st == DDT_OK; i++) {

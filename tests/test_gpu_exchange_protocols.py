@@ -331,3 +331,57 @@ def test_k_exchanges_captured_in_one_graph(ddt, monkeypatch):
             g.replay()
             p.check(f"graph replay {it}")
         p.close()
+
+
+@pytest.mark.parametrize("local,dirs,nvars,base,dst_off", [
+    ((128, 128, 128), FACE_DIRS, 1, "double", None),   # configs[1]
+    ((10, 14, 18), ALL_DIRS, 2, "double", None),
+    ((12, 20, 36), ALL_DIRS, 2, "float", 4),            # receiver at 4 mod 8: 4-B vectors on that side
+    ((256, 256, 256), ALL_DIRS, 1, "double", None),     # multi-wave (resident grid claiming chunks)
+])
+@pytest.mark.parametrize("graph", [False, True])
+def test_direct_protocol_pack_free(ddt, monkeypatch, local, dirs, nvars, base, dst_off, graph):
+    """P2P_DIRECT (pack-free, §IV-B's DirectIPC path between GPUs):
+    with DDT_SELF_VIA_DIRECT=1 the self messages take the remote protocol --
+    the receiver's ready flag, the sender's gather straight into the
+    "peer's" receive layout (no staging), the per-message done flag the
+    receiver waits on -- the one-GPU stand-in for the IPC-mapped peer."""
+    _env(monkeypatch, DDT_SELF_VIA_DIRECT="1")
+    p = Plan(ddt, local, dirs, nvars, "p2p_direct", graph=graph, base=base, dst_off=dst_off)
+    _run(p, 4, f"direct {local} {base} graph={graph}")
+    p.close()
+
+
+def test_direct_protocol_k_exchanges_in_one_graph(ddt, monkeypatch):
+    """K = 5 pack-free exchanges (ready / done flags, device-resident epoch)
+    captured in one graph, replayed twice."""
+    import torch
+    _env(monkeypatch, DDT_SELF_VIA_DIRECT="1")
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        p = Plan(ddt, (20, 24, 28), ALL_DIRS, 2, "p2p_direct")
+        g = torch.cuda.CUDAGraph()
+        p.fill(0)
+        torch.cuda.synchronize()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(5):
+                p.h.exchange()
+        for it in range(1, 3):
+            p.fill(it)
+            g.replay()
+            p.check(f"direct graph replay {it}")
+        p.close()
+
+
+@pytest.mark.parametrize("dst_off", [None, 4])
+def test_window_protocol_multiwave_chunk_flags(ddt, monkeypatch, dst_off):
+    """A multi-wave plan (resident grid claiming chunks) with every message on
+    per-chunk flags (DDT_NO_LL=1): messages <= 512 KB keep their 1-vector
+    items (xub_for, the chunking the receiver's flags assume) -- a regression
+    test for the multi-wave table build once resetting every item size to the
+    plan's; dst_off = 4: different vector widths on the two sides, the
+    whole-message release through the per-message counter."""
+    _env(monkeypatch, DDT_SELF_VIA_WINDOW="1", DDT_NO_LL="1")
+    p = Plan(ddt, (200, 200, 200), ALL_DIRS, 1, "p2p", dst_off=dst_off)
+    _run(p, 3, f"multi-wave flags dst_off={dst_off}")
+    p.close()

@@ -1,8 +1,10 @@
-"""Trace one fused P2P exchange (configs[1], self messages through the window
-path) and print the per-phase critical path (diagnostic)."""
+"""Trace one fused P2P exchange (configs[1], or COMB with argument "comb"; self
+messages through the window path, or with XMODE=direct through the pack-free
+P2P_DIRECT protocol) and print the per-phase critical path (diagnostic)."""
 import os
 import sys
-os.environ.setdefault("DDT_SELF_VIA_WINDOW", "1")
+DIRECT = os.environ.get("XMODE") == "direct"
+os.environ.setdefault("DDT_SELF_VIA_DIRECT" if DIRECT else "DDT_SELF_VIA_WINDOW", "1")
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np  # noqa: E402
 import torch  # noqa: E402
@@ -17,7 +19,7 @@ arrs = [torch.zeros(tuple(n + 2 for n in local), dtype=torch.int64, device="cuda
 msgs = halo_messages(0, 1, local, dirs=ALL_DIRS if comb else FACE_DIRS, nvars=nvars)
 sends = [(m["peer"], m["tag"], ddt.Type.from_spec(m["send_spec"]), arrs[m["var"]], 1) for m in msgs]
 recvs = [(m["recv_peer"], m["recv_tag"], ddt.Type.from_spec(m["recv_spec"]), arrs[m["var"]], 1) for m in msgs]
-h = ddt.Halo(ddt.Queue(), ddt.Comm.single(0), sends, recvs, mode="p2p", graph=False)
+h = ddt.Halo(ddt.Queue(), ddt.Comm.single(0), sends, recvs, mode="p2p_direct" if DIRECT else "p2p", graph=False)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 for _ in range(5):
     h.exchange()
@@ -30,10 +32,9 @@ for it in range(3):
     r = read()
     t = r["t0"].min()
     ph = {k: (r[k] - t) / 1e3 for k in ("t0", "t1", "t2", "t3")}
-    pack = r["op"] == 0
-    unp = r["op"] == 1
     print(f"iter {it}: records {len(r)}  span {ph['t3'].max():.2f} us  CTAs {len(set(r['cta'].tolist()))}")
-    for name, m in (("pack", pack), ("unpack", unp)):
+    for name, m in (("pack", r["op"] == 0), ("unpack", r["op"] == 1), ("direct", r["op"] == 2),
+                    ("signal", r["op"] == 3)):
         if m.any():
             print(f"  {name:6s} start [{ph['t0'][m].min():.2f}, {ph['t0'][m].max():.2f}]  wait-done max {ph['t1'][m].max():.2f}"
                   f"  data-done [{ph['t2'][m].min():.2f}, {ph['t2'][m].max():.2f}]  signal-done max {ph['t3'][m].max():.2f}"

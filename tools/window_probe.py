@@ -28,6 +28,9 @@ VARIANTS = {
     "direct_dense4": {"DDT_SPREAD_DENSE_UB": "4"},
     "direct_dense2": {"DDT_SPREAD_DENSE_UB": "2"},
     "window": {"DDT_SELF_VIA_WINDOW": "1"},
+    "pdirect": {"DDT_SELF_VIA_DIRECT": "1", "_mode": "p2p_direct"},
+    "pdirect_sys": {"DDT_SELF_VIA_DIRECT": "1", "DDT_FORCE_SYS_SCOPE": "1", "_mode": "p2p_direct"},
+    "window_sys": {"DDT_SELF_VIA_WINDOW": "1", "DDT_FORCE_SYS_SCOPE": "1"},
     "window_xgrid1": {"DDT_SELF_VIA_WINDOW": "1", "DDT_XGRID_MODE": "1"},
     "window_xgrid2": {"DDT_SELF_VIA_WINDOW": "1", "DDT_XGRID_MODE": "2"},
     "window_claim1": {"DDT_SELF_VIA_WINDOW": "1", "DDT_XGRID_MODE": "1", "DDT_XCLAIM": "1"},
@@ -46,16 +49,18 @@ def build(cfg, names):
     wls = {}
     base_env = dict(os.environ)
     for n in names:
-        for k in ("DDT_SELF_VIA_WINDOW", "DDT_XGRID_MODE", "DDT_XCLAIM", "DDT_NO_LL", "DDT_NO_PAIR", "DDT_SPREAD_UB", "DDT_SPREAD_DENSE_UB", "DDT_XUB_LL", "DDT_NO_XPAIR", "DDT_GRID_MODE", "DDT_SPREAD", "DDT_XONCE_G", "DDT_XUB_SMALL"):
+        for k in ("DDT_SELF_VIA_WINDOW", "DDT_XGRID_MODE", "DDT_XCLAIM", "DDT_NO_LL", "DDT_NO_PAIR", "DDT_SPREAD_UB", "DDT_SPREAD_DENSE_UB", "DDT_XUB_LL", "DDT_NO_XPAIR", "DDT_GRID_MODE", "DDT_SPREAD", "DDT_XONCE_G", "DDT_XUB_SMALL", "DDT_SELF_VIA_DIRECT", "DDT_FORCE_SYS_SCOPE"):
             os.environ.pop(k, None)
-        os.environ.update(VARIANTS[n])
+        env = dict(VARIANTS[n])
+        mode = env.pop("_mode", "p2p")
+        os.environ.update(env)
         ddt.reload_env()
         c = ddt.Comm.single(0)
         if cfg == "cfg1":
-            wls[n] = bench.HaloWorkload(ddt, torch, 0, 1, (128, 128, 128), FACE_DIRS, 1, "p2p", c, 2,
+            wls[n] = bench.HaloWorkload(ddt, torch, 0, 1, (128, 128, 128), FACE_DIRS, 1, mode, c, 2,
                                         replicas=int(os.environ.get("R", "96")), graph=False)
         else:
-            wls[n] = bench.HaloWorkload(ddt, torch, 0, 1, (512, 512, 512), ALL_DIRS, 4, "p2p", c, 4, replicas=1,
+            wls[n] = bench.HaloWorkload(ddt, torch, 0, 1, (512, 512, 512), ALL_DIRS, 4, mode, c, 4, replicas=1,
                                         graph=False)
     os.environ.clear()
     os.environ.update(base_env)
