@@ -223,6 +223,11 @@ def _spawn(target, world, extra, timeout=400):
     # exchange pairs (+x / -x packs and unpacks in one item) between real processes
     (2, dict(dirs="all", local=(12, 20, 24), iters=3, env={"DDT_XPAIR_ALWAYS": "1"})),
     (8, dict(dirs="all", local=(6, 10, 12), iters=2, env={"DDT_XPAIR_ALWAYS": "1", "DDT_NO_LL": "1"})),
+    # resident grid claiming chunks (the multi-wave launch form) with per-chunk flags, whole-message
+    # counters and the pack-free protocol: every message keeps its own item size (xub_for)
+    (2, dict(dirs="all", local=(24, 40, 48), iters=3, mode="p2p_direct", env={"DDT_XGRID_MODE": "1"})),
+    (2, dict(dirs="all", local=(24, 40, 48), iters=3, mode="p2p_direct", mis=True, env={"DDT_XGRID_MODE": "1"})),
+    (2, dict(dirs="all", local=(24, 40, 48), iters=3, mis=True, env={"DDT_XGRID_MODE": "1", "DDT_NO_LL": "1"})),
 ])
 def test_exchange_protocols_multiprocess(world, opts):
     res = _spawn(_worker_bytes, world, (opts,))
