@@ -621,6 +621,11 @@ def main():
               "l2": ("inputs larger than L2: steps rotate over R independent arrays + plans (R x ~4 MB > 2x "
                      "the 126 MB L2), and L2 is evicted by a read sweep right before the timed steps, so no "
                      "timed step finds its data in L2 at any K")}
+    # the same config dict in both arms (the driver compares them); run details of
+    # this arm go to the line's "run" key
+    R = int(os.environ.get("DDT_BENCH_REPLICAS", "96"))
+    config.update(replicas=R, distinct_replicas_timed=min(args.steps, R))
+    DATA = "synthetic (seeded random 64-bit patterns)"
 
     if args.impl == "reference":
         if rank != 0:
@@ -662,7 +667,9 @@ def main():
         line = {"impl": "reference", "metric": METRIC, "value": round(per, 2), "unit": "us/iter", "n_gpus": N,
                 "steps": len(times), "warmup": args.warmup, "ms_per_step": round(per / 1e3, 4),
                 "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
-                "data": "synthetic (PCG64 random 64-bit patterns)", "config": dict(config, impl="cpu oracle"),
+                "data": DATA, "config": config,
+                "run": {"impl": "cpu oracle (plain C, oracle/), one rank's messages per step; the GPU arm's "
+                                "replica / L2 fields of config describe the workload's timing there"},
                 "cpu_baseline": {"value": round(per, 2), "unit": "us/iter", "cores": thr, "kind": "oracle",
                                  "sample": (f"{len(times)} timed oracle exchanges of one rank's 6 faces (plain C "
                                             f"oracle, messages split over {thr} threads on a {nc}-core host, "
@@ -707,7 +714,6 @@ def main():
     # the P2P exchange kernel keeps its epoch on the device, NCCL mode captures
     # its send/recv), so the K steps are one captured CUDA graph at every N;
     # a mode whose capture fails falls back to host-issued steps (reported)
-    R = int(os.environ.get("DDT_BENCH_REPLICAS", "96"))
 
     # bring the GPU to its steady clocks before the first timed mode (the first
     # mode measured otherwise pays the ramp: nccl 2.76 vs p2p 2.35 us/iter at
@@ -873,12 +879,12 @@ def main():
             "metric": METRIC, "value": round(best["mean_ms"] * 1e3, 3), "unit": "us/iter", "n_gpus": N,
             "steps": K, "warmup": args.warmup, "ms_per_step": round(best["mean_ms"], 5),
             "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "u8",
-            "data": "synthetic (seeded random int64 bit patterns)",
-            "config": dict(config, mode=best_mode, replicas=R, distinct_replicas_timed=min(K, R),
-                           launch=("K-step CUDA graph (captured time-step loop)" if best["capture"]
-                                   else "host-issued, one ddt_exchange per step"),
-                           l2_evict=("256 MiB read sweep enqueued before the start event (L2 holds none of the "
-                                     "timed steps' data, no dirty lines to write back)")),
+            "data": DATA, "config": config,
+            "run": {"mode": best_mode,
+                    "launch": ("K-step CUDA graph (captured time-step loop)" if best["capture"]
+                               else "host-issued, one ddt_exchange per step"),
+                    "l2_evict": ("256 MiB read sweep enqueued before the start event (L2 holds none of the "
+                                 "timed steps' data, no dirty lines to write back)")},
             "e2e": {"value": round(e2e_ms * 1e3, 2), "unit": "us/iter", "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": d2h, "breakdown": e2e_bd,
                     "device_resident_us": round(best["mean_ms"] * 1e3, 3),

@@ -32,7 +32,18 @@ def test_bench_n1():
     r = subprocess.run([sys.executable, "bench.py", "--steps", "30", "--warmup", "3", "--no-extras"], cwd=ROOT,
                        capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stderr[-3000:]
-    _check(_line(r.stdout), 1)
+    d = _line(r.stdout)
+    _check(d, 1)
+    # the reference arm (CPU oracle) prints the same metric / unit / direction / config
+    r2 = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--steps", "3", "--warmup", "1"],
+                        cwd=ROOT, capture_output=True, text=True, timeout=600)
+    assert r2.returncode == 0, r2.stderr[-3000:]
+    ref = _line(r2.stdout)
+    assert ref["impl"] == "reference"
+    for k in ("metric", "unit", "higher_is_better", "data"):
+        assert ref[k] == d[k], k
+    assert ref["config"] == dict(d["config"], distinct_replicas_timed=min(3, d["config"]["replicas"])), \
+        (ref["config"], d["config"])
 
 
 @pytest.mark.parametrize("mode,port", [("p2p", 29533), ("p2p_direct", 29534)])
@@ -47,5 +58,5 @@ def test_bench_n2_shared_gpu(mode, port):
     assert r.returncode == 0, (r.stdout[-2000:], r.stderr[-3000:])
     d = _line(r.stdout)
     _check(d, 2)
-    assert d["config"]["mode"] == mode
-    assert d["config"]["launch"].startswith("K-step CUDA graph"), d["config"]["launch"]
+    assert d["run"]["mode"] == mode
+    assert d["run"]["launch"].startswith("K-step CUDA graph"), d["run"]["launch"]
