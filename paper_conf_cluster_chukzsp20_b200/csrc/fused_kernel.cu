@@ -58,6 +58,12 @@
 #ifndef DDT_V7_MINB
 #define DDT_V7_MINB 4
 #endif
+#ifndef DDT_V9_MINB
+#define DDT_V9_MINB DDT_V7_MINB
+#endif
+#ifndef DDT_DIAG_TRACE
+#define DDT_DIAG_TRACE 0
+#endif
 
 namespace ddt {
 
@@ -78,6 +84,16 @@ __device__ __forceinline__ uint32_t divu(uint32_t n, const DivU32& d) {
         if (H) asm volatile("ld.global." NCQ ".L2::64B" V : __VA_ARGS__);                        \
         else asm volatile("ld.global." NCQ V : __VA_ARGS__);                                      \
     } while (0)
+// Loads that follow griddepcontrol.wait read data the preceding grid may have
+// written, i.e. data that is NOT read-only for this kernel's lifetime (its
+// lifetime overlaps the predecessor's under PDL), so they use the coherent
+// path: ptxas keeps ld.global.cg after the wait (SASS ACQBULK ... LDG.STRONG),
+// while it may hoist an ld.global.nc above it (observed: tools/cfg1_lab.cu,
+// LDG.E.CONSTANT scheduled before ACQBULK).  Later items' loads keep .nc.
+#ifndef DDT_PDL_NC
+#define DDT_PDL_NC 0
+#endif
+constexpr bool kPdlNc = DDT_PDL_NC != 0;
 template <bool NC, int LW>
 __device__ __forceinline__ uint4 ld_vec(const uint8_t* p, int lw_rt, bool h64 = false) {
     const int lw = LW >= 0 ? LW : lw_rt;  // compile-time width folds the switch
@@ -116,6 +132,15 @@ __device__ __forceinline__ uint4 ld_vec(const uint8_t* p, int lw_rt, bool h64 = 
     return r;
 }
 #undef DDT_LD
+
+// A weak (coherent, L1-allocating) 4-B load: ordered after griddepcontrol.wait
+// like .cg, but later loads of the same sector hit L1.
+__device__ __forceinline__ uint32_t ld_u32_weak(const uint8_t* p, bool h64) {
+    uint32_t r;
+    if (h64) asm volatile("ld.global.L2::64B.u32 %0, [%1];" : "=r"(r) : "l"(p));
+    else asm volatile("ld.global.u32 %0, [%1];" : "=r"(r) : "l"(p));
+    return r;
+}
 
 template <int LW>
 __device__ __forceinline__ void st_vec(uint8_t* p, int lw_rt, const uint4& r) {
@@ -199,6 +224,22 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
     return t;
 }
+
+#if DDT_DIAG_TRACE
+// diagnostic builds (-DDDT_DIAG_TRACE=1): per-CTA {launch tag, start, after the
+// PDL wait (0: not recorded), end} globaltimer records of the parameter-batch
+// kernels (tools/diag_cfg1.py)
+struct DiagRec { unsigned long long t0, t1, t2; unsigned int cta, tag; };
+__device__ DiagRec g_diag[1 << 20];
+__device__ unsigned int g_diag_n;
+__device__ __forceinline__ void diag_rec(unsigned long long t0, unsigned long long t1, unsigned int tag) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        const unsigned int i = atomicAdd(&g_diag_n, 1u);
+        if (i < (1u << 20)) g_diag[i] = DiagRec{t0, t1, globaltimer_ns(), blockIdx.x, tag};
+    }
+}
+#endif
 
 // LL receive: spin until both halves of the 16-B word carry this epoch.
 __device__ __forceinline__ uint4 ll_load(const uint8_t* p, uint32_t epoch, const XArgs* xa) {
@@ -374,9 +415,9 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
 #pragma unroll
                 for (int u = 0; u < UNR; u++) {
                     const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-                    if (u < ub && v < nvec) {
-                        if (wd[u]) buf[u] = coh ? ld_vec<false, 4>(ps[u], 4) : ld_vec<true, 4>(ps[u], 4);
-                        else buf[u] = coh ? ld_vec<false, 3>(ps[u], 3) : ld_vec<true, 3>(ps[u], 3);
+                    if (u < ub && v < nvec) {  // kPdlNc: see ld_vec
+                        if (wd[u]) buf[u] = (coh || !kPdlNc) ? ld_vec<false, 4>(ps[u], 4) : ld_vec<true, 4>(ps[u], 4);
+                        else buf[u] = (coh || !kPdlNc) ? ld_vec<false, 3>(ps[u], 3) : ld_vec<true, 3>(ps[u], 3);
                     }
                 }
             } else {
@@ -447,7 +488,8 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
 #pragma unroll
         for (int u = 0; u < UNR; u++) {
             const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-            if (u < ub && v < nvec) buf[u] = coh ? ld_vec<false, LW>(ps[u], lw, h64) : ld_vec<true, LW>(ps[u], lw, h64);
+            if (u < ub && v < nvec)
+                buf[u] = (coh || !kPdlNc) ? ld_vec<false, LW>(ps[u], lw, h64) : ld_vec<true, LW>(ps[u], lw, h64);
         }
     } else {
 #pragma unroll
@@ -512,7 +554,9 @@ __device__ __forceinline__ void run_seg(const ReqDesc& S, const ReqDesc& D, uint
             const uint8_t* p = src + (s_list ? loff[u] : (int64_t)sg * vps * 4);
 #pragma unroll
             for (int c = 0; c < 4; c++)
-                if (c < (int)vps) w[u][c] = ld_vec<true, 2>(p + 4 * c, 2, h64).x;
+                if (c < (int)vps)  // after the PDL wait: weak L1-allocating loads (the segment's
+                                   // later words hit L1; .cg would send each word to L2)
+                    w[u][c] = (pdlw && !kPdlNc) ? ld_u32_weak(p + 4 * c, h64) : ld_vec<true, 2>(p + 4 * c, 2, h64).x;
         }
     }
 #pragma unroll
@@ -553,9 +597,12 @@ __device__ __forceinline__ void run_pair(const ReqDesc& SA, const ReqDesc& DA, c
                 if (pdlw) {
                     pdl_wait();
                     pdlw = false;
+                    a[k] = kPdlNc ? ld_vec<true, LW>(pa, lw, ha) : ld_vec<false, LW>(pa, lw, ha);
+                    b[k] = kPdlNc ? ld_vec<true, LW>(pb, lw, hb) : ld_vec<false, LW>(pb, lw, hb);
+                } else {
+                    a[k] = ld_vec<true, LW>(pa, lw, ha);
+                    b[k] = ld_vec<true, LW>(pb, lw, hb);
                 }
-                a[k] = ld_vec<true, LW>(pa, lw, ha);
-                b[k] = ld_vec<true, LW>(pb, lw, hb);
             }
         }
         uint8_t* da = reinterpret_cast<uint8_t*>(DA.ptr);
@@ -1055,7 +1102,7 @@ template <int V0> struct VarT {
     // almost every item and needs the extra CTAs to keep loads in flight
     // (tools/pack_probe.py: 1 MiB x 1024 packs 4.74 -> 6.08 TB/s from 3 to 5
     // CTAs/SM); exchange kernels (flags, tracing) keep their registers.
-    static constexpr int MINB = (V == 7 || V == 9) ? DDT_V7_MINB : ((V == 8 || V == 10) ? DDT_V8_MINB : DDT_MINB);
+    static constexpr int MINB = V == 9 ? DDT_V9_MINB : V == 7 ? DDT_V7_MINB : ((V == 8 || V == 10) ? DDT_V8_MINB : DDT_MINB);
     // paired requests (device-table spread plans): the one-slot variants only
     // (batch.cpp kPairVariants), so the register budget of the others is untouched
     static constexpr bool PAIR = V == 9 || V == 7 || V == 4;
@@ -1080,13 +1127,20 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_dev(const u
 
 template <int CAP, int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const __grid_constant__ ParamBatch<CAP> pb) {
+#if DDT_DIAG_TRACE
+    const unsigned long long dt0 = globaltimer_ns();
+#endif
     pdl_trigger();
     // parameter batches run pairs in the one-slot instance only (one-wave plans
     // pair on request, halo.cpp DDT_PAIR1; carrying the branch also measured
     // faster for the unpaired configs[1] step: 2.08 -> 1.99 us)
     fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_PARAM, VarT<V>::UNR, true,
                VarT<V>::SEG, V == 9>(view_of(pb), nullptr);
+#if DDT_DIAG_TRACE
+    diag_rec(dt0, 0ull, (unsigned int)(uintptr_t)pb.descs[0].ptr);
+#endif
 }
+
 
 template <int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
@@ -1242,3 +1296,18 @@ int launch_exchange_form(int form, int variant, const void* src, uint32_t total_
 }  // namespace ddt
 
 extern "C" int32_t ddt_built_sm(void) { return 100; }
+
+#if DDT_DIAG_TRACE
+// diagnostic builds: copy out (and reset) the per-CTA records; returns the count
+extern "C" int32_t ddt_diag_trace(void* out, int32_t max) {
+    unsigned int n = 0;
+    cudaDeviceSynchronize();
+    cudaMemcpyFromSymbol(&n, ddt::g_diag_n, sizeof(n));
+    if (n > (1u << 20)) n = 1u << 20;
+    if ((int32_t)n > max) n = (unsigned int)max;
+    if (out && n) cudaMemcpyFromSymbol(out, ddt::g_diag, n * sizeof(ddt::DiagRec));
+    unsigned int z = 0;
+    cudaMemcpyToSymbol(ddt::g_diag_n, &z, sizeof(z));
+    return (int32_t)n;
+}
+#endif
