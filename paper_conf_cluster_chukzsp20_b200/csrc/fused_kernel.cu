@@ -94,6 +94,12 @@ __device__ __forceinline__ uint32_t divu(uint32_t n, const DivU32& d) {
 #define DDT_PDL_NC 0
 #endif
 constexpr bool kPdlNc = DDT_PDL_NC != 0;
+// Exchange kernels wait (griddepcontrol.wait, flags, LL words) before their
+// items' loads as well: every load of theirs is coherent.
+#ifndef DDT_XCHG_NC
+#define DDT_XCHG_NC 0
+#endif
+constexpr bool kXchgNc = DDT_XCHG_NC != 0;
 template <bool NC, int LW>
 __device__ __forceinline__ uint4 ld_vec(const uint8_t* p, int lw_rt, bool h64 = false) {
     const int lw = LW >= 0 ? LW : lw_rt;  // compile-time width folds the switch
@@ -631,7 +637,7 @@ __device__ __forceinline__ void run_pair_x(const ReqDesc& SA, const ReqDesc& DA,
                                            uint32_t epoch) {
     const int lw = LW >= 0 ? LW : SA.lw;
     const uint32_t nvec = SA.nvec;
-    const bool coh = SA.op == OP_UNPACK;
+    const bool coh = SA.op == OP_UNPACK || !kXchgNc;
     for (int u = 0; u < ub; u++) {
         const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
         if (v >= nvec) break;
@@ -641,8 +647,8 @@ __device__ __forceinline__ void run_pair_x(const ReqDesc& SA, const ReqDesc& DA,
         if (SA.kind == K_LL) {
             ll_load2(pa, pb, epoch, xa, a, b);  // one polling loop for both words
         } else if (coh) {
-            a = ld_vec<false, LW>(pa, lw);
-            b = ld_vec<false, LW>(pb, lw);
+            a = ld_vec<false, LW>(pa, lw, SA.l2_64 != 0);
+            b = ld_vec<false, LW>(pb, lw, SB.l2_64 != 0);
         } else {
             a = ld_vec<true, LW>(pa, lw, SA.l2_64 != 0);
             b = ld_vec<true, LW>(pb, lw, SB.l2_64 != 0);
@@ -967,7 +973,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         } else if (XCHG && PAIR && S->pair) {
             if (run) run_pair_x<LW, SONLY>(sd, sa, sd2, sa2, v0, ubr, xa, (uint32_t)epoch);
         } else {
-            if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, ubr, xa,
+            if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && (S->op == OP_UNPACK || !kXchgNc), ubr, xa,
                                                               (uint32_t)epoch, !waited);
         }
         waited = true;
