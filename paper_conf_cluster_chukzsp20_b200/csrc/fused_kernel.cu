@@ -27,6 +27,7 @@
 // ...): NaN payloads and -0.0 survive bit-exactly.  Small batches arrive in the
 // kernel parameters (ParamBatch), large ones as a device table.
 #include <cuda_runtime.h>
+#include <stddef.h>
 #include <stdint.h>
 
 #include "device_desc.h"
@@ -61,6 +62,9 @@
 #ifndef DDT_V9_MINB
 #define DDT_V9_MINB DDT_V7_MINB
 #endif
+#ifndef DDT_V9DEV_MINB
+#define DDT_V9DEV_MINB DDT_V9_MINB
+#endif
 #ifndef DDT_DIAG_TRACE
 #define DDT_DIAG_TRACE 0
 #endif
@@ -84,22 +88,23 @@ __device__ __forceinline__ uint32_t divu(uint32_t n, const DivU32& d) {
         if (H) asm volatile("ld.global." NCQ ".L2::64B" V : __VA_ARGS__);                        \
         else asm volatile("ld.global." NCQ V : __VA_ARGS__);                                      \
     } while (0)
-// Loads that follow griddepcontrol.wait read data the preceding grid may have
-// written, i.e. data that is NOT read-only for this kernel's lifetime (its
-// lifetime overlaps the predecessor's under PDL), so they use the coherent
-// path: ptxas keeps ld.global.cg after the wait (SASS ACQBULK ... LDG.STRONG),
-// while it may hoist an ld.global.nc above it (observed: tools/cfg1_lab.cu,
-// LDG.E.CONSTANT scheduled before ACQBULK).  Later items' loads keep .nc.
-#ifndef DDT_PDL_NC
-#define DDT_PDL_NC 0
+// Data loads are coherent (ld.global.cg: L2, strong gpu-scope in SASS), not
+// the non-coherent read-only path (ld.global.nc.L1::no_allocate), for two
+// reasons measured / observed on B200:
+//  * ordering: a load that follows griddepcontrol.wait reads data the
+//    preceding grid may have written -- data that is NOT read-only for this
+//    kernel's lifetime, which under PDL overlaps the predecessor's.  ptxas
+//    keeps ld.global.cg after the wait (ACQBULK), but may schedule an
+//    ld.global.nc above it (observed: tools/cfg1_lab.cu, LDG.E.CONSTANT before
+//    ACQBULK) -- a stale read;
+//  * speed: scattered 8-B cells and dense rows alike move faster through the
+//    coherent path -- configs[1] step 2.0 -> 1.78 us, COMB P = 1 87.5 -> 75.9 us
+//    (x faces alone 78.3 -> 56.0 us), dense 1 MiB packs 6.04 -> 6.19 TB/s.
+// DDT_NC_LOADS=1 (build macro, experiments) restores the .nc loads.
+#ifndef DDT_NC_LOADS
+#define DDT_NC_LOADS 0
 #endif
-constexpr bool kPdlNc = DDT_PDL_NC != 0;
-// Exchange kernels wait (griddepcontrol.wait, flags, LL words) before their
-// items' loads as well: every load of theirs is coherent.
-#ifndef DDT_XCHG_NC
-#define DDT_XCHG_NC 0
-#endif
-constexpr bool kXchgNc = DDT_XCHG_NC != 0;
+constexpr bool kNcLoads = DDT_NC_LOADS != 0;
 template <bool NC, int LW>
 __device__ __forceinline__ uint4 ld_vec(const uint8_t* p, int lw_rt, bool h64 = false) {
     const int lw = LW >= 0 ? LW : lw_rt;  // compile-time width folds the switch
@@ -421,9 +426,9 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
 #pragma unroll
                 for (int u = 0; u < UNR; u++) {
                     const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
-                    if (u < ub && v < nvec) {  // kPdlNc: see ld_vec
-                        if (wd[u]) buf[u] = (coh || !kPdlNc) ? ld_vec<false, 4>(ps[u], 4) : ld_vec<true, 4>(ps[u], 4);
-                        else buf[u] = (coh || !kPdlNc) ? ld_vec<false, 3>(ps[u], 3) : ld_vec<true, 3>(ps[u], 3);
+                    if (u < ub && v < nvec) {
+                        if (wd[u]) buf[u] = coh ? ld_vec<false, 4>(ps[u], 4) : ld_vec<kNcLoads, 4>(ps[u], 4);
+                        else buf[u] = coh ? ld_vec<false, 3>(ps[u], 3) : ld_vec<kNcLoads, 3>(ps[u], 3);
                     }
                 }
             } else {
@@ -435,8 +440,8 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
                         bool wide;
                         phased_unit(S, v, s, within, wide);
                         const uint8_t* p = src + seg_offset(S, s) + within;
-                        if (wide) buf[u] = coh ? ld_vec<false, 4>(p, 4) : ld_vec<true, 4>(p, 4);
-                        else buf[u] = coh ? ld_vec<false, 3>(p, 3) : ld_vec<true, 3>(p, 3);
+                        if (wide) buf[u] = coh ? ld_vec<false, 4>(p, 4) : ld_vec<kNcLoads, 4>(p, 4);
+                        else buf[u] = coh ? ld_vec<false, 3>(p, 3) : ld_vec<kNcLoads, 3>(p, 3);
                     }
                 }
             }
@@ -495,7 +500,7 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
         for (int u = 0; u < UNR; u++) {
             const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
             if (u < ub && v < nvec)
-                buf[u] = (coh || !kPdlNc) ? ld_vec<false, LW>(ps[u], lw, h64) : ld_vec<true, LW>(ps[u], lw, h64);
+                buf[u] = coh ? ld_vec<false, LW>(ps[u], lw, h64) : ld_vec<kNcLoads, LW>(ps[u], lw, h64);
         }
     } else {
 #pragma unroll
@@ -505,7 +510,7 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
                 const uint8_t* p =
                     src + (win_s ? gen_offset_win(S, v, *win, pre0, cnt, lw) : vec_offset<LW, SONLY>(S, v));
                 if (XC && S.kind == K_LL) buf[u] = ll_load(p, epoch, xa);
-                else buf[u] = coh ? ld_vec<false, LW>(p, lw, h64) : ld_vec<true, LW>(p, lw, h64);
+                else buf[u] = coh ? ld_vec<false, LW>(p, lw, h64) : ld_vec<kNcLoads, LW>(p, lw, h64);
             }
         }
     }
@@ -560,9 +565,9 @@ __device__ __forceinline__ void run_seg(const ReqDesc& S, const ReqDesc& D, uint
             const uint8_t* p = src + (s_list ? loff[u] : (int64_t)sg * vps * 4);
 #pragma unroll
             for (int c = 0; c < 4; c++)
-                if (c < (int)vps)  // after the PDL wait: weak L1-allocating loads (the segment's
-                                   // later words hit L1; .cg would send each word to L2)
-                    w[u][c] = (pdlw && !kPdlNc) ? ld_u32_weak(p + 4 * c, h64) : ld_vec<true, 2>(p + 4 * c, 2, h64).x;
+                if (c < (int)vps)  // weak L1-allocating loads: the segment's later words hit
+                                   // L1 (.cg would send each word to L2: configs[2] 44 -> 50 us, weak 46)
+                    w[u][c] = kNcLoads ? ld_vec<true, 2>(p + 4 * c, 2, h64).x : ld_u32_weak(p + 4 * c, h64);
         }
     }
 #pragma unroll
@@ -603,12 +608,9 @@ __device__ __forceinline__ void run_pair(const ReqDesc& SA, const ReqDesc& DA, c
                 if (pdlw) {
                     pdl_wait();
                     pdlw = false;
-                    a[k] = kPdlNc ? ld_vec<true, LW>(pa, lw, ha) : ld_vec<false, LW>(pa, lw, ha);
-                    b[k] = kPdlNc ? ld_vec<true, LW>(pb, lw, hb) : ld_vec<false, LW>(pb, lw, hb);
-                } else {
-                    a[k] = ld_vec<true, LW>(pa, lw, ha);
-                    b[k] = ld_vec<true, LW>(pb, lw, hb);
                 }
+                a[k] = ld_vec<kNcLoads, LW>(pa, lw, ha);
+                b[k] = ld_vec<kNcLoads, LW>(pb, lw, hb);
             }
         }
         uint8_t* da = reinterpret_cast<uint8_t*>(DA.ptr);
@@ -637,7 +639,7 @@ __device__ __forceinline__ void run_pair_x(const ReqDesc& SA, const ReqDesc& DA,
                                            uint32_t epoch) {
     const int lw = LW >= 0 ? LW : SA.lw;
     const uint32_t nvec = SA.nvec;
-    const bool coh = SA.op == OP_UNPACK || !kXchgNc;
+    const bool coh = SA.op == OP_UNPACK || !kNcLoads;
     for (int u = 0; u < ub; u++) {
         const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
         if (v >= nvec) break;
@@ -650,8 +652,8 @@ __device__ __forceinline__ void run_pair_x(const ReqDesc& SA, const ReqDesc& DA,
             a = ld_vec<false, LW>(pa, lw, SA.l2_64 != 0);
             b = ld_vec<false, LW>(pb, lw, SB.l2_64 != 0);
         } else {
-            a = ld_vec<true, LW>(pa, lw, SA.l2_64 != 0);
-            b = ld_vec<true, LW>(pb, lw, SB.l2_64 != 0);
+            a = ld_vec<kNcLoads, LW>(pa, lw, SA.l2_64 != 0);
+            b = ld_vec<kNcLoads, LW>(pb, lw, SB.l2_64 != 0);
         }
         uint8_t* qa = reinterpret_cast<uint8_t*>(DA.ptr) + vec_offset<LW, SONLY>(DA, v);
         uint8_t* qb = reinterpret_cast<uint8_t*>(DB.ptr) + vec_offset<LW, SONLY>(DB, v);
@@ -666,11 +668,12 @@ __device__ __forceinline__ void run_pair_x(const ReqDesc& SA, const ReqDesc& DA,
 }
 
 // Largest r with prefix[r] <= item (prefix strictly increasing, prefix[0] = 0).
+__device__ __forceinline__ uint32_t tbl_u32(const uint32_t* p);
 __device__ __forceinline__ uint32_t find_request(const uint32_t* prefix, uint32_t nreq, uint32_t item) {
     uint32_t lo = 0, hi = nreq;
     while (hi - lo > 1) {
         uint32_t mid = (lo + hi) >> 1;
-        if (prefix[mid] <= item) lo = mid;
+        if (tbl_u32(prefix + mid) <= item) lo = mid;
         else hi = mid;
     }
     return lo;
@@ -723,9 +726,46 @@ __device__ __forceinline__ TableView view_of(const ParamBatch<CAP>& p) {
     return v;
 }
 
+// Device-table entries (prefix, item order, descriptors) are read by every CTA
+// of a launch while the launch's data streams through L2; they are loaded with
+// an L2 evict_last policy so that they stay resident instead of costing each
+// CTA's prologue DRAM round trips (COMB: 104 requests, ~200 MB of data per
+// launch).  Weak loads, not .nc: a flushed batch's table is copied right before
+// the launch, behind the PDL wait.  Parameter batches (param space) load plainly.
+#ifndef DDT_TABLE_KEEP
+#define DDT_TABLE_KEEP 1
+#endif
+__device__ __forceinline__ uint64_t l2_keep_policy() {
+    uint64_t pol;
+    asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+    return pol;
+}
+__device__ __forceinline__ uint32_t tbl_u32(const uint32_t* p) {
+    if (DDT_TABLE_KEEP && __isGlobal(p)) {
+        uint32_t r;
+        asm volatile("ld.global.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(r) : "l"(p), "l"(l2_keep_policy()));
+        return r;
+    }
+    return *p;
+}
 __device__ __forceinline__ void copy_words(void* dst, const void* src, int words, int tid0) {
     int t = (int)threadIdx.x - tid0;
-    if (t >= 0 && t < words) reinterpret_cast<uint4*>(dst)[t] = reinterpret_cast<const uint4*>(src)[t];
+    if (t >= 0 && t < words) {
+        const uint4* q = reinterpret_cast<const uint4*>(src) + t;
+        uint4 r;
+        if (DDT_TABLE_KEEP && __isGlobal(q))
+            asm volatile("ld.global.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+                         : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(q), "l"(l2_keep_policy()));
+        else
+            r = *q;
+        reinterpret_cast<uint4*>(dst)[t] = r;
+    }
+}
+// ReqDesc::pair of descs[r] through the table path
+__device__ __forceinline__ bool desc_pair(const ReqDesc* d) {
+    constexpr size_t off = offsetof(ReqDesc, pair);
+    const uint32_t w = tbl_u32(reinterpret_cast<const uint32_t*>(reinterpret_cast<const uint8_t*>(d) + (off & ~(size_t)3)));
+    return ((w >> (8 * (off & 3))) & 0xffu) != 0;
 }
 
 // ------------------------------------------------------------------------
@@ -866,15 +906,15 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         if (dyn && threadIdx.x == 0) s_tk[par ^ 1] = atomicAdd(tv.ticket, 1u);
         uint32_t r, local;  // the item's request and chunk index within it
         if (tv.order) {     // spread batch: explicit item table
-            const uint32_t e = __ldg(tv.order + item);
+            const uint32_t e = tbl_u32(tv.order + item);
             r = e >> kSpreadShift;
             local = e & ((1u << kSpreadShift) - 1u);
         } else {
             r = find_request(tv.prefix, tv.nreq, item);
-            local = item - tv.prefix[r];
+            local = item - tbl_u32(tv.prefix + r);
         }
         if (!tv.order && (tv.flags & kBatchGrouped)) {  // interleaved group: chunk local / m of member local % m
-            const uint32_t m = tv.gm[r];
+            const uint32_t m = tbl_u32(tv.gm + r);
             if (m > 1) {
                 r = r + 1u - m + local % m;
                 local /= m;
@@ -891,13 +931,13 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
             if constexpr (XCHG) copy_words(&sx, tv.xinfo + r, kXWords, 32);
             copy_words(&sa, tv.aux + r, kWords, 64);  // destination descriptor (aux[r], see HostBatch::add)
             if constexpr (!XCHG && PAIR) {
-                if (tv.descs[r].pair) {  // paired request: its partner r + 1 too (spread table or prefix form)
+                if (desc_pair(tv.descs + r)) {  // paired request: its partner r + 1 too (spread table or prefix form)
                     copy_words(&sd2, tv.descs + r + 1, kWords, 128);
                     copy_words(&sa2, tv.aux + r + 1, kWords, 192);
                 }
             }
             if constexpr (XCHG && PAIR) {
-                if (tv.descs[r].pair) {  // exchange pair: the partner's descriptors and exchange info
+                if (desc_pair(tv.descs + r)) {  // exchange pair: the partner's descriptors and exchange info
                     copy_words(&sd2, tv.descs + r + 1, kWords, 128);
                     copy_words(&sa2, tv.aux + r + 1, kWords, 160);
                     copy_words(&sx2, tv.xinfo + r + 1, kXWords, 192);
@@ -973,7 +1013,7 @@ __device__ __forceinline__ void fused_body(const TableView& tv, const XArgs* xa)
         } else if (XCHG && PAIR && S->pair) {
             if (run) run_pair_x<LW, SONLY>(sd, sa, sd2, sa2, v0, ubr, xa, (uint32_t)epoch);
         } else {
-            if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && (S->op == OP_UNPACK || !kXchgNc), ubr, xa,
+            if (run) run_desc<LW, SONLY, XCHG, GW, PH, UNR>(*S, *D, v0, XCHG && S->op == OP_UNPACK, ubr, xa,
                                                               (uint32_t)epoch, !waited);
         }
         waited = true;
@@ -1109,6 +1149,7 @@ template <int V0> struct VarT {
     // (tools/pack_probe.py: 1 MiB x 1024 packs 4.74 -> 6.08 TB/s from 3 to 5
     // CTAs/SM); exchange kernels (flags, tracing) keep their registers.
     static constexpr int MINB = V == 9 ? DDT_V9_MINB : V == 7 ? DDT_V7_MINB : ((V == 8 || V == 10) ? DDT_V8_MINB : DDT_MINB);
+    static constexpr int DMINB = V == 9 ? DDT_V9DEV_MINB : MINB;  // device-table form
     // paired requests (device-table spread plans): the one-slot variants only
     // (batch.cpp kPairVariants), so the register budget of the others is untouched
     static constexpr bool PAIR = V == 9 || V == 7 || V == 4;
@@ -1124,7 +1165,7 @@ template <int V0> struct VarT {
 };
 
 template <int V>
-__global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_dev(const uint8_t* __restrict__ table) {
+__global__ void __launch_bounds__(kThreads, VarT<V>::DMINB) ddt_fused_dev(const uint8_t* __restrict__ table) {
     pdl_trigger();
     pdl_wait();  // the table may come from a copy just before this launch
     fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_DEV, VarT<V>::UNR, false,
@@ -1175,8 +1216,21 @@ int device_sm_count(int device) {
     return n;
 }
 
+// DDT_CARVEOUT (experiments): cudaFuncAttributePreferredSharedMemoryCarveout
+// for every fused kernel, in percent of the maximum shared memory (-1: unset).
+static int carveout_knob() {
+    static const int c = [] {
+        const char* e = getenv("DDT_CARVEOUT");
+        return e ? atoi(e) : -1;
+    }();
+    return c;
+}
+
 template <class K>
 static int resident_ctas(K kernel) {
+    if (carveout_knob() >= 0)
+        cudaFuncSetAttribute(reinterpret_cast<const void*>(kernel), cudaFuncAttributePreferredSharedMemoryCarveout,
+                             carveout_knob());
     int b = 0;
     if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, kernel, kThreads, 0) != cudaSuccess || b <= 0) b = 1;
     int dev = 0;
