@@ -47,6 +47,9 @@
 #ifndef DDT_PDL_PREFETCH
 #define DDT_PDL_PREFETCH 1
 #endif
+#ifndef DDT_PF_DST
+#define DDT_PF_DST 0  // experiments: also prefetch the first item's destination lines
+#endif
 #ifndef DDT_PREFETCH_MAX_UB
 #define DDT_PREFETCH_MAX_UB 1
 #endif
@@ -420,7 +423,10 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
                     wd[u] = false;
                     if (u < ub && v < nvec) phased_unit(S, v, s, within, wd[u]);
                     ps[u] = src + seg_offset(S, s) + within;
-                    if (DDT_PDL_PREFETCH && ub <= DDT_PREFETCH_MAX_UB && u < ub && v < nvec) prefetch_l2(ps[u]);
+                    if (DDT_PDL_PREFETCH && ub <= DDT_PREFETCH_MAX_UB && u < ub && v < nvec) {
+                        prefetch_l2(ps[u]);
+                        if (DDT_PF_DST) prefetch_l2(dst + seg_offset(D, s) + within);
+                    }
                 }
                 pdl_wait();
 #pragma unroll
@@ -493,7 +499,10 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
             ps[u] = src + ((u < ub && v < nvec) ? (win_s ? gen_offset_win(S, v, *win, pre0, cnt, lw)
                                                          : vec_offset<LW, SONLY>(S, v))
                                                 : 0);
-            if (DDT_PDL_PREFETCH && ub <= DDT_PREFETCH_MAX_UB && u < ub && v < nvec) prefetch_l2(ps[u]);
+            if (DDT_PDL_PREFETCH && ub <= DDT_PREFETCH_MAX_UB && u < ub && v < nvec) {
+                prefetch_l2(ps[u]);
+                if (DDT_PF_DST && !win_d) prefetch_l2(dst + vec_offset<LW, SONLY>(D, v));
+            }
         }
         pdl_wait();
 #pragma unroll
