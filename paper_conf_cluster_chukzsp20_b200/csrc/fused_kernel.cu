@@ -1197,7 +1197,6 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const
 #endif
 }
 
-
 template <int V>
 __global__ void __launch_bounds__(kThreads, VarT<V>::XMINB)
     ddt_exchange_dev(const uint8_t* __restrict__ table, const XArgs xa) {
