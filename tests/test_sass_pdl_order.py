@@ -5,10 +5,11 @@ CTAs start while the preceding kernel still runs and block in
 griddepcontrol.wait (SASS ACQBULK) before touching user data.  ptxas may
 schedule an ld.global.nc load above that wait (observed on
 tools/cfg1_lab.cu: LDG.E.CONSTANT before ACQBULK), so the library's loads that
-follow the wait are coherent ones (fused_kernel.cu kPdlNc).  This test
+follow the wait are coherent ones (fused_kernel.cu kNcLoads).  This test
 disassembles libddt.so and checks, for every parameter-batch instance of the
 closed-form variants (no commit-time list tables that may legally be read
-before the wait), that no global load precedes the first ACQBULK.
+before the wait), that no global load precedes the first ACQBULK and that no
+load at all takes the non-coherent path.
 """
 import os
 import re
@@ -44,5 +45,9 @@ def test_no_data_load_before_the_pdl_wait():
         assert acq, f"{name}: no griddepcontrol.wait"
         early = [x for x in ins[:acq[0]] if re.match(r"(@!?U?P\d+\s+)?LDG", x)]
         assert not early, f"{name}: global loads before the PDL wait: {early[:3]}"
+        # the closed-form variants read no commit-time list table, so no load of theirs may take the
+        # non-coherent path (LDG ... CONSTANT) that ptxas is free to move above the wait
+        nc = [x for x in ins if re.match(r"(@!?U?P\d+\s+)?LDG\S*CONSTANT", x)]
+        assert not nc, f"{name}: non-coherent loads in a PDL kernel: {nc[:3]}"
         checked += 1
     assert checked >= 14, checked  # 7 variants x 2 parameter forms
