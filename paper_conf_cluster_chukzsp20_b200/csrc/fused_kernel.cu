@@ -241,11 +241,16 @@ __device__ __forceinline__ uint64_t globaltimer_ns() {
 
 #if DDT_DIAG_TRACE
 // diagnostic builds (-DDDT_DIAG_TRACE=1): per-CTA {launch tag, start, after the
-// PDL wait (0: not recorded), end} globaltimer records of the parameter-batch
-// kernels (tools/diag_cfg1.py)
+// PDL wait (strided / phased items), end} globaltimer records of the
+// parameter-batch kernels (tools/diag_cfg1.py)
 struct DiagRec { unsigned long long t0, t1, t2; unsigned int cta, tag; };
 __device__ DiagRec g_diag[1 << 20];
 __device__ unsigned int g_diag_n;
+__shared__ unsigned long long g_diag_t1;  // per CTA: thread 0 passed the first griddepcontrol.wait
+#define DDT_DIAG_WAITED() \
+    do {                   \
+        if (threadIdx.x == 0) g_diag_t1 = globaltimer_ns(); \
+    } while (0)
 __device__ __forceinline__ void diag_rec(unsigned long long t0, unsigned long long t1, unsigned int tag) {
     __syncthreads();
     if (threadIdx.x == 0) {
@@ -253,6 +258,10 @@ __device__ __forceinline__ void diag_rec(unsigned long long t0, unsigned long lo
         if (i < (1u << 20)) g_diag[i] = DiagRec{t0, t1, globaltimer_ns(), blockIdx.x, tag};
     }
 }
+#else
+#define DDT_DIAG_WAITED() \
+    do {                   \
+    } while (0)
 #endif
 
 // LL receive: spin until both halves of the 16-B word carry this epoch.
@@ -429,6 +438,7 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
                     }
                 }
                 pdl_wait();
+                DDT_DIAG_WAITED();
 #pragma unroll
                 for (int u = 0; u < UNR; u++) {
                     const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
@@ -505,6 +515,7 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
             }
         }
         pdl_wait();
+        DDT_DIAG_WAITED();
 #pragma unroll
         for (int u = 0; u < UNR; u++) {
             const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
@@ -1193,7 +1204,7 @@ __global__ void __launch_bounds__(kThreads, VarT<V>::MINB) ddt_fused_param(const
     fused_body<false, VarT<V>::LW, VarT<V>::SONLY, VarT<V>::GW, VarT<V>::PH, DDT_INPLACE_PARAM, VarT<V>::UNR, true,
                VarT<V>::SEG, V == 9>(view_of(pb), nullptr);
 #if DDT_DIAG_TRACE
-    diag_rec(dt0, 0ull, (unsigned int)(uintptr_t)pb.descs[0].ptr);
+    diag_rec(dt0, g_diag_t1, (unsigned int)(uintptr_t)pb.descs[0].ptr);
 #endif
 }
 

@@ -84,7 +84,21 @@ def main():
     def med(k):
         v = [x[k] for x in mid if x[k] is not None]
         return statistics.median(v) if v else None
+    # per CTA index (the batch's items in order): median time from passing the wait to the CTA's end
+    mids = launches[len(launches) // 4: 3 * len(launches) // 4]
+    by_cta = {}
+    for q in mids:
+        if not q["t1"].min():
+            continue
+        for rec in q:
+            by_cta.setdefault(int(rec["cta"]), []).append(int(rec["t2"]) - int(rec["t1"]))
+    cta_ns = {c: statistics.median(v) for c, v in sorted(by_cta.items())}
+    buckets = {}
+    for c, v in cta_ns.items():
+        buckets.setdefault(c // 20 * 20, []).append(v)
+    out_b = {f"{b}-{b + 19}": round(statistics.median(v)) for b, v in buckets.items()}
     out = {"lib": os.environ.get("DDT_LIBDDT", ""), "K": K, "us_per_step_events": round(us, 3), "records": int(n),
+           "wait_to_end_ns_by_cta": out_b,
            "launches": len(launches), "median_over_middle_half_ns": {k: med(k) for k in rows[0]},
            "sample": rows[len(rows) // 2: len(rows) // 2 + 5]}
     print(json.dumps(out))
