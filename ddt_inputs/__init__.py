@@ -79,6 +79,21 @@ def milc_spec(L: int = 16):
     return spec, L ** 4 * 48
 
 
+def nas_mg_specs(n1: int = 34, n2: int = 34, n3: int = 34):
+    """NAS_MG-style face types ("vectors (NAS_MG)"; ddtbench's
+    MG kernel): the three boundary faces of an n1 x n2 x n3 grid of doubles, x
+    (extent n1) fastest, each face at its first index (i = 0, j = 0, k = 0):
+      x face: vector(n2*n3, 1, n1)        -- one element per x-row
+      y face: vector(n3, n1, n1*n2)       -- one x-row per plane
+      z face: contiguous(n1*n2)           -- one whole plane
+    Returns ({"x": spec, "y": spec, "z": spec}, footprint_bytes)."""
+    d = ("basic", "double")
+    specs = {"x": ("vector", n2 * n3, 1, n1, d),
+             "y": ("vector", n3, n1, n1 * n2, d),
+             "z": ("contiguous", n1 * n2, d)}
+    return specs, n1 * n2 * n3 * 8
+
+
 # ----------------------------------------------------------------- config 5
 def config5_spec(S: int):
     """BASELINE.json configs[4]: dense vector of doubles, block = min(S, 256 B),

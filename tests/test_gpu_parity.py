@@ -636,6 +636,18 @@ def test_milc_nested_vector(ddt, q, L):
     _run_case(ddt, q, Case(ddt, spec, 2, misalign=8, seed=L + 1))
 
 
+@pytest.mark.parametrize("face", ["x", "y", "z"])
+@pytest.mark.parametrize("n", [(34, 34, 34), (66, 34, 18)])
+def test_nas_mg_vector_faces(ddt, q, face, n):
+    """NAS_MG-style vector faces (x: one element per row, y: one row per plane,
+    z: a whole plane): pack + unpack bit-exact vs the oracle, one instance at an
+    aligned base and two at a misaligned one."""
+    from ddt_inputs import nas_mg_specs
+    specs, _ = nas_mg_specs(*n)
+    _run_case(ddt, q, Case(ddt, specs[face], 1, misalign=0, seed=sum(n)))
+    _run_case(ddt, q, Case(ddt, specs[face], 2, misalign=8, seed=sum(n) + 1))
+
+
 def _irregular_hindexed(nblocks, npoints, base, maxlen, seed_, ones=False):
     """hindexed with irregular block lengths (a GENERAL_LIST layout); ones=True:
     mostly 1-element blocks of bytes (windows overflow -> per-vector fallback)."""

@@ -566,3 +566,18 @@ def test_milc_nested_vector_matches_numpy():
     src = random_bytes(fp, 31)
     lat = src.view(np.float64).reshape(L, L, L, L, 6)          # [t][z][y][x][6]
     np.testing.assert_array_equal(oracle.pack(t, src).view(np.float64), lat[:, :, 0, :, :].reshape(-1))
+
+
+def test_nas_mg_faces_match_numpy():
+    """NAS_MG-style vector faces against numpy slicing of the
+    (n3, n2, n1) C-order grid, x fastest."""
+    from ddt_inputs import nas_mg_specs
+    n1, n2, n3 = 6, 5, 7
+    specs, fp = nas_mg_specs(n1, n2, n3)
+    src = random_bytes(fp, 41)
+    g = src.view(np.float64).reshape(n3, n2, n1)
+    want = {"x": g[:, :, 0], "y": g[:, 0, :], "z": g[0, :, :]}
+    for face, spec in specs.items():
+        t = oracle.Type(spec)
+        np.testing.assert_array_equal(oracle.pack(t, src).view(np.float64), want[face].reshape(-1), err_msg=face)
+        assert t.size == want[face].size * 8
