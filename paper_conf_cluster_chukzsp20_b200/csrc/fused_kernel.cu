@@ -47,6 +47,12 @@
 #ifndef DDT_PDL_PREFETCH
 #define DDT_PDL_PREFETCH 1
 #endif
+#ifndef DDT_DESC_PF_DST
+#define DDT_DESC_PF_DST 0
+#endif
+#ifndef DDT_SEG_PF_DST
+#define DDT_SEG_PF_DST 1
+#endif
 #ifndef DDT_PF_DST
 #define DDT_PF_DST 0  // experiments: also prefetch the first item's destination lines
 #endif
@@ -533,6 +539,15 @@ __device__ __forceinline__ void run_desc(const ReqDesc& S, const ReqDesc& D, uin
                 else buf[u] = coh ? ld_vec<false, LW>(p, lw, h64) : ld_vec<kNcLoads, LW>(p, lw, h64);
             }
         }
+        if (DDT_DESC_PF_DST && D.l2_64 && !win_d && !(XC && D.kind == K_LL)) {
+            // scattered short destination segments: fetch their sectors into L2 while the
+            // loads are in flight (a partial-sector store to an absent line costs a DRAM read)
+#pragma unroll
+            for (int u = 0; u < UNR; u++) {
+                const uint32_t v = v0 + (uint32_t)(u * kThreads) + threadIdx.x;
+                if (u < ub && v < nvec) prefetch_l2(dst + vec_offset<LW, SONLY>(D, v));
+            }
+        }
     }
 #pragma unroll
     for (int u = 0; u < UNR; u++) {
@@ -574,6 +589,17 @@ __device__ __forceinline__ void run_seg(const ReqDesc& S, const ReqDesc& D, uint
             const int64_t o = L.kind == K_UNIFORM32 ? (int64_t)__ldg(reinterpret_cast<const int32_t*>(L.list) + j)
                                                     : (int64_t)__ldg(reinterpret_cast<const long long*>(L.list) + j);
             loff[u] = (int64_t)k * L.extent + o;  // list offsets are relative to the side's pointer
+        }
+    }
+    // unpack into 12-16-B list segments: fetch the destination sectors into L2 now, in
+    // parallel with the packed-side loads -- a partial-sector store to a line L2 does not
+    // hold is completed with a DRAM read later (configs[2] B=16 unpack 64.5 -> 50.2 us);
+    // 4-8-B segments (struct-on-indexed) would only double the requests
+    if (DDT_SEG_PF_DST && !s_list && vps >= 3) {
+#pragma unroll
+        for (int u = 0; u < SR; u++) {
+            const uint32_t sg = s0 + (uint32_t)(u * kThreads) + threadIdx.x;
+            if (u < rounds && sg < nsegs) prefetch_l2(dst + loff[u]);
         }
     }
     if (pdlw) pdl_wait();
