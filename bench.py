@@ -484,6 +484,24 @@ def sparse_roofline(ddt, torch, hbm_peak, flush_buf, reps=20):
     if traffic:
         out["traffic_gbs"] = round(traffic / tmed / 1e9, 1)
         out["traffic_frac"] = round(traffic / tmed / 1e9 / hbm_peak, 3)
+    # the unpack batch of the same layout (packed -> scattered 12-B segments), timed alike
+    back = torch.empty((B, nb), dtype=torch.uint8, device="cuda")
+    q.enqueue_many("unpack", t, list(dst), 1, list(back))
+    uplan = ddt.Plan(q)
+    for _ in range(3):
+        uplan.launch()
+    utimes = []
+    for k in range(reps):
+        l2_evict(torch, flush_buf)
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        uplan.launch()
+        b.record(stream)
+        torch.cuda.synchronize()
+        utimes.append(a.elapsed_time(b) / 1e3)
+    umed = statistics.median(utimes)
+    out["unpack"] = {"us": round(umed * 1e6, 2), "alg_gbs": round(alg / umed / 1e9, 1)}
+    uplan.destroy()
     plan.destroy()
     q.destroy()
     return out
