@@ -48,6 +48,7 @@ def main():
                             replicas=96, graph=False)
     for _ in range(5):
         wl.step()
+    first = wl.k  # the first captured (timed) step's replica
     g = torch.cuda.CUDAGraph()
     with torch.cuda.graph(g, stream=s):
         for _ in range(K):
@@ -59,6 +60,7 @@ def main():
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         torch.cuda.synchronize()
         bench.l2_evict(torch, flush)
+        wl.step_at(first - 1)  # bench.run_steps: the code-warming step on a non-timed replica
         a.record(s)
         g.replay()
         b.record(s)
@@ -67,10 +69,13 @@ def main():
     torch.cuda.synchronize()
     with profile(activities=[ProfilerActivity.CUDA]) as prof:
         bench.l2_evict(torch, flush)
+        wl.step_at(first - 1)
         g.replay()
         torch.cuda.synchronize()
     ks = kernels(prof)
     steps = [k for k in ks if "ddt_" in k[0]]
+    if len(steps) == K + 1:
+        steps = steps[1:]  # the untimed code-warming step before the replay
     other = [k for k in ks if "ddt_" not in k[0]]
     dur = [(e - st) / 1e3 for _, st, e in steps]
     gaps = [(steps[i + 1][1] - steps[i][2]) / 1e3 for i in range(len(steps) - 1)]
