@@ -47,7 +47,8 @@ __global__ void xk(Arr A) {
     const int v = MODE == 4 ? (int)(blockIdx.x % NV) : (int)(t / ROWS);
     const long long r = MODE == 4 ? (long long)(blockIdx.x / NV) * blockDim.x + threadIdx.x : t % ROWS;
     double* a = A.a[v];
-    const long long b = MODE == 2 ? row_base_z(r) : row_base(r);
+    // MODE 5: rows visited in a scattered order (r * 1021 mod ROWS, 1021 prime: a permutation)
+    const long long b = MODE == 2 ? row_base_z(r) : (MODE == 5 ? row_base((r * 1021) % ROWS) : row_base(r));
     if (MODE == 1 && r + D < ROWS) {
         const long long bn = row_base(r + D);
         pf(a + bn); pf(a + bn + 512);
@@ -90,6 +91,7 @@ int main() {
         pr("row_z", timeit([&] { xk<2, 0><<<G, T>>>(A); }, K));
         pr("row_v2", timeit([&] { xk<3, 0><<<G / 2, T>>>(A); }, K));
         pr("row_varrot", timeit([&] { xk<4, 0><<<G, T>>>(A); }, K));
+        pr("row_perm", timeit([&] { xk<5, 0><<<G, T>>>(A); }, K));
         cudaFuncSetAttribute(xk<0, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 110 * 1024);
         cudaFuncSetAttribute(xk<3, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, 110 * 1024);
         pr("row_occ4", timeit([&] { xk<0, 0><<<G, T, 50 * 1024>>>(A); }, K));
