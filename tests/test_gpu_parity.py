@@ -393,6 +393,48 @@ def test_pdl_launches_respect_stream_order(ddt):
     q.destroy()
 
 
+def test_pdl_read_after_write_inside_a_captured_graph(ddt):
+    """Inside ONE captured CUDA graph (programmatic edges between consecutive
+    ddt kernels): 30 rounds of [pack A -> packed buffer] -> [unpack of that
+    buffer into B] -> [pack of B's typemap -> second buffer], each kernel
+    reading what its immediate predecessor wrote, so a load scheduled above
+    griddepcontrol.wait would read the previous round's bytes; torch kernels
+    rewrite the source between rounds.  Every round is checked vs the oracle."""
+    import torch
+    spec = ("vector", 64, 3, 7, ("basic", "double"))
+    o = oracle.Type(spec)
+    t = ddt.Type.from_spec(spec)
+    lo, hi = o.footprint(1)
+    s = torch.cuda.Stream()
+    R = 30
+    with torch.cuda.stream(s):
+        q = ddt.Queue()
+        src = torch.empty(hi, dtype=torch.uint8, device="cuda")
+        pk = torch.empty(o.size, dtype=torch.uint8, device="cuda")
+        mid = torch.empty(hi, dtype=torch.uint8, device="cuda")
+        pk2 = torch.empty((R, o.size), dtype=torch.uint8, device="cuda")
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for k in range(R):
+                src.fill_((11 * k + 5) & 0xFF)
+                src[k: k + 16].fill_(k)
+                mid.fill_(0xA5)
+                q.pack(t, src, 1, pk)
+                q.flush()
+                q.unpack(t, pk, 1, mid)
+                q.flush()
+                q.pack(t, mid, 1, pk2[k])
+                q.flush()
+        g.replay()
+    torch.cuda.synchronize()
+    got = pk2.cpu().numpy()
+    for k in range(R):
+        s_host = np.full(hi, (11 * k + 5) & 0xFF, np.uint8)
+        s_host[k: k + 16] = k
+        assert_bytes_equal(got[k], oracle.pack(o, s_host), f"round {k}")
+    q.destroy()
+
+
 def test_ring_reclaim_with_many_inflight_batches(ddt):
     """A 64-slot ring driven by 300 one-request flushes with no host wait: the
     ring fills repeatedly and enqueue reclaims completed batches (newest-first
