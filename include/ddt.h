@@ -221,7 +221,9 @@ int64_t ddt_direct_enqueue(ddt_queue_t q, ddt_type_t src_type, const void* src, 
 
 /* Scheduler (2): launch every pending request (Head..Tail) as ONE fused
  * kernel on the queue's stream (P:217, P:221, P:255 trigger (1)).  Returns
- * the number of requests launched (0 => nothing pending, no launch) or < 0. */
+ * the number of requests launched (0 => nothing pending, no launch) or < 0.
+ * DDT_ERR_STATE while the queue's stream is being captured into a CUDA graph
+ * (the requests stay pending): graphs capture ddt_plan_launch / ddt_exchange. */
 int32_t ddt_flush(ddt_queue_t q);
 /* Scheduler (4): state of a uid: *state = DDT_PENDING (enqueued, not
  * flushed), DDT_BUSY (flushed, GPU not done), DDT_COMPLETED.  Non-blocking.

@@ -1304,7 +1304,7 @@ static bool pdl_enabled() {
 // Plain fused kernels launch with programmatic stream serialisation (see
 // pdl_trigger / pdl_wait above).
 template <class... Args>
-static void launch_pdl(void (*k)(Args...), uint32_t grid, cudaStream_t s, const Args&... args) {
+static cudaError_t launch_pdl(void (*k)(Args...), uint32_t grid, cudaStream_t s, const Args&... args) {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(grid);
     cfg.blockDim = dim3(kThreads);
@@ -1314,28 +1314,28 @@ static void launch_pdl(void (*k)(Args...), uint32_t grid, cudaStream_t s, const 
     at[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     cfg.numAttrs = pdl_enabled() ? 1 : 0;
-    cudaLaunchKernelEx(&cfg, k, args...);
+    return cudaLaunchKernelEx(&cfg, k, args...);  // this launch's own status (not a stale last error)
 }
 
 template <int V>
-static void launch_fused_v(int form, const void* src, uint32_t total, cudaStream_t s, int grid_cap) {
+static cudaError_t launch_fused_v(int form, const void* src, uint32_t total, cudaStream_t s, int grid_cap) {
     static int res[4] = {0, 0, 0, 0};
     if (form == 1) {
         if (!res[1]) res[1] = resident_ctas(ddt_fused_param<kParamSmall, V>);
-        launch_pdl(ddt_fused_param<kParamSmall, V>, grid_for(total, res[1], grid_cap), s,
+        return launch_pdl(ddt_fused_param<kParamSmall, V>, grid_for(total, res[1], grid_cap), s,
                    *reinterpret_cast<const ParamBatch<kParamSmall>*>(src));
     } else if (form == 2) {
         if (!res[2]) res[2] = resident_ctas(ddt_fused_param<kParamLarge, V>);
-        launch_pdl(ddt_fused_param<kParamLarge, V>, grid_for(total, res[2], grid_cap), s,
+        return launch_pdl(ddt_fused_param<kParamLarge, V>, grid_for(total, res[2], grid_cap), s,
                    *reinterpret_cast<const ParamBatch<kParamLarge>*>(src));
     } else {
         if (!res[3]) res[3] = resident_ctas(ddt_fused_dev<V>);
-        launch_pdl(ddt_fused_dev<V>, grid_for(total, res[3], grid_cap), s, reinterpret_cast<const uint8_t*>(src));
+        return launch_pdl(ddt_fused_dev<V>, grid_for(total, res[3], grid_cap), s, reinterpret_cast<const uint8_t*>(src));
     }
 }
 
 template <int V>
-static void launch_exchange_v(int form, const void* src, uint32_t total, const XArgs& xa, cudaStream_t s,
+static cudaError_t launch_exchange_v(int form, const void* src, uint32_t total, const XArgs& xa, cudaStream_t s,
                               int grid_cap) {
     static int res[4] = {0, 0, 0, 0};
     // programmatic serialisation: the launch overlaps the previous kernel's
@@ -1344,15 +1344,15 @@ static void launch_exchange_v(int form, const void* src, uint32_t total, const X
     // by ticket, so the grid may exceed the resident CTAs)
     if (form == 1) {
         if (!res[1]) res[1] = resident_ctas(ddt_exchange_param<kParamSmall, V>);
-        launch_pdl(ddt_exchange_param<kParamSmall, V>, grid_for(total, res[1], grid_cap), s,
+        return launch_pdl(ddt_exchange_param<kParamSmall, V>, grid_for(total, res[1], grid_cap), s,
                    *reinterpret_cast<const ParamBatch<kParamSmall>*>(src), xa);
     } else if (form == 2) {
         if (!res[2]) res[2] = resident_ctas(ddt_exchange_param<kParamLarge, V>);
-        launch_pdl(ddt_exchange_param<kParamLarge, V>, grid_for(total, res[2], grid_cap), s,
+        return launch_pdl(ddt_exchange_param<kParamLarge, V>, grid_for(total, res[2], grid_cap), s,
                    *reinterpret_cast<const ParamBatch<kParamLarge>*>(src), xa);
     } else {
         if (!res[3]) res[3] = resident_ctas(ddt_exchange_dev<V>);
-        launch_pdl(ddt_exchange_dev<V>, grid_for(total, res[3], grid_cap), s, reinterpret_cast<const uint8_t*>(src),
+        return launch_pdl(ddt_exchange_dev<V>, grid_for(total, res[3], grid_cap), s, reinterpret_cast<const uint8_t*>(src),
                    xa);
     }
 }
@@ -1361,41 +1361,43 @@ static void launch_exchange_v(int form, const void* src, uint32_t total, const X
 int launch_fused_form(int form, int variant, const void* src, uint32_t total_items, void* stream, int grid_cap) {
     if (total_items == 0) return 0;
     cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e = cudaSuccess;
     switch (variant) {
-    case 1: launch_fused_v<1>(form, src, total_items, s, grid_cap); break;
-    case 2: launch_fused_v<2>(form, src, total_items, s, grid_cap); break;
-    case 3: launch_fused_v<3>(form, src, total_items, s, grid_cap); break;
-    case 4: launch_fused_v<4>(form, src, total_items, s, grid_cap); break;
-    case 5: launch_fused_v<5>(form, src, total_items, s, grid_cap); break;
-    case 6: launch_fused_v<6>(form, src, total_items, s, grid_cap); break;
-    case 7: launch_fused_v<7>(form, src, total_items, s, grid_cap); break;
-    case 8: launch_fused_v<8>(form, src, total_items, s, grid_cap); break;
-    case 9: launch_fused_v<9>(form, src, total_items, s, grid_cap); break;
-    case 10: launch_fused_v<10>(form, src, total_items, s, grid_cap); break;
-    default: launch_fused_v<0>(form, src, total_items, s, grid_cap); break;
+    case 1: e = launch_fused_v<1>(form, src, total_items, s, grid_cap); break;
+    case 2: e = launch_fused_v<2>(form, src, total_items, s, grid_cap); break;
+    case 3: e = launch_fused_v<3>(form, src, total_items, s, grid_cap); break;
+    case 4: e = launch_fused_v<4>(form, src, total_items, s, grid_cap); break;
+    case 5: e = launch_fused_v<5>(form, src, total_items, s, grid_cap); break;
+    case 6: e = launch_fused_v<6>(form, src, total_items, s, grid_cap); break;
+    case 7: e = launch_fused_v<7>(form, src, total_items, s, grid_cap); break;
+    case 8: e = launch_fused_v<8>(form, src, total_items, s, grid_cap); break;
+    case 9: e = launch_fused_v<9>(form, src, total_items, s, grid_cap); break;
+    case 10: e = launch_fused_v<10>(form, src, total_items, s, grid_cap); break;
+    default: e = launch_fused_v<0>(form, src, total_items, s, grid_cap); break;
     }
-    return (int)cudaGetLastError();
+    return (int)e;
 }
 
 int launch_exchange_form(int form, int variant, const void* src, uint32_t total_items, const XArgs& xa, void* stream,
                          int grid_cap) {
     if (total_items == 0) return 0;
     cudaStream_t s = (cudaStream_t)stream;
+    cudaError_t e = cudaSuccess;
     switch (variant) {
-    case 1: launch_exchange_v<1>(form, src, total_items, xa, s, grid_cap); break;
-    case 2: launch_exchange_v<2>(form, src, total_items, xa, s, grid_cap); break;
-    case 3: launch_exchange_v<3>(form, src, total_items, xa, s, grid_cap); break;
-    case 4: launch_exchange_v<4>(form, src, total_items, xa, s, grid_cap); break;
-    case 5: launch_exchange_v<5>(form, src, total_items, xa, s, grid_cap); break;
-    case 6: launch_exchange_v<6>(form, src, total_items, xa, s, grid_cap); break;
-    case 7: launch_exchange_v<7>(form, src, total_items, xa, s, grid_cap); break;
-    case 8: launch_exchange_v<8>(form, src, total_items, xa, s, grid_cap); break;
-    case 9: launch_exchange_v<9>(form, src, total_items, xa, s, grid_cap); break;
-    case 11: launch_exchange_v<11>(form, src, total_items, xa, s, grid_cap); break;
-    case 12: launch_exchange_v<12>(form, src, total_items, xa, s, grid_cap); break;
-    default: launch_exchange_v<0>(form, src, total_items, xa, s, grid_cap); break;
+    case 1: e = launch_exchange_v<1>(form, src, total_items, xa, s, grid_cap); break;
+    case 2: e = launch_exchange_v<2>(form, src, total_items, xa, s, grid_cap); break;
+    case 3: e = launch_exchange_v<3>(form, src, total_items, xa, s, grid_cap); break;
+    case 4: e = launch_exchange_v<4>(form, src, total_items, xa, s, grid_cap); break;
+    case 5: e = launch_exchange_v<5>(form, src, total_items, xa, s, grid_cap); break;
+    case 6: e = launch_exchange_v<6>(form, src, total_items, xa, s, grid_cap); break;
+    case 7: e = launch_exchange_v<7>(form, src, total_items, xa, s, grid_cap); break;
+    case 8: e = launch_exchange_v<8>(form, src, total_items, xa, s, grid_cap); break;
+    case 9: e = launch_exchange_v<9>(form, src, total_items, xa, s, grid_cap); break;
+    case 11: e = launch_exchange_v<11>(form, src, total_items, xa, s, grid_cap); break;
+    case 12: e = launch_exchange_v<12>(form, src, total_items, xa, s, grid_cap); break;
+    default: e = launch_exchange_v<0>(form, src, total_items, xa, s, grid_cap); break;
     }
-    return (int)cudaGetLastError();
+    return (int)e;
 }
 
 }  // namespace ddt

@@ -395,6 +395,14 @@ int32_t ddt_flush(ddt_queue_t q) {
     if (q->sticky != DDT_OK) return q->sticky;
     if (q->flushed == q->tail) return 0;
     DeviceGuard g(q->device);
+    // a flushed batch is one-shot (its ring slots, types and table slot are
+    // reclaimed through a completion event): graphs capture persistent plans
+    // (ddt_plan_*), whose tables live as long as the plan, not flushes
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(q->stream, &cs) == cudaSuccess && cs != cudaStreamCaptureStatusNone) {
+        set_error("ddt_flush while the queue's stream is being captured: capture ddt_plan_launch instead");
+        return DDT_ERR_STATE;
+    }
     int64_t moved = gather_pending(q);
     int32_t nflushed = (int32_t)(q->tail - q->flushed);
     if (!q->scratch.descs.empty()) {

@@ -129,3 +129,38 @@ def test_p2p_wait_times_out_instead_of_hanging():
             if p.is_alive():
                 p.kill()
     assert res == {0: True, 1: True}, res
+
+
+def test_flush_refused_during_stream_capture(ddt):
+    """ddt_flush while the queue's stream is being captured returns
+    DDT_ERR_STATE and leaves the requests pending (graphs capture persistent
+    plans); after the capture the same requests flush normally, bit-exact,
+    and later launches in the process are unaffected."""
+    import torch
+    spec = config1_spec()
+    o = oracle.Type(spec)
+    t = ddt.Type.from_spec(spec)
+    src_h = random_bytes(8192, 77)
+    s = torch.cuda.Stream()
+    with torch.cuda.stream(s):
+        q = ddt.Queue()
+        src = torch.from_numpy(src_h).cuda()
+        out = torch.full((o.size,), 0xA5, dtype=torch.uint8, device="cuda")
+        q.pack(t, src, 1, out)
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            with pytest.raises(ddt.DDTError) as ei:
+                q.flush()
+        assert ei.value.code == -2  # DDT_ERR_STATE
+        assert q.flush() == 1       # still pending: flushes after the capture
+        q.wait()
+    assert np.array_equal(out.cpu().numpy(), oracle.pack(o, src_h))
+    q.destroy()
+    q2 = ddt.Queue()                # a later launch reports no stale error
+    out2 = torch.full((o.size,), 0xA5, dtype=torch.uint8, device="cuda")
+    q2.pack(t, src, 1, out2)
+    assert q2.flush() == 1
+    q2.wait()
+    assert np.array_equal(out2.cpu().numpy(), oracle.pack(o, src_h))
+    q2.destroy()

@@ -396,35 +396,42 @@ def test_pdl_launches_respect_stream_order(ddt):
 def test_pdl_read_after_write_inside_a_captured_graph(ddt):
     """Inside ONE captured CUDA graph (programmatic edges between consecutive
     ddt kernels): 30 rounds of [pack A -> packed buffer] -> [unpack of that
-    buffer into B] -> [pack of B's typemap -> second buffer], each kernel
-    reading what its immediate predecessor wrote, so a load scheduled above
-    griddepcontrol.wait would read the previous round's bytes; torch kernels
-    rewrite the source between rounds.  Every round is checked vs the oracle."""
+    buffer into B] -> [pack of B's typemap -> a per-round buffer], each kernel
+    reading what its immediate predecessor wrote (persistent plans launched
+    during capture), so a load scheduled above griddepcontrol.wait would read
+    the previous round's bytes; torch kernels rewrite the source between
+    rounds.  Every round is checked vs the oracle."""
     import torch
     spec = ("vector", 64, 3, 7, ("basic", "double"))
     o = oracle.Type(spec)
     t = ddt.Type.from_spec(spec)
     lo, hi = o.footprint(1)
-    s = torch.cuda.Stream()
     R = 30
+    s = torch.cuda.Stream()
     with torch.cuda.stream(s):
         q = ddt.Queue()
         src = torch.empty(hi, dtype=torch.uint8, device="cuda")
         pk = torch.empty(o.size, dtype=torch.uint8, device="cuda")
         mid = torch.empty(hi, dtype=torch.uint8, device="cuda")
         pk2 = torch.empty((R, o.size), dtype=torch.uint8, device="cuda")
+        q.pack(t, src, 1, pk)
+        p_pack = ddt.Plan(q)
+        q.unpack(t, pk, 1, mid)
+        p_unpack = ddt.Plan(q)
+        p_out = []
+        for k in range(R):
+            q.pack(t, mid, 1, pk2[k])
+            p_out.append(ddt.Plan(q))
+        torch.cuda.synchronize()
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g, stream=s):
             for k in range(R):
                 src.fill_((11 * k + 5) & 0xFF)
                 src[k: k + 16].fill_(k)
                 mid.fill_(0xA5)
-                q.pack(t, src, 1, pk)
-                q.flush()
-                q.unpack(t, pk, 1, mid)
-                q.flush()
-                q.pack(t, mid, 1, pk2[k])
-                q.flush()
+                p_pack.launch()
+                p_unpack.launch()
+                p_out[k].launch()
         g.replay()
     torch.cuda.synchronize()
     got = pk2.cpu().numpy()
@@ -432,6 +439,9 @@ def test_pdl_read_after_write_inside_a_captured_graph(ddt):
         s_host = np.full(hi, (11 * k + 5) & 0xFF, np.uint8)
         s_host[k: k + 16] = k
         assert_bytes_equal(got[k], oracle.pack(o, s_host), f"round {k}")
+    del g
+    for p_ in [p_pack, p_unpack] + p_out:
+        p_.destroy()
     q.destroy()
 
 
